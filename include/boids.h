@@ -1,0 +1,171 @@
+/*
+ * boids.h -- C ABI of libboids.so, the B200 (sm_100a) Boids step.
+ *
+ * One call of boids_step() advances every agent by one OpenSteer Boids update
+ * stage (PAPER.md = the thesis text; "P:<line> sec" cites it):
+ *   1. neighbour search: the up-to-7 nearest agents within the search radius,
+ *      brute force over all agents (Listing 5.2, sec 5.2.1;
+ *      Listing 6.3, sec 6.3.1) or, with search_mode = BOIDS_GRID, over
+ *      a uniform grid that returns the identical sets (future work);
+ *   2. steering: weighted sum of normalised separation, alignment and
+ *      cohesion over those neighbours (Listings 5.1, 5.3-5.5);
+ *   3. modification substage: clamp force, integrate velocity and position,
+ *      regenerate the local space, wrap around the world sphere (P:345,
+ *      P:418 sec 5.3, sec 6.2.3).
+ * The update is synchronous: all of S(t+1) is computed from S(t) (the two
+ * substages of P:418 / the two kernels of P:440).  Exact arithmetic contract:
+ * DESIGN.md Appendix A; parameter readings: DESIGN.md Table C1 / Q1-Q17.
+ *
+ * Conventions
+ *   - Every function returns BOIDS_OK (0) or a negative BOIDS_E* code and
+ *     never throws; boids_last_error() gives a thread-local message.
+ *   - Host arrays are AoS float32: pos3/fwd3/up3/side3 are n*3 floats
+ *     (x,y,z per agent), speed is n floats, caller-owned.  A NULL output
+ *     array is skipped.  The device layout is private (SoA float4, DESIGN.md
+ *     "Data layout"); the 4x4 draw matrix of P:502 is (side, up, fwd, pos).
+ *   - The handle owns all device memory.  Device pointers escape only via
+ *     boids_shard_buffers (for the caller's NCCL all-gather).
+ *   - Work is enqueued on the stream set with boids_set_stream (default: the
+ *     legacy default stream) and is asynchronous; launch errors surface at the
+ *     next synchronising call (get_*, set_*, boids_sync).
+ */
+#ifndef BOIDS_H
+#define BOIDS_H
+
+#include <stdint.h>
+
+#if defined(__GNUC__)
+#define BOIDS_API __attribute__((visibility("default")))
+#else
+#define BOIDS_API
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define BOIDS_OK 0
+#define BOIDS_EINVAL (-1) /* bad argument: n < 1, max_neighbors != 7, radius <= 0, NaN param,
+                             dt < 0 or NaN, steps < 0, NULL handle/pointer, wrong call for mode */
+#define BOIDS_ECUDA (-2)  /* CUDA runtime error; message holds cudaGetErrorString */
+#define BOIDS_ENCCL (-3)  /* reserved for the Python binding (torch.distributed failures) */
+#define BOIDS_ENOMEM (-4) /* device or host allocation failed */
+
+#define BOIDS_BRUTE 0 /* O(n^2) scan over all agents, Listing 5.2 */
+#define BOIDS_GRID 1  /* uniform-grid binned search, identical neighbour sets */
+
+#define BOIDS_INIT_OPENSTEER 0 /* positions uniform in the ball of radius init_radius */
+#define BOIDS_INIT_WORLD 1     /* positions uniform in the ball of radius world_radius */
+
+/* Parameters.  Defaults (boids_default_params) are DESIGN.md Table C1; the
+ * thesis prints only k = 7, every other value is a documented reading. */
+typedef struct boids_params {
+  float search_radius;   /* neighbour search radius r; candidate iff d2 < fl(r*r) (Q2). 9.0 */
+  float w_separation;    /* weightA of Listing 5.1. 12 */
+  float w_alignment;     /* weightB. 8 */
+  float w_cohesion;      /* weightC. 8 */
+  float max_force;       /* steering vector length clamp. 27 */
+  float max_speed;       /* speed clamp. 9 */
+  float mass;            /* a = F / mass (length of the steering vector = acceleration). 1 */
+  float world_radius;    /* spherical world radius R. 50 */
+  float init_radius;     /* ball radius of BOIDS_INIT_OPENSTEER. 20 */
+  float init_speed_frac; /* initial speed = init_speed_frac * max_speed. 0.3 */
+  int32_t max_neighbors; /* must be 7 */
+  int32_t search_mode;   /* BOIDS_BRUTE or BOIDS_GRID */
+  int32_t init_mode;     /* BOIDS_INIT_OPENSTEER or BOIDS_INIT_WORLD */
+} boids_params;
+
+typedef struct boids_ctx boids_ctx; /* opaque handle */
+
+/* Read-only description of a handle (boids_info). */
+typedef struct boids_info_t {
+  int64_t n;         /* total agents */
+  int64_t lo, hi;    /* agents [lo, hi) are owned (updated) by this handle */
+  int64_t slice;     /* padded per-rank slice m (multiple of 256); agent j lives in slice j / m */
+  int32_t rank, world;
+  int32_t kernel;    /* brute-force kernel variant in use (BOIDS_KERNEL_*) */
+  int32_t cluster;   /* candidate split (CTAs per cluster) of the fused kernel */
+  int64_t launches;  /* number of kernels this handle has launched so far */
+} boids_info_t;
+
+#define BOIDS_KERNEL_FUSED 0  /* default: one fused search+steer+modify kernel per step */
+#define BOIDS_KERNEL_SIMPLE 1 /* two kernels: tiled search -> neighbour lists -> update */
+
+/* Options for boids_set_option. */
+#define BOIDS_OPT_RECORD_STEERING 1 /* 1: keep the last step's steering vectors (boids_get_steering) */
+#define BOIDS_OPT_KERNEL 2          /* BOIDS_KERNEL_* */
+#define BOIDS_OPT_PROFILE 3         /* 1: bracket each kernel launch with CUDA events (boids_get_profile) */
+#define BOIDS_OPT_CLUSTER 4         /* 0 = automatic, else force the fused kernel's cluster size (1..16) */
+
+BOIDS_API void boids_default_params(boids_params* out);
+
+/* Allocate and initialise n agents from (params, seed) per DESIGN.md Appendix B.
+ * Returns BOIDS_EINVAL for bad params, BOIDS_ENOMEM / BOIDS_ECUDA on failure.
+ * The initial state is a pure function of (n, params, seed). */
+BOIDS_API int boids_create(int64_t n, const boids_params* p, uint64_t seed, boids_ctx** out);
+
+/* Like boids_create, but this handle owns agents [rank*m, min((rank+1)*m, n)) of an
+ * n-agent flock split over `world` ranks (m = boids_info.slice).  The caller
+ * exchanges positions between ranks (all-gather of the send slices, see
+ * boids_shard_buffers) before every boids_step_shard.  world == 1 is allowed. */
+BOIDS_API int boids_create_shard(int64_t n, const boids_params* p, uint64_t seed, int32_t rank,
+                       int32_t world, boids_ctx** out);
+
+/* Enqueue all later work on `cuda_stream` (a cudaStream_t; NULL = legacy default). */
+BOIDS_API int boids_set_stream(boids_ctx* ctx, void* cuda_stream);
+
+BOIDS_API int boids_set_option(boids_ctx* ctx, int32_t option, int64_t value);
+
+/* Advance `steps` synchronous steps of length dt (single-rank handles only).
+ * steps = 0 is a no-op; dt = 0 computes steering but leaves positions unchanged.
+ * Asynchronous on the handle's stream. */
+BOIDS_API int boids_step(boids_ctx* ctx, float dt, int32_t steps);
+
+/* One step of a shard handle: reads the full gathered (pos, fwd) buffer, writes
+ * this rank's new slice into the send buffer.  Asynchronous. */
+BOIDS_API int boids_step_shard(boids_ctx* ctx, float dt);
+
+/* Device buffers of a shard handle, for the caller's all-gather:
+ *   *send: this rank's slice, 2*m float4 = [pos4(m) | fwd4(m)], *slice_bytes bytes;
+ *   *full: world * (*slice_bytes) bytes, rank g's slice at byte offset g * (*slice_bytes).
+ * all_gather(full <- send) must complete (stream-ordered) before boids_step_shard. */
+BOIDS_API int boids_shard_buffers(boids_ctx* ctx, void** send, void** full, int64_t* slice_bytes);
+
+/* Copy the owned agents' state to host AoS arrays (count = hi - lo).  Synchronises. */
+BOIDS_API int boids_get_state(boids_ctx* ctx, float* pos3, float* fwd3, float* up3, float* side3,
+                    float* speed);
+
+/* Overwrite the owned agents' state from host AoS arrays (count = hi - lo).
+ * side is recomputed by the next step; warm-start neighbour data is invalidated.
+ * pos3, fwd3, up3, speed must be non-NULL; side3 may be NULL (then zero).  Synchronises. */
+BOIDS_API int boids_set_state(boids_ctx* ctx, const float* pos3, const float* fwd3, const float* up3,
+                    const float* side3, const float* speed);
+
+/* Neighbour lists of the last step for the owned agents: idx7 = count*7 int32,
+ * ascending by (d2, index), -1 padded; cnt = count int32.  Synchronises.
+ * Before the first step cnt is 0 everywhere. */
+BOIDS_API int boids_get_neighbors(boids_ctx* ctx, int32_t* idx7, int32_t* cnt);
+
+/* Steering vectors F (before the max_force clamp) of the last step, count*3 floats.
+ * Requires BOIDS_OPT_RECORD_STEERING = 1 before that step (else BOIDS_EINVAL). */
+BOIDS_API int boids_get_steering(boids_ctx* ctx, float* force3);
+
+/* Wait for all enqueued work; returns the first pending CUDA error. */
+BOIDS_API int boids_sync(boids_ctx* ctx);
+
+BOIDS_API int boids_info(boids_ctx* ctx, boids_info_t* out);
+
+/* Accumulated kernel time (ms) and launch count per kernel class since the last
+ * reset, measured with CUDA events on the handle's stream (BOIDS_OPT_PROFILE).
+ * Classes: 0 fused/search, 1 update, 2 binning, 3 grid search.  Synchronises. */
+#define BOIDS_PROF_CLASSES 4
+BOIDS_API int boids_get_profile(boids_ctx* ctx, double* ms, int64_t* launches, int32_t reset);
+
+BOIDS_API void boids_destroy(boids_ctx* ctx);
+
+BOIDS_API const char* boids_last_error(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* BOIDS_H */

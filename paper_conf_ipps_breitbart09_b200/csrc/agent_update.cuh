@@ -1,0 +1,63 @@
+// agent_update.cuh -- steering (Listings 5.1, 5.3-5.5) and the modification
+// substage (Q10-Q13) for ONE agent, given
+// its neighbour list.  Shared by the standalone update kernel and the fused
+// epilogue.  Appendix A arithmetic (device_math.cuh).
+#pragma once
+#include "device_math.cuh"
+#include "internal.h"
+
+namespace boids {
+
+// Steering vector of agent g from its <=7 neighbours (in key order, Q8).
+__device__ __forceinline__ V3 steer_agent(const StepArgs& a, V3 me, V3 fme, const int* nb,
+                                          int cnt) {
+  V3 sep = v3(0.f, 0.f, 0.f), coh = v3(0.f, 0.f, 0.f), ali = v3(0.f, 0.f, 0.f);
+#pragma unroll
+  for (int k = 0; k < 7; ++k) {
+    if (k >= cnt) break;
+    int64_t j = nb[k];
+    float4 pj = __ldg(pos_of(a.full, a.m, j));
+    float4 fj = __ldg(fwd_of(a.full, a.m, j));
+    V3 o = sub(v3(pj), me);  // A.position - me.position (Listing 5.3 line 7)
+    float L = len(o);
+    if (L > 0.0f) sep = sub(sep, divs(divs(o, L), L));  // 1/d fall-off (Listing 5.3 line 10)
+    coh = add(coh, o);                                  // Listing 5.4 line 8
+    ali = add(ali, v3(fj));                             // Listing 5.5 line 7
+  }
+  ali = sub(ali, scale(fme, (float)cnt));  // Listing 5.5 line 10
+  V3 sw = scale(normalize(sep), a.p.w_separation);
+  V3 aw = scale(normalize(ali), a.p.w_alignment);
+  V3 cw = scale(normalize(coh), a.p.w_cohesion);
+  return add(add(sw, aw), cw);  // Listing 5.1 line 5
+}
+
+// Modification substage for local agent i (global g = lo + i); writes the new state.
+__device__ __forceinline__ void modify_agent(const StepArgs& a, int64_t i, V3 pos, float4 f4, V3 F) {
+  const boids_params& p = a.p;
+  V3 f = v3(f4);
+  float speed = f4.w;
+  float4 u4 = a.up4[i];
+  float4 s4 = a.side4[i];
+  V3 u = v3(u4), s = v3(s4);
+  V3 Fc = trunc_len(F, p.max_force);
+  V3 acc = divs(Fc, p.mass);
+  V3 v = scale(f, speed);
+  V3 v1 = add(v, scale(acc, a.dt));
+  V3 v2 = trunc_len(v1, p.max_speed);
+  float sp = len(v2);
+  V3 p1 = add(pos, scale(v2, a.dt));
+  if (sp > 0.0f) {
+    f = divs(v2, sp);
+    s = normalize(cross(f, u));
+    u = cross(s, f);
+  }
+  float L = len(p1);
+  if (L > p.world_radius) p1 = add(p1, scale(scale(divs(p1, L), p.world_radius), -2.0f));
+  a.out[i] = make_float4(p1.x, p1.y, p1.z, 0.0f);
+  a.out[a.m + i] = make_float4(f.x, f.y, f.z, sp);
+  a.up4[i] = make_float4(u.x, u.y, u.z, 0.0f);
+  a.side4[i] = make_float4(s.x, s.y, s.z, 0.0f);
+  if (a.force4) a.force4[i] = make_float4(F.x, F.y, F.z, 0.0f);
+}
+
+}  // namespace boids

@@ -1,0 +1,488 @@
+// api.cu -- the C ABI of include/boids.h: handles, buffers, validation, the step
+// loop and host<->device state transfer.  No exception crosses the ABI.
+#include <cmath>
+#include <cstring>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "internal.h"
+
+using namespace boids;
+
+namespace {
+
+thread_local std::string g_err;
+
+int fail(int code, const std::string& msg) {
+  g_err = msg;
+  return code;
+}
+
+#define CK(expr)                                                                  \
+  do {                                                                            \
+    cudaError_t e_ = (expr);                                                      \
+    if (e_ != cudaSuccess) {                                                      \
+      (void)cudaGetLastError();                                                   \
+      return fail(e_ == cudaErrorMemoryAllocation ? BOIDS_ENOMEM : BOIDS_ECUDA,   \
+                  std::string(#expr) + ": " + cudaGetErrorString(e_));            \
+    }                                                                             \
+  } while (0)
+
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    if (cudaGetDevice(&prev) == cudaSuccess && prev != dev) cudaSetDevice(dev);
+    else prev = -1;
+  }
+  ~DeviceGuard() {
+    if (prev >= 0) cudaSetDevice(prev);
+  }
+};
+
+}  // namespace
+
+struct boids_ctx {
+  int64_t n = 0, m = 0, lo = 0, hi = 0, nloc = 0;
+  int32_t rank = 0, world = 1;
+  bool shard = false;
+  boids_params p{};
+  int dev = 0, sm_count = 148;
+  cudaStream_t stream = nullptr;
+  // !shard: buf[0], buf[1] = ping-pong full buffers (2m float4 each), current = buf[cur].
+  //  shard: buf[0] = full gathered buffer (world*2m), buf[1] = this rank's send slice (2m).
+  float4* buf[2] = {nullptr, nullptr};
+  int cur = 0;
+  float4 *up4 = nullptr, *side4 = nullptr, *force4 = nullptr;
+  int32_t *nbr = nullptr, *cnt = nullptr;
+  bool warm = false;
+  bool record_steering = false, steering_valid = false;
+  int kernel = BOIDS_KERNEL_FUSED;
+  int cluster_opt = 0;
+  bool profile = false;
+  int64_t launches = 0;
+  struct Rec {
+    int cls;
+    cudaEvent_t a, b;
+  };
+  std::vector<Rec> recs;
+  std::vector<cudaEvent_t> pool;
+  double prof_ms[BOIDS_PROF_CLASSES] = {0, 0, 0, 0};
+  int64_t prof_n[BOIDS_PROF_CLASSES] = {0, 0, 0, 0};
+
+  float4* local() const { return shard ? buf[1] : buf[cur]; }
+};
+
+namespace {
+
+bool finite(float x) { return std::isfinite(x); }
+
+int validate(const boids_params* p) {
+  if (!p) return fail(BOIDS_EINVAL, "params is NULL");
+  if (p->max_neighbors != 7) return fail(BOIDS_EINVAL, "max_neighbors must be 7 (P:364)");
+  if (!finite(p->search_radius) || p->search_radius <= 0.f)
+    return fail(BOIDS_EINVAL, "search_radius must be finite and > 0");
+  if (!finite(p->w_separation) || !finite(p->w_alignment) || !finite(p->w_cohesion))
+    return fail(BOIDS_EINVAL, "weights must be finite");
+  if (!finite(p->max_force) || p->max_force < 0.f) return fail(BOIDS_EINVAL, "max_force must be >= 0");
+  if (!finite(p->max_speed) || p->max_speed < 0.f) return fail(BOIDS_EINVAL, "max_speed must be >= 0");
+  if (!finite(p->mass) || p->mass <= 0.f) return fail(BOIDS_EINVAL, "mass must be > 0");
+  if (!finite(p->world_radius) || p->world_radius <= 0.f)
+    return fail(BOIDS_EINVAL, "world_radius must be > 0");
+  if (!finite(p->init_radius) || p->init_radius <= 0.f)
+    return fail(BOIDS_EINVAL, "init_radius must be > 0");
+  if (!finite(p->init_speed_frac) || p->init_speed_frac < 0.f)
+    return fail(BOIDS_EINVAL, "init_speed_frac must be >= 0");
+  if (p->search_mode != BOIDS_BRUTE && p->search_mode != BOIDS_GRID)
+    return fail(BOIDS_EINVAL, "search_mode must be BOIDS_BRUTE or BOIDS_GRID");
+  if (p->init_mode != BOIDS_INIT_OPENSTEER && p->init_mode != BOIDS_INIT_WORLD)
+    return fail(BOIDS_EINVAL, "init_mode must be BOIDS_INIT_OPENSTEER or BOIDS_INIT_WORLD");
+  return BOIDS_OK;
+}
+
+void free_ctx(boids_ctx* c) {
+  if (!c) return;
+  DeviceGuard g(c->dev);
+  for (float4* b : c->buf) cudaFree(b);
+  cudaFree(c->up4);
+  cudaFree(c->side4);
+  cudaFree(c->force4);
+  cudaFree(c->nbr);
+  cudaFree(c->cnt);
+  for (auto& r : c->recs) {
+    cudaEventDestroy(r.a);
+    cudaEventDestroy(r.b);
+  }
+  for (auto e : c->pool) cudaEventDestroy(e);
+  delete c;
+}
+
+cudaEvent_t get_event(boids_ctx* c) {
+  if (!c->pool.empty()) {
+    cudaEvent_t e = c->pool.back();
+    c->pool.pop_back();
+    return e;
+  }
+  cudaEvent_t e = nullptr;
+  cudaEventCreate(&e);
+  return e;
+}
+
+// Launch wrapper: counts launches and, when profiling, brackets with events.
+template <class F>
+int launch(boids_ctx* c, int cls, F&& f) {
+  cudaEvent_t a = nullptr, b = nullptr;
+  if (c->profile) {
+    a = get_event(c);
+    b = get_event(c);
+    CK(cudaEventRecord(a, c->stream));
+  }
+  CK(f());
+  c->launches++;
+  if (c->profile) {
+    CK(cudaEventRecord(b, c->stream));
+    c->recs.push_back({cls, a, b});
+  }
+  return BOIDS_OK;
+}
+
+int create_impl(int64_t n, const boids_params* p, uint64_t seed, int32_t rank, int32_t world,
+                bool shard, boids_ctx** out) {
+  if (!out) return fail(BOIDS_EINVAL, "out is NULL");
+  *out = nullptr;
+  if (n < 1) return fail(BOIDS_EINVAL, "n must be >= 1");
+  if (n > (int64_t)0x7FFFFFFF) return fail(BOIDS_EINVAL, "n must fit in int32 (neighbour indices)");
+  if (world < 1 || rank < 0 || rank >= world) return fail(BOIDS_EINVAL, "bad rank/world");
+  int rc = validate(p);
+  if (rc) return rc;
+  boids_ctx* c = new (std::nothrow) boids_ctx();
+  if (!c) return fail(BOIDS_ENOMEM, "host allocation failed");
+  c->n = n;
+  c->rank = rank;
+  c->world = world;
+  c->shard = shard;
+  c->p = *p;
+  cudaGetDevice(&c->dev);
+  cudaDeviceGetAttribute(&c->sm_count, cudaDevAttrMultiProcessorCount, c->dev);
+  int64_t per = (n + world - 1) / world;
+  c->m = (per + TILE - 1) / TILE * TILE;
+  c->lo = std::min<int64_t>((int64_t)rank * c->m, n);
+  c->hi = std::min<int64_t>((int64_t)(rank + 1) * c->m, n);
+  c->nloc = c->hi - c->lo;
+  int64_t m = c->m;
+  auto alloc = [&](void** ptr, size_t bytes) -> int {
+    cudaError_t e = cudaMalloc(ptr, bytes);
+    if (e != cudaSuccess) {
+      (void)cudaGetLastError();
+      return fail(BOIDS_ENOMEM, std::string("cudaMalloc: ") + cudaGetErrorString(e));
+    }
+    return BOIDS_OK;
+  };
+  size_t seg = (size_t)2 * m * sizeof(float4);
+  if ((rc = alloc((void**)&c->buf[0], shard ? seg * world : seg)) ||
+      (rc = alloc((void**)&c->buf[1], seg)) ||
+      (rc = alloc((void**)&c->up4, m * sizeof(float4))) ||
+      (rc = alloc((void**)&c->side4, m * sizeof(float4))) ||
+      (rc = alloc((void**)&c->nbr, m * 7 * sizeof(int32_t))) ||
+      (rc = alloc((void**)&c->cnt, m * sizeof(int32_t)))) {
+    free_ctx(c);
+    return rc;
+  }
+  cudaStream_t s = c->stream;
+  cudaError_t e = cudaSuccess;
+  // phantoms in every segment of every buffer; then the owned agents
+  if (e == cudaSuccess) e = cudaMemsetAsync(c->buf[0], 0, shard ? seg * world : seg, s);
+  if (e == cudaSuccess) e = cudaMemsetAsync(c->buf[1], 0, seg, s);
+  if (e == cudaSuccess) e = cudaMemsetAsync(c->cnt, 0, m * sizeof(int32_t), s);
+  if (e == cudaSuccess) e = cudaMemsetAsync(c->nbr, 0xFF, m * 7 * sizeof(int32_t), s);
+  if (e == cudaSuccess) e = cudaMemsetAsync(c->up4, 0, m * sizeof(float4), s);
+  if (e == cudaSuccess) e = cudaMemsetAsync(c->side4, 0, m * sizeof(float4), s);
+  if (e == cudaSuccess)
+    e = launch_fill_phantoms(c->buf[0], m, shard ? 0 : c->nloc, shard ? world : 1, s);
+  if (e == cudaSuccess) e = launch_fill_phantoms(c->buf[1], m, c->nloc, 1, s);
+  if (e == cudaSuccess) e = launch_init(c->local(), c->up4, c->side4, m, c->lo, c->nloc, c->p, seed, s);
+  if (e == cudaSuccess && !shard) e = cudaMemcpyAsync(c->buf[1], c->buf[0], seg, cudaMemcpyDeviceToDevice, s);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+  if (e != cudaSuccess) {
+    (void)cudaGetLastError();
+    free_ctx(c);
+    return fail(BOIDS_ECUDA, std::string("create: ") + cudaGetErrorString(e));
+  }
+  *out = c;
+  return BOIDS_OK;
+}
+
+StepArgs make_args(boids_ctx* c, float dt) {
+  StepArgs a;
+  a.full = c->shard ? c->buf[0] : c->buf[c->cur];
+  a.out = c->shard ? c->buf[1] : c->buf[c->cur ^ 1];
+  a.up4 = c->up4;
+  a.side4 = c->side4;
+  a.force4 = c->record_steering ? c->force4 : nullptr;
+  a.nbr = c->nbr;
+  a.cnt = c->cnt;
+  a.n = c->n;
+  a.m = c->m;
+  a.lo = c->lo;
+  a.nloc = c->nloc;
+  a.world = c->shard ? c->world : 1;
+  a.warm = c->warm ? 1 : 0;
+  a.dt = dt;
+  a.p = c->p;
+  return a;
+}
+
+int one_step(boids_ctx* c, float dt) {
+  StepArgs a = make_args(c, dt);
+  int rc;
+  if (c->kernel == BOIDS_KERNEL_SIMPLE) {
+    if ((rc = launch(c, 0, [&] { return launch_search_simple(a, c->stream); }))) return rc;
+    if ((rc = launch(c, 1, [&] { return launch_update(a, c->stream); }))) return rc;
+  } else {
+    int cl = c->cluster_opt;
+    if ((rc = launch(c, 0, [&] { return launch_fused(a, cl, c->stream); }))) return rc;
+  }
+  if (!c->shard) c->cur ^= 1;
+  c->warm = true;
+  c->steering_valid = c->record_steering;
+  return BOIDS_OK;
+}
+
+int check_dt(float dt) {
+  if (!std::isfinite(dt) || dt < 0.f) return fail(BOIDS_EINVAL, "dt must be finite and >= 0");
+  return BOIDS_OK;
+}
+
+void to_aos(const std::vector<float4>& v, int64_t count, float* out, bool w) {
+  for (int64_t i = 0; i < count; ++i) {
+    if (w) {
+      out[i] = v[i].w;
+    } else {
+      out[3 * i] = v[i].x;
+      out[3 * i + 1] = v[i].y;
+      out[3 * i + 2] = v[i].z;
+    }
+  }
+}
+
+}  // namespace
+
+extern "C" {
+
+BOIDS_API void boids_default_params(boids_params* out) {
+  if (!out) return;
+  out->search_radius = 9.0f;
+  out->w_separation = 12.0f;
+  out->w_alignment = 8.0f;
+  out->w_cohesion = 8.0f;
+  out->max_force = 27.0f;
+  out->max_speed = 9.0f;
+  out->mass = 1.0f;
+  out->world_radius = 50.0f;
+  out->init_radius = 20.0f;
+  out->init_speed_frac = 0.3f;
+  out->max_neighbors = 7;
+  out->search_mode = BOIDS_BRUTE;
+  out->init_mode = BOIDS_INIT_OPENSTEER;
+}
+
+BOIDS_API int boids_create(int64_t n, const boids_params* p, uint64_t seed, boids_ctx** out) {
+  return create_impl(n, p, seed, 0, 1, false, out);
+}
+
+BOIDS_API int boids_create_shard(int64_t n, const boids_params* p, uint64_t seed, int32_t rank,
+                       int32_t world, boids_ctx** out) {
+  return create_impl(n, p, seed, rank, world, true, out);
+}
+
+BOIDS_API int boids_set_stream(boids_ctx* c, void* stream) {
+  if (!c) return fail(BOIDS_EINVAL, "NULL handle");
+  c->stream = (cudaStream_t)stream;
+  return BOIDS_OK;
+}
+
+BOIDS_API int boids_set_option(boids_ctx* c, int32_t opt, int64_t v) {
+  if (!c) return fail(BOIDS_EINVAL, "NULL handle");
+  DeviceGuard g(c->dev);
+  switch (opt) {
+    case BOIDS_OPT_RECORD_STEERING:
+      if (v && !c->force4) CK(cudaMalloc((void**)&c->force4, c->m * sizeof(float4)));
+      c->record_steering = v != 0;
+      return BOIDS_OK;
+    case BOIDS_OPT_KERNEL:
+      if (v != BOIDS_KERNEL_FUSED && v != BOIDS_KERNEL_SIMPLE) return fail(BOIDS_EINVAL, "bad kernel");
+      c->kernel = (int)v;
+      return BOIDS_OK;
+    case BOIDS_OPT_PROFILE:
+      c->profile = v != 0;
+      return BOIDS_OK;
+    case BOIDS_OPT_CLUSTER:
+      if (v < 0 || v > 16 || (v & (v - 1))) return fail(BOIDS_EINVAL, "cluster must be 0 or a power of two <= 16");
+      c->cluster_opt = (int)v;
+      return BOIDS_OK;
+    default:
+      return fail(BOIDS_EINVAL, "unknown option");
+  }
+}
+
+BOIDS_API int boids_step(boids_ctx* c, float dt, int32_t steps) {
+  if (!c) return fail(BOIDS_EINVAL, "NULL handle");
+  if (c->shard) return fail(BOIDS_EINVAL, "shard handle: use boids_step_shard after the all-gather");
+  int rc = check_dt(dt);
+  if (rc) return rc;
+  if (steps < 0) return fail(BOIDS_EINVAL, "steps must be >= 0");
+  DeviceGuard g(c->dev);
+  for (int32_t t = 0; t < steps; ++t)
+    if ((rc = one_step(c, dt))) return rc;
+  return BOIDS_OK;
+}
+
+BOIDS_API int boids_step_shard(boids_ctx* c, float dt) {
+  if (!c) return fail(BOIDS_EINVAL, "NULL handle");
+  if (!c->shard) return fail(BOIDS_EINVAL, "not a shard handle");
+  int rc = check_dt(dt);
+  if (rc) return rc;
+  DeviceGuard g(c->dev);
+  return one_step(c, dt);
+}
+
+BOIDS_API int boids_shard_buffers(boids_ctx* c, void** send, void** full, int64_t* slice_bytes) {
+  if (!c) return fail(BOIDS_EINVAL, "NULL handle");
+  if (!c->shard) return fail(BOIDS_EINVAL, "not a shard handle");
+  if (send) *send = c->buf[1];
+  if (full) *full = c->buf[0];
+  if (slice_bytes) *slice_bytes = 2 * c->m * (int64_t)sizeof(float4);
+  return BOIDS_OK;
+}
+
+BOIDS_API int boids_get_state(boids_ctx* c, float* pos3, float* fwd3, float* up3, float* side3, float* speed) {
+  if (!c) return fail(BOIDS_EINVAL, "NULL handle");
+  DeviceGuard g(c->dev);
+  int64_t k = c->nloc, m = c->m;
+  std::vector<float4> h((size_t)k);
+  const float4* L = c->local();
+  if (pos3) {
+    CK(cudaMemcpyAsync(h.data(), L, k * sizeof(float4), cudaMemcpyDeviceToHost, c->stream));
+    CK(cudaStreamSynchronize(c->stream));
+    to_aos(h, k, pos3, false);
+  }
+  if (fwd3 || speed) {
+    CK(cudaMemcpyAsync(h.data(), L + m, k * sizeof(float4), cudaMemcpyDeviceToHost, c->stream));
+    CK(cudaStreamSynchronize(c->stream));
+    if (fwd3) to_aos(h, k, fwd3, false);
+    if (speed) to_aos(h, k, speed, true);
+  }
+  if (up3) {
+    CK(cudaMemcpyAsync(h.data(), c->up4, k * sizeof(float4), cudaMemcpyDeviceToHost, c->stream));
+    CK(cudaStreamSynchronize(c->stream));
+    to_aos(h, k, up3, false);
+  }
+  if (side3) {
+    CK(cudaMemcpyAsync(h.data(), c->side4, k * sizeof(float4), cudaMemcpyDeviceToHost, c->stream));
+    CK(cudaStreamSynchronize(c->stream));
+    to_aos(h, k, side3, false);
+  }
+  CK(cudaStreamSynchronize(c->stream));
+  return BOIDS_OK;
+}
+
+BOIDS_API int boids_set_state(boids_ctx* c, const float* pos3, const float* fwd3, const float* up3,
+                    const float* side3, const float* speed) {
+  if (!c) return fail(BOIDS_EINVAL, "NULL handle");
+  if (!pos3 || !fwd3 || !up3 || !speed) return fail(BOIDS_EINVAL, "pos3, fwd3, up3, speed required");
+  DeviceGuard g(c->dev);
+  int64_t k = c->nloc, m = c->m;
+  std::vector<float4> hp((size_t)k), hf((size_t)k), hu((size_t)k), hs((size_t)k);
+  for (int64_t i = 0; i < k; ++i) {
+    hp[i] = make_float4(pos3[3 * i], pos3[3 * i + 1], pos3[3 * i + 2], 0.f);
+    hf[i] = make_float4(fwd3[3 * i], fwd3[3 * i + 1], fwd3[3 * i + 2], speed[i]);
+    hu[i] = make_float4(up3[3 * i], up3[3 * i + 1], up3[3 * i + 2], 0.f);
+    hs[i] = side3 ? make_float4(side3[3 * i], side3[3 * i + 1], side3[3 * i + 2], 0.f)
+                  : make_float4(0.f, 0.f, 0.f, 0.f);
+  }
+  float4* L = c->local();
+  CK(cudaMemcpyAsync(L, hp.data(), k * sizeof(float4), cudaMemcpyHostToDevice, c->stream));
+  CK(cudaMemcpyAsync(L + m, hf.data(), k * sizeof(float4), cudaMemcpyHostToDevice, c->stream));
+  CK(cudaMemcpyAsync(c->up4, hu.data(), k * sizeof(float4), cudaMemcpyHostToDevice, c->stream));
+  CK(cudaMemcpyAsync(c->side4, hs.data(), k * sizeof(float4), cudaMemcpyHostToDevice, c->stream));
+  CK(cudaMemsetAsync(c->cnt, 0, m * sizeof(int32_t), c->stream));
+  CK(cudaMemsetAsync(c->nbr, 0xFF, m * 7 * sizeof(int32_t), c->stream));
+  CK(cudaStreamSynchronize(c->stream));
+  c->warm = false;
+  c->steering_valid = false;
+  return BOIDS_OK;
+}
+
+BOIDS_API int boids_get_neighbors(boids_ctx* c, int32_t* idx7, int32_t* cnt) {
+  if (!c) return fail(BOIDS_EINVAL, "NULL handle");
+  DeviceGuard g(c->dev);
+  if (idx7) CK(cudaMemcpyAsync(idx7, c->nbr, c->nloc * 7 * sizeof(int32_t), cudaMemcpyDeviceToHost, c->stream));
+  if (cnt) CK(cudaMemcpyAsync(cnt, c->cnt, c->nloc * sizeof(int32_t), cudaMemcpyDeviceToHost, c->stream));
+  CK(cudaStreamSynchronize(c->stream));
+  return BOIDS_OK;
+}
+
+BOIDS_API int boids_get_steering(boids_ctx* c, float* force3) {
+  if (!c) return fail(BOIDS_EINVAL, "NULL handle");
+  if (!c->steering_valid) return fail(BOIDS_EINVAL, "no recorded steering (set BOIDS_OPT_RECORD_STEERING before stepping)");
+  if (!force3) return fail(BOIDS_EINVAL, "force3 is NULL");
+  DeviceGuard g(c->dev);
+  std::vector<float4> h((size_t)c->nloc);
+  CK(cudaMemcpyAsync(h.data(), c->force4, c->nloc * sizeof(float4), cudaMemcpyDeviceToHost, c->stream));
+  CK(cudaStreamSynchronize(c->stream));
+  to_aos(h, c->nloc, force3, false);
+  return BOIDS_OK;
+}
+
+BOIDS_API int boids_sync(boids_ctx* c) {
+  if (!c) return fail(BOIDS_EINVAL, "NULL handle");
+  DeviceGuard g(c->dev);
+  CK(cudaStreamSynchronize(c->stream));
+  CK(cudaGetLastError());
+  return BOIDS_OK;
+}
+
+BOIDS_API int boids_info(boids_ctx* c, boids_info_t* o) {
+  if (!c || !o) return fail(BOIDS_EINVAL, "NULL argument");
+  o->n = c->n;
+  o->lo = c->lo;
+  o->hi = c->hi;
+  o->slice = c->m;
+  o->rank = c->rank;
+  o->world = c->world;
+  o->kernel = c->kernel;
+  o->cluster = c->cluster_opt ? c->cluster_opt
+                              : fused_auto_cluster((int64_t)(c->shard ? c->world : 1) * c->m, c->nloc, c->sm_count);
+  o->launches = c->launches;
+  return BOIDS_OK;
+}
+
+BOIDS_API int boids_get_profile(boids_ctx* c, double* ms, int64_t* launches, int32_t reset) {
+  if (!c) return fail(BOIDS_EINVAL, "NULL handle");
+  DeviceGuard g(c->dev);
+  CK(cudaStreamSynchronize(c->stream));
+  for (auto& r : c->recs) {
+    float t = 0.f;
+    CK(cudaEventElapsedTime(&t, r.a, r.b));
+    c->prof_ms[r.cls] += t;
+    c->prof_n[r.cls] += 1;
+    c->pool.push_back(r.a);
+    c->pool.push_back(r.b);
+  }
+  c->recs.clear();
+  for (int k = 0; k < BOIDS_PROF_CLASSES; ++k) {
+    if (ms) ms[k] = c->prof_ms[k];
+    if (launches) launches[k] = c->prof_n[k];
+    if (reset) {
+      c->prof_ms[k] = 0;
+      c->prof_n[k] = 0;
+    }
+  }
+  return BOIDS_OK;
+}
+
+BOIDS_API void boids_destroy(boids_ctx* c) { free_ctx(c); }
+
+BOIDS_API const char* boids_last_error(void) { return g_err.c_str(); }
+
+}  // extern "C"

@@ -1,0 +1,139 @@
+// k_basic.cu -- initial state, phantom fill, the two-kernel step
+// (tiled search -> neighbour lists; update from lists).
+//
+// The two-kernel step mirrors the thesis's own structure (search kernel with a
+// shared-memory position cache, Listing 6.2; separate modification
+// kernel) and doubles as the standalone HBM-bound update kernel of
+// SURVEY.md B5.  The default step is the fused kernel in k_fused.cu.
+#include "agent_update.cuh"
+
+namespace boids {
+
+// ---------------------------------------------------------------- init ----
+// DESIGN.md Appendix B; agent g's stream depends only on (seed, g).
+__device__ __forceinline__ float draw_coord(uint64_t& s) {
+  s += SM64_GAMMA;
+  uint64_t out = sm64_mix(s);
+  float u = __fmul_rn((float)(uint32_t)(out >> 40), 5.9604644775390625e-08f);  // exact
+  return __fsub_rn(__fmul_rn(u, 2.0f), 1.0f);
+}
+__device__ __forceinline__ V3 draw_ball(uint64_t& s) {
+  for (;;) {
+    float x = draw_coord(s), y = draw_coord(s), z = draw_coord(s);
+    V3 v = v3(x, y, z);
+    if (dot(v, v) < 1.0f) return v;
+  }
+}
+
+__global__ void k_init(float4* out, float4* up4, float4* side4, int64_t m, int64_t lo,
+                       int64_t nloc, boids_params p, uint64_t seed) {
+  int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= nloc) return;
+  uint64_t g = (uint64_t)(lo + i);
+  uint64_t s = sm64(seed ^ sm64(g));
+  float R = p.init_mode == BOIDS_INIT_WORLD ? p.world_radius : p.init_radius;
+  V3 pos = scale(draw_ball(s), R);
+  V3 f = normalize(draw_ball(s));
+  V3 side = normalize(cross(f, v3(0.f, 1.f, 0.f)));
+  V3 up = cross(side, f);
+  float sp = __fmul_rn(p.init_speed_frac, p.max_speed);
+  out[i] = make_float4(pos.x, pos.y, pos.z, 0.f);
+  out[m + i] = make_float4(f.x, f.y, f.z, sp);
+  up4[i] = make_float4(up.x, up.y, up.z, 0.f);
+  side4[i] = make_float4(side.x, side.y, side.z, 0.f);
+}
+
+cudaError_t launch_init(float4* out, float4* up4, float4* side4, int64_t m, int64_t lo,
+                        int64_t nloc, const boids_params& p, uint64_t seed, cudaStream_t s) {
+  if (nloc <= 0) return cudaSuccess;
+  int64_t blocks = (nloc + 255) / 256;
+  k_init<<<(unsigned)blocks, 256, 0, s>>>(out, up4, side4, m, lo, nloc, p, seed);
+  return cudaGetLastError();
+}
+
+// Phantom agents [nloc, m) of each segment: NaN position (d2 = NaN is never < r2), zero fwd.
+__global__ void k_fill_phantoms(float4* base, int64_t m, int64_t nloc, int64_t segments) {
+  int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  int64_t per = m - nloc;
+  if (k >= per * segments) return;
+  int64_t seg = k / per, i = nloc + k % per;
+  float nan = __int_as_float(0x7fc00000);
+  base[seg * 2 * m + i] = make_float4(nan, nan, nan, 0.f);
+  base[seg * 2 * m + m + i] = make_float4(0.f, 0.f, 0.f, 0.f);
+}
+
+cudaError_t launch_fill_phantoms(float4* base, int64_t m, int64_t nloc, int64_t segments,
+                                 cudaStream_t s) {
+  int64_t total = (m - nloc) * segments;
+  if (total <= 0) return cudaSuccess;
+  k_fill_phantoms<<<(unsigned)((total + 255) / 256), 256, 0, s>>>(base, m, nloc, segments);
+  return cudaGetLastError();
+}
+
+// ------------------------------------------------------- simple search ----
+// One thread per owned agent; candidate positions staged through shared memory
+// one TILE at a time (the thesis's version-2 structure, Listing 6.2), register
+// top-7 of (d2, idx) keys.  Candidates are scanned in increasing index order, so
+// the strict d2 < worst test realises the index tie-break of reading Q4.
+__global__ void __launch_bounds__(TILE) k_search_simple(StepArgs a) {
+  __shared__ float4 tile[TILE];
+  int64_t i = (int64_t)blockIdx.x * TILE + threadIdx.x;
+  bool active = i < a.nloc;
+  int64_t g = a.lo + i;
+  float4 me = active ? *pos_of(a.full, a.m, g) : make_float4(0.f, 0.f, 0.f, 0.f);
+  float r2 = __fmul_rn(a.p.search_radius, a.p.search_radius);
+  key_t L[7];
+#pragma unroll
+  for (int s = 0; s < 7; ++s) L[s] = KEY_EMPTY;
+  float lim = r2;
+  int cnt = 0;
+  int64_t total = (int64_t)a.world * a.m;
+  for (int64_t base = 0; base < total; base += TILE) {
+    tile[threadIdx.x] = *pos_of(a.full, a.m, base + threadIdx.x);
+    __syncthreads();
+    for (int k = 0; k < TILE; ++k) {
+      float d2 = dist2(me.x, me.y, me.z, tile[k]);
+      int64_t j = base + k;
+      if (d2 < lim && j != g) {
+        insert7(L, make_key(d2, (int)j));
+        cnt = cnt < 7 ? cnt + 1 : 7;
+        if (cnt == 7) lim = fminf(r2, key_d2(L[6]));
+      }
+    }
+    __syncthreads();
+  }
+  if (!active) return;
+#pragma unroll
+  for (int s = 0; s < 7; ++s) a.nbr[i * 7 + s] = s < cnt ? key_idx(L[s]) : -1;
+  a.cnt[i] = cnt;
+}
+
+cudaError_t launch_search_simple(const StepArgs& a, cudaStream_t s) {
+  if (a.nloc <= 0) return cudaSuccess;
+  k_search_simple<<<(unsigned)((a.nloc + TILE - 1) / TILE), TILE, 0, s>>>(a);
+  return cudaGetLastError();
+}
+
+// -------------------------------------------------------------- update ----
+// Steering + modification from the neighbour lists: one thread per owned agent.
+__global__ void __launch_bounds__(256) k_update(StepArgs a) {
+  int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= a.nloc) return;
+  int64_t g = a.lo + i;
+  float4 p4 = __ldg(pos_of(a.full, a.m, g));
+  float4 f4 = __ldg(fwd_of(a.full, a.m, g));
+  int cnt = a.cnt[i];
+  int nb[7];
+#pragma unroll
+  for (int s = 0; s < 7; ++s) nb[s] = a.nbr[i * 7 + s];
+  V3 F = steer_agent(a, v3(p4), v3(f4), nb, cnt);
+  modify_agent(a, i, v3(p4), f4, F);
+}
+
+cudaError_t launch_update(const StepArgs& a, cudaStream_t s) {
+  if (a.nloc <= 0) return cudaSuccess;
+  k_update<<<(unsigned)((a.nloc + 255) / 256), 256, 0, s>>>(a);
+  return cudaGetLastError();
+}
+
+}  // namespace boids

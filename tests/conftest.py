@@ -24,3 +24,30 @@ def orc():
 
     oracle.build()
     return oracle
+
+
+@pytest.fixture(scope="session")
+def boidslib():
+    """Build (if stale) and load libboids.so -- the CUDA path; no fallback."""
+    from paper_conf_ipps_breitbart09_b200 import abi, build
+
+    build.build()
+    return abi.load()
+
+
+def _has_gpu():
+    try:
+        import torch
+
+        return torch.cuda.is_available()
+    except Exception:
+        return False
+
+
+def pytest_collection_modifyitems(config, items):
+    if _has_gpu():
+        return
+    skip = pytest.mark.skip(reason="no CUDA device here (run with -m gpu under gpurun)")
+    for it in items:
+        if "gpu" in it.keywords:
+            it.add_marker(skip)
