@@ -1,0 +1,327 @@
+#!/usr/bin/env python
+"""Benchmark of the B200 Boids step (one JSON line on rank 0).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload c4] [--impl ours|reference]
+    torchrun --nproc-per-node N --master-addr 127.0.0.1 bench.py --gpus N ...
+
+A "step" is one synchronous Boids update of ALL agents (every SURVEY.md 8(a)
+row: [a1 all-gather at N>1] -> a3 search -> a4 split merge -> a5 steering ->
+a6 modification; a2 binning in grid mode), through the C ABI of libboids.so.
+
+* value      agent-steps/s of the whole job = n * K / max-over-ranks device time,
+             CUDA events on the launching stream, L2 flushed (256 MiB write)
+             before every timed step (the state of every config fits in L2).
+* e2e        the same metric through the public C ABI with HOST buffers: every
+             step boids_set_state (H2D) + step + boids_get_state (D2H), wall clock.
+* roofline   the dominant kernel (the fused search kernel): algorithmic FP32
+             lane-ops per launch (8 per candidate pair) / its mean
+             launch duration (library-side CUDA events on the same stream),
+             against the FP32 SIMT peak 148 SMs x 128 lanes x sm_max_mhz.
+* cpu_baseline  the CPU oracle (oracle/, single thread) on a bounded sample of
+             the same workload: full O(n) search + steer + modify for each sampled
+             agent, extrapolated per agent-step (rank 0, N=1 only).
+* --impl reference  times that oracle alone (the tier's reference arm).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+import workloads as W  # noqa: E402
+
+METRIC = json.load(open(os.path.join(ROOT, "BASELINE.json")))["metric"]
+UNIT = "agent-steps/s"
+LANES_PER_SM = 128
+OPS_PER_PAIR = 8  # 3 sub + 3 mul + 2 add, no FMA
+
+
+def peaks():
+    p = {}
+    path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(path):
+        p = json.load(open(path))
+    return p
+
+
+def env_rank():
+    return int(os.environ.get("RANK", 0)), int(os.environ.get("WORLD_SIZE", 1)), int(os.environ.get("LOCAL_RANK", 0))
+
+
+class ClockSampler:
+    """Samples SM clock + throttle reasons via NVML while the timed region runs."""
+
+    def __init__(self, dev_index: int, period: float = 0.005):
+        self.samples, self.reasons, self.max_mhz = [], set(), None
+        self.period = period
+        self._stop = threading.Event()
+        self._t = None
+        try:
+            import pynvml
+
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(dev_index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+        except Exception:
+            self.nv = None
+
+    _REASONS = {
+        0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap", 0x8: "hw_slowdown",
+        0x10: "sync_boost", 0x20: "sw_thermal_slowdown", 0x40: "hw_thermal_slowdown",
+        0x80: "hw_power_brake_slowdown", 0x100: "display_clock_setting",
+    }
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+                r = self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                for bit, name in self._REASONS.items():
+                    if r & bit and name != "gpu_idle":
+                        self.reasons.add(name)
+            except Exception:
+                pass
+            time.sleep(self.period)
+
+    def __enter__(self):
+        if self.nv:
+            self._t = threading.Thread(target=self._run, daemon=True)
+            self._t.start()
+        return self
+
+    def __exit__(self, *exc):
+        self._stop.set()
+        if self._t:
+            self._t.join()
+
+    def summary(self):
+        if not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons), "samples": 0}
+        return {"sm_mhz": float(np.median(self.samples)), "sm_max_mhz": self.max_mhz,
+                "reasons": sorted(self.reasons), "samples": len(self.samples)}
+
+
+def cpu_oracle_rate(cfg: W.Config, agents: int, seed: int = 1):
+    """Oracle (single thread) on `agents` sampled agents of the config's initial state."""
+    import oracle
+
+    p = oracle.default_params(init_mode=cfg.init_mode, search_mode=cfg.search_mode)
+    s = oracle.init(cfg.n, p, seed=seed)
+    ag = W.sample_agents(cfg.n, agents, seed=seed)
+    t = time.perf_counter()
+    oracle.step_sample(s, ag, float(W.DT), p)
+    dt = time.perf_counter() - t
+    return len(ag) / dt, len(ag), dt
+
+
+def cpu_sample_size(cfg: W.Config, seconds: float) -> int:
+    """Agents per sample for ~`seconds` of oracle work (about 5 ns per candidate pair)."""
+    return int(max(64, min(cfg.n, seconds / (5e-9 * cfg.n))))
+
+
+def run_reference(args, cfg):
+    rank, world, _ = env_rank()
+    if rank != 0:
+        return 0
+    m = cpu_sample_size(cfg, 1.5)
+    for _ in range(args.warmup):
+        cpu_oracle_rate(cfg, max(64, m // 8))
+    times, agents = [], 0
+    for k in range(args.steps):
+        _, agents, dt = cpu_oracle_rate(cfg, m, seed=1)
+        times.append(dt)
+    total = float(np.sum(times))
+    value = agents * args.steps / total
+    sample = (f"{agents} of {cfg.n} agents per step (seeded sample), each a full O(n) search + steer + "
+              f"modify from the config's initial state; {args.steps} steps")
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": total / args.steps * 1e3,
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f32",
+        "data": "synthetic", "config": config_dict(cfg, args.gpus),
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+        "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def config_dict(cfg: W.Config, gpus: int):
+    return {"workload": cfg.name, "desc": cfg.desc, "n": cfg.n,
+            "search": "grid" if cfg.search_mode else "brute",
+            "init": "world_ball_r50" if cfg.init_mode else "opensteer_ball_r20",
+            "parallelism": f"agents sharded by index over {gpus} GPU(s), NCCL all-gather of pos+fwd per step"
+            if gpus > 1 else "single GPU",
+            "dt": float(W.DT), "seed": 1, "l2": "flushed (256 MiB write) before every timed step"}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--workload", default="c4", choices=sorted(W.CONFIGS))
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--cpu-seconds", type=float, default=10.0, help="oracle sample size (seconds of CPU work)")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--kernel", type=int, default=0, help="0 fused (default), 1 two-kernel simple path")
+    args = ap.parse_args()
+    cfg = W.CONFIGS[args.workload]
+    if args.warmup < 3:
+        args.warmup = 3  # timing rule: at least 3 warm-up steps
+    if args.impl == "reference":
+        return run_reference(args, cfg)
+
+    import torch
+
+    rank, world, local = env_rank()
+    if world != args.gpus:
+        args.gpus = world
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+
+        dist.init_process_group("nccl", device_id=dev)
+
+    import paper_conf_ipps_breitbart09_b200 as pk
+    from paper_conf_ipps_breitbart09_b200 import abi
+    from paper_conf_ipps_breitbart09_b200.shard import ShardedFlock
+
+    params = pk.boids_default_params(init_mode=cfg.init_mode, search_mode=cfg.search_mode)
+    dt = float(W.DT)
+    if world > 1:
+        fl = ShardedFlock(cfg.n, params, seed=1, kernel=args.kernel)
+        h = fl.h
+        step = lambda: fl.step(dt, 1)  # noqa: E731
+        nloc = fl.hi - fl.lo
+    else:
+        fl = pk.Flock(cfg.n, params, seed=1, kernel=args.kernel)
+        h = fl.h
+        step = lambda: fl.step(dt, 1)  # noqa: E731
+        nloc = cfg.n
+
+    flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
+    stream = torch.cuda.current_stream()
+
+    def barrier():
+        if dist is not None:
+            dist.barrier()
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+
+    # ---------------- timed region: K steps, L2 flushed before each ----------------
+    abi.boids_set_option(h, abi.BOIDS_OPT_PROFILE, 1)
+    abi.boids_get_profile(h, reset=True)
+    launches0 = abi.boids_info(h).launches
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    barrier()
+    torch.cuda.synchronize()
+    with ClockSampler(local) as clk:
+        for k in range(args.steps):
+            flush.fill_(float(k))
+            ev[k][0].record(stream)
+            step()
+            ev[k][1].record(stream)
+        torch.cuda.synchronize()
+        barrier()
+    launches = abi.boids_info(h).launches - launches0
+    prof = abi.boids_get_profile(h, reset=True)
+    abi.boids_set_option(h, abi.BOIDS_OPT_PROFILE, 0)
+    ms = float(sum(a.elapsed_time(b) for a, b in ev))
+    if dist is not None:
+        t = torch.tensor([ms], device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+    value = cfg.n * args.steps / (ms / 1e3)
+
+    # ---------------- roofline of the dominant kernel ----------------
+    kname = "fused_or_search"
+    k_ms, k_n = prof[kname]
+    k_ms_per = k_ms / max(k_n, 1)
+    pairs_per_launch = float(nloc) * float(cfg.n)
+    achieved = OPS_PER_PAIR * pairs_per_launch / (k_ms_per / 1e3) / 1e12  # T lane-op/s
+    pk_ = peaks()
+    sm_max = float(pk_.get("sm_max_mhz", 1965.0))
+    peak = 148 * LANES_PER_SM * sm_max * 1e6 / 1e12
+    clocks = clk.summary()
+    traffic = None
+    summ = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    if os.path.exists(summ):
+        try:
+            traffic = json.load(open(summ)).get(cfg.name, {}).get("dram_bytes_per_launch")
+        except Exception:
+            traffic = None
+    roofline = {"bound": "alu", "kernel": "k_fused (search+merge+steer+modify)",
+                "achieved": achieved, "peak": peak, "unit": "TFLOP/s", "frac": achieved / peak,
+                "traffic": traffic,
+                "peak_note": f"FP32 SIMT lane-ops: 148 SM x 128 lanes x {sm_max:.0f} MHz "
+                             f"(sm_max_mhz of MEASURED_PEAKS.json; each add/sub/mul counted once, no FMA)",
+                "work_per_launch": f"{OPS_PER_PAIR} lane-ops x {pairs_per_launch:.4g} pairs",
+                "kernel_ms_per_launch": k_ms_per, "kernel_share_of_step": k_ms / ms if ms else None,
+                "frac_at_measured_clock": (achieved / (148 * LANES_PER_SM * clocks["sm_mhz"] * 1e6 / 1e12))
+                if clocks.get("sm_mhz") else None}
+
+    # ---------------- e2e through the C ABI with host buffers ----------------
+    e2e = None
+    st = abi.boids_get_state(h)
+    host = {k: np.ascontiguousarray(v) for k, v in st.items()}
+    h2d = nloc * 4 * 16  # set_state uploads pos4, fwd4 (+speed), up4, side4
+    d2h = nloc * 4 * 16  # get_state downloads pos4, fwd4, up4, side4
+    barrier()
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        abi.boids_set_state(h, host)
+        step()
+        abi.boids_get_state(h, host)
+    t1 = time.perf_counter()
+    e2e_s = t1 - t0
+    if dist is not None:
+        t = torch.tensor([e2e_s], device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        e2e_s = float(t.item())
+    e2e = {"value": cfg.n * args.steps / e2e_s, "unit": UNIT, "h2d_bytes_per_step": h2d * world,
+           "d2h_bytes_per_step": d2h * world,
+           "note": "boids_set_state (host AoS -> device) + step + boids_get_state (device -> host AoS), wall clock"}
+
+    # ---------------- CPU oracle baseline (rank 0, N=1) ----------------
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        m = cpu_sample_size(cfg, args.cpu_seconds)
+        rate, agents, secs = cpu_oracle_rate(cfg, m)
+        cpu = {"value": rate, "unit": UNIT, "cores": 1, "kind": "oracle",
+               "sample": f"{agents} of {cfg.n} agents x 1 step (seeded sample of the config's initial state; "
+                         f"each agent a full O(n) search + steer + modify), {secs:.1f} s single-threaded"}
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": config_dict(cfg, world), "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
+            "gpu_launches": int(launches), "clocks": clocks,
+            "kernel_profile_ms": {k: v[0] for k, v in prof.items() if v[1]},
+            "thesis_context": "thesis v5 GPU (GeForce 8800 GTS) vs CPU (Athlon 64 3700+): ~42x at 4096 agents "
+                              "(PAPER.md P:499, P:465); different hardware and baseline, not comparable",
+        }
+        print(json.dumps(line), flush=True)
+    fl.close()
+    if dist is not None:
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())
