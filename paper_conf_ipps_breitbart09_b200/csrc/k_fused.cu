@@ -5,16 +5,19 @@
 // position cache (Listing 6.2), version 4's recompute-not-cache
 // (P:493), version 5's device-resident modification.  What is new:
 //
-//  * Work unit = (query block of QB = 256 agents, candidate chunk).  A thread
+//  * Work unit = (query block of QB = NT * Q agents, candidate chunk).  A thread
 //    block cluster of K CTAs (K in {1,2,4,8,16}) shares one query block; CTA r
-//    of the cluster scans candidate chunk r of K.  K is chosen so the grid is
-//    close to a whole multiple of the SM count (fused_auto_cluster).
+//    of the cluster scans candidate chunk r of K.  NT (64 or 128 threads) and K
+//    are chosen by plan_launch so the grid is close to a whole multiple of the
+//    SM count with enough warps per SM.
 //  * Candidate positions are streamed global -> shared memory by the TMA bulk
 //    copy engine (cp.async.bulk + mbarrier complete_tx) through a STAGES-deep
 //    ring of 256-candidate tiles; all 4 warps read each candidate with a
 //    broadcast LDS.128.
-//  * Each thread owns Q = 2 queries and keeps two register-resident sorted
-//    top-7 lists of (d2, index) keys (64-bit, reading Q4 total order).
+//  * Each thread owns Q = 4 queries (4 independent distance chains per LDS;
+//    measured 0.87 of the FP32 lane-op peak vs 0.58 for Q = 2) and keeps four
+//    register-resident sorted top-7 lists of (d2, index) keys (64-bit, the
+//    reading-Q4 total order).  Packed FADD2/FMUL2 were measured slower.
 //  * Warm threshold: t0 = max d2 to the previous step's 7 neighbours at the
 //    current positions is an upper bound on the true 7th key, so only
 //    candidates with d2 <= t0 can enter (identical result, far fewer inserts).
@@ -36,13 +39,9 @@ namespace cg = cooperative_groups;
 namespace boids {
 namespace {
 
-constexpr int NT = 128;      // threads per CTA (4 warps), all consumers
-constexpr int Q = 2;         // queries per thread
-constexpr int QB = NT * Q;   // queries per CTA / cluster
-constexpr int CT = 256;      // candidates per tile (4 KB)
-constexpr int STAGES = 4;    // TMA ring depth
-constexpr int U = 4;         // candidates per vote
-static_assert(CT % U == 0, "tile");
+constexpr int Q = 4;        // queries per thread (4 independent distance chains)
+constexpr int CT = 256;     // candidates per tile (4 KB)
+constexpr int STAGES = 4;   // TMA ring depth
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
   return (uint32_t)__cvta_generic_to_shared(p);
@@ -75,15 +74,24 @@ __device__ __forceinline__ void tma_load_1d(void* dst, const void* src, uint32_t
       "l"(src), "r"(bytes), "r"(smem_u32(bar))
       : "memory");
 }
-__device__ __forceinline__ void consumer_bar() { asm volatile("bar.sync 1, %0;" ::"n"(NT) : "memory"); }
+__device__ __forceinline__ void cluster_arrive() {
+  asm volatile("barrier.cluster.arrive.release.aligned;" ::: "memory");
+}
+__device__ __forceinline__ void cluster_wait() {
+  asm volatile("barrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
 
+template <int NT>
 struct __align__(16) Smem {
-  float4 tile[STAGES][CT];  // 16 KB candidate ring; reused for the partial lists
-  float t0[QB];             // warm thresholds of this CTA's share of the queries
+  static constexpr int QB = NT * Q;
+  static constexpr int RING = STAGES * CT * (int)sizeof(float4);
+  static constexpr int LISTS = 7 * QB * (int)sizeof(key_t);
+  // candidate ring during the scan, then the partial lists [7][QB] (k-major) for the merge
+  __align__(128) unsigned char buf[RING > LISTS ? RING : LISTS];
+  float t0[QB];  // warm thresholds (each cluster rank fills its share)
   uint64_t full[STAGES];
   uint64_t empty[STAGES];
 };
-static_assert(sizeof(key_t) * 7 * QB <= sizeof(float4) * STAGES * CT, "lists fit in the ring");
 
 __device__ __forceinline__ const float4* tile_src(const StepArgs& a, int64_t tile) {
   return pos_of(a.full, a.m, tile * CT);  // m % CT == 0: a tile never straddles a slice
@@ -103,15 +111,34 @@ __device__ __forceinline__ float warm_t0(const StepArgs& a, int64_t ql) {
   return t;
 }
 
-template <int K>
+// Final list of local query qi -> neighbour list, count, steering, modification.
+__device__ __forceinline__ void finish_query(const StepArgs& a, int64_t qi, const key_t (&A)[7]) {
+  if (qi >= a.nloc) return;
+  int nb[7], cnt = 0;
+#pragma unroll
+  for (int s = 0; s < 7; ++s) {
+    nb[s] = A[s] == KEY_EMPTY ? -1 : key_idx(A[s]);
+    cnt += A[s] == KEY_EMPTY ? 0 : 1;
+  }
+#pragma unroll
+  for (int s = 0; s < 7; ++s) a.nbr[qi * 7 + s] = nb[s];
+  a.cnt[qi] = cnt;
+  float4 p4 = __ldg(pos_of(a.full, a.m, a.lo + qi));
+  float4 f4 = __ldg(fwd_of(a.full, a.m, a.lo + qi));
+  V3 F = steer_agent(a, v3(p4), v3(f4), nb, cnt);
+  modify_agent(a, qi, v3(p4), f4, F);
+}
+
+template <int NT, int K, int U>
 __global__ void __launch_bounds__(NT) k_fused(StepArgs a, int64_t tiles_total) {
-  __shared__ Smem sm;
+  constexpr int QB = NT * Q;    // queries per CTA (and per cluster)
+  constexpr int QPC = QB / K;   // queries owned (merged + finished) by each cluster rank
+  constexpr int NW = NT / 32;
+  __shared__ Smem<NT> sm;
+  float4(*ring)[CT] = reinterpret_cast<float4(*)[CT]>(sm.buf);
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int r = K > 1 ? (int)cg::this_cluster().block_rank() : 0;
-  const int64_t qb = blockIdx.x / K;
-  const int64_t q_base = qb * QB;  // local index of this cluster's first query
-  constexpr int QPC = QB / K;      // queries per cluster rank (merge + epilogue owner)
-
+  const int64_t q_base = (int64_t)(blockIdx.x / K) * QB;  // local index of the block's first query
   const int64_t t_lo = tiles_total * r / K, t_hi = tiles_total * (r + 1) / K;
   const int nt = (int)(t_hi - t_lo);
 
@@ -119,20 +146,18 @@ __global__ void __launch_bounds__(NT) k_fused(StepArgs a, int64_t tiles_total) {
 #pragma unroll
     for (int s = 0; s < STAGES; ++s) {
       mbar_init(&sm.full[s], 1);
-      mbar_init(&sm.empty[s], NT / 32);
+      mbar_init(&sm.empty[s], NW);
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
-  // prologue: fill the ring
-  if (tid == 0) {
+  if (tid == 0) {  // prologue: fill the ring
     for (int t = 0; t < STAGES && t < nt; ++t) {
       mbar_arrive_expect_tx(&sm.full[t], CT * sizeof(float4));
-      tma_load_1d(sm.tile[t], tile_src(a, t_lo + t), CT * sizeof(float4), &sm.full[t]);
+      tma_load_1d(ring[t], tile_src(a, t_lo + t), CT * sizeof(float4), &sm.full[t]);
     }
   }
-
-  // warm thresholds of this rank's share of the queries
+  // warm thresholds of this rank's share of the queries, exchanged through DSMEM
   for (int k = tid; k < QPC; k += NT) sm.t0[r * QPC + k] = warm_t0(a, q_base + r * QPC + k);
   if constexpr (K > 1) cg::this_cluster().sync();
   else __syncthreads();
@@ -143,8 +168,8 @@ __global__ void __launch_bounds__(NT) k_fused(StepArgs a, int64_t tiles_total) {
   key_t L[Q][7];
 #pragma unroll
   for (int q = 0; q < Q; ++q) {
-    int ql = warp * 64 + q * 32 + lane;  // query slot within the block
-    int64_t qi = q_base + ql;
+    const int ql = warp * 32 * Q + q * 32 + lane;  // query slot within the block
+    const int64_t qi = q_base + ql;
     gq[q] = a.lo + qi;
     float4 me = qi < a.nloc ? __ldg(pos_of(a.full, a.m, a.lo + qi))
                             : make_float4(__int_as_float(0x7fc00000), 0.f, 0.f, 0.f);
@@ -154,7 +179,7 @@ __global__ void __launch_bounds__(NT) k_fused(StepArgs a, int64_t tiles_total) {
     float t0;
     if constexpr (K > 1) t0 = *cg::this_cluster().map_shared_rank(&sm.t0[ql], ql / QPC);
     else t0 = sm.t0[ql];
-    // accept d2 <= t0 (inclusive, so ties at t0 are kept) and d2 < r2
+    // accept d2 <= t0 (inclusive: ties at t0 are kept) and d2 < r2
     float nt0 = t0 < __int_as_float(0x7f800000) ? __uint_as_float(__float_as_uint(t0) + 1u) : t0;
     lim[q] = fminf(r2, nt0);
 #pragma unroll
@@ -165,7 +190,7 @@ __global__ void __launch_bounds__(NT) k_fused(StepArgs a, int64_t tiles_total) {
   for (int t = 0; t < nt; ++t) {
     const int s = t % STAGES;
     mbar_wait(&sm.full[s], (uint32_t)((t / STAGES) & 1));
-    const float4* tile = sm.tile[s];
+    const float4* tile = ring[s];
     const int64_t jb = (t_lo + t) * CT;
 #pragma unroll 2
     for (int c = 0; c < CT; c += U) {
@@ -181,12 +206,12 @@ __global__ void __launch_bounds__(NT) k_fused(StepArgs a, int64_t tiles_total) {
           d[q][u] = dist2(px[q], py[q], pz[q], cc[u]);
           hit |= d[q][u] < lim[q];
         }
-      if (__any_sync(0xffffffffu, hit)) {
+      if (__any_sync(0xffffffffu, hit)) {  // rare, warp-uniform
 #pragma unroll
         for (int u = 0; u < U; ++u)
 #pragma unroll
           for (int q = 0; q < Q; ++q) {
-            int64_t j = jb + c + u;
+            const int64_t j = jb + c + u;
             if (d[q][u] < lim[q] && j != gq[q]) {
               insert7(L[q], make_key(d[q][u], (int)j));
               lim[q] = fminf(lim[q], key_d2(L[q][6]));
@@ -200,92 +225,93 @@ __global__ void __launch_bounds__(NT) k_fused(StepArgs a, int64_t tiles_total) {
     if (tid == 0 && t + STAGES < nt) {
       mbar_wait(&sm.empty[s], (uint32_t)((t / STAGES) & 1));
       mbar_arrive_expect_tx(&sm.full[s], CT * sizeof(float4));
-      tma_load_1d(sm.tile[s], tile_src(a, t_lo + t + STAGES), CT * sizeof(float4), &sm.full[s]);
+      tma_load_1d(ring[s], tile_src(a, t_lo + t + STAGES), CT * sizeof(float4), &sm.full[s]);
     }
   }
 
-  // ----------------------------------------------------- split merge ----
+  // ------------------------------------------- split merge + epilogue ----
   if constexpr (K == 1) {
 #pragma unroll
-    for (int q = 0; q < Q; ++q) {
-      int ql = warp * 64 + q * 32 + lane;
-      int64_t qi = q_base + ql;
-      if (qi >= a.nloc) continue;
-      int nb[7], cnt = 0;
-#pragma unroll
-      for (int s = 0; s < 7; ++s) {
-        key_t k = L[q][s];
-        nb[s] = k == KEY_EMPTY ? -1 : key_idx(k);
-        cnt += k == KEY_EMPTY ? 0 : 1;
-      }
-#pragma unroll
-      for (int s = 0; s < 7; ++s) a.nbr[qi * 7 + s] = nb[s];
-      a.cnt[qi] = cnt;
-      float4 p4 = __ldg(pos_of(a.full, a.m, a.lo + qi));
-      float4 f4 = __ldg(fwd_of(a.full, a.m, a.lo + qi));
-      V3 F = steer_agent(a, v3(p4), v3(f4), nb, cnt);
-      modify_agent(a, qi, v3(p4), f4, F);
-    }
+    for (int q = 0; q < Q; ++q) finish_query(a, q_base + warp * 32 * Q + q * 32 + lane, L[q]);
   } else {
-    key_t* lists = reinterpret_cast<key_t*>(&sm.tile[0][0]);  // [7][QB], k-major
-    consumer_bar();  // every warp is done reading the ring
+    key_t* lists = reinterpret_cast<key_t*>(sm.buf);  // [7][QB]
+    __syncthreads();  // every warp is done reading the ring
 #pragma unroll
     for (int q = 0; q < Q; ++q) {
-      int ql = warp * 64 + q * 32 + lane;
+      const int ql = warp * 32 * Q + q * 32 + lane;
 #pragma unroll
       for (int s = 0; s < 7; ++s) lists[s * QB + ql] = L[q][s];
     }
     cg::cluster_group cl = cg::this_cluster();
     cl.sync();  // all partial lists of the cluster are in shared memory
-    // LP lanes per query; each lane merges 2 of the K source lists, then a
-    // butterfly over the LP lanes.  K == 2 * LP.
-    constexpr int LP = K / 2;
-    const int my_q = r * QPC + tid / LP;  // query slot within the cluster block
-    const int sub = tid % LP;
-    key_t A[7], B[7];
-    {
-      const key_t* la = cl.map_shared_rank(lists, sub);
-      const key_t* lb = cl.map_shared_rank(lists, sub + LP);
+    if constexpr (QPC >= NT) {
+      // K <= Q: each thread owns QPC / NT queries and merges all K lists of each.
+      constexpr int QPT = QPC / NT;
+      key_t A[QPT][7];
 #pragma unroll
-      for (int s = 0; s < 7; ++s) {
-        A[s] = la[s * QB + my_q];
-        B[s] = lb[s * QB + my_q];
+      for (int w = 0; w < QPT; ++w) {
+        const int my_q = r * QPC + w * NT + tid;
+#pragma unroll
+        for (int src = 0; src < K; ++src) {
+          const key_t* l = cl.map_shared_rank(lists, src);
+          key_t B[7];
+#pragma unroll
+          for (int s = 0; s < 7; ++s) B[s] = l[s * QB + my_q];
+          if (src == 0) {
+#pragma unroll
+            for (int s = 0; s < 7; ++s) A[w][s] = B[s];
+          } else {
+            merge7(A[w], B);
+          }
+        }
       }
-    }
-    cl.sync();  // no CTA reads a peer's shared memory after this point
-    merge7(A, B);
+      cluster_arrive();  // done reading peers' shared memory
 #pragma unroll
-    for (int w = 1; w < LP; w <<= 1) {
+      for (int w = 0; w < QPT; ++w) finish_query(a, q_base + r * QPC + w * NT + tid, A[w]);
+      cluster_wait();
+    } else {
+      // K > Q: LP = K / Q lanes per query; each lane merges Q of the K lists,
+      // then a shuffle butterfly over the LP lanes.
+      constexpr int LP = K / Q;
+      const int my_q = r * QPC + tid / LP;
+      const int sub = tid % LP;
+      key_t A[7];
 #pragma unroll
-      for (int s = 0; s < 7; ++s) B[s] = __shfl_xor_sync(0xffffffffu, A[s], w);
-      merge7(A, B);
-    }
-    const int64_t qi = q_base + my_q;
-    if (sub == 0 && qi < a.nloc) {
-      int nb[7], cnt = 0;
+      for (int i = 0; i < Q; ++i) {
+        const key_t* l = cl.map_shared_rank(lists, sub + i * LP);
+        key_t B[7];
 #pragma unroll
-      for (int s = 0; s < 7; ++s) {
-        nb[s] = A[s] == KEY_EMPTY ? -1 : key_idx(A[s]);
-        cnt += A[s] == KEY_EMPTY ? 0 : 1;
+        for (int s = 0; s < 7; ++s) B[s] = l[s * QB + my_q];
+        if (i == 0) {
+#pragma unroll
+          for (int s = 0; s < 7; ++s) A[s] = B[s];
+        } else {
+          merge7(A, B);
+        }
       }
+      cluster_arrive();  // done reading peers' shared memory
 #pragma unroll
-      for (int s = 0; s < 7; ++s) a.nbr[qi * 7 + s] = nb[s];
-      a.cnt[qi] = cnt;
-      float4 p4 = __ldg(pos_of(a.full, a.m, a.lo + qi));
-      float4 f4 = __ldg(fwd_of(a.full, a.m, a.lo + qi));
-      V3 F = steer_agent(a, v3(p4), v3(f4), nb, cnt);
-      modify_agent(a, qi, v3(p4), f4, F);
+      for (int w = 1; w < LP; w <<= 1) {
+        key_t B[7];
+#pragma unroll
+        for (int s = 0; s < 7; ++s) B[s] = __shfl_xor_sync(0xffffffffu, A[s], w);
+        merge7(A, B);
+      }
+      if (sub == 0) finish_query(a, q_base + my_q, A);
+      cluster_wait();
     }
   }
 }
 
-template <int K>
-cudaError_t launch_k(const StepArgs& a, int64_t tiles, int64_t nqb, cudaStream_t s) {
-  auto kern = k_fused<K>;
+template <int NT, int K>
+cudaError_t launch_k(const StepArgs& a, int64_t tiles, cudaStream_t s) {
+  constexpr int U = 2;
+  auto kern = k_fused<NT, K, U>;
   if (K > 8) {
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
     if (e != cudaSuccess) return e;
   }
+  const int64_t nqb = (a.nloc + NT * Q - 1) / (NT * Q);
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3((unsigned)(nqb * K));
   cfg.blockDim = dim3(NT);
@@ -301,46 +327,77 @@ cudaError_t launch_k(const StepArgs& a, int64_t tiles, int64_t nqb, cudaStream_t
   return cudaLaunchKernelEx(&cfg, kern, a, tiles);
 }
 
+template <int NT>
+cudaError_t launch_nt(const StepArgs& a, int K, int64_t tiles, cudaStream_t s) {
+  switch (K) {
+    case 1: return launch_k<NT, 1>(a, tiles, s);
+    case 2: return launch_k<NT, 2>(a, tiles, s);
+    case 4: return launch_k<NT, 4>(a, tiles, s);
+    case 8: return launch_k<NT, 8>(a, tiles, s);
+    default: return launch_k<NT, 16>(a, tiles, s);
+  }
+}
+
 }  // namespace
 
-// Choose the cluster size K: the grid (K * query blocks) should fill the SMs as
-// evenly as possible (efficiency (C/S) / ceil(C/S)), with at least 2 candidate
-// tiles per CTA; ties go to the smaller K (less merge work).
-int fused_auto_cluster(int64_t total_candidates, int64_t nloc, int sm_count) {
-  int64_t nqb = (nloc + QB - 1) / QB;
-  int64_t tiles = total_candidates / CT;
-  int best = 1;
-  double best_eff = -1.0;
-  for (int K = 1; K <= 16; K *= 2) {
-    if (K > 1 && tiles / K < 2) break;
-    double C = (double)(nqb * K), S = (double)sm_count;
-    double eff = (C / S) / std::ceil(C / S);
-    if (C < 4 * S) eff *= C / (4 * S);  // too few warps per SM to hide latency
-    if (eff > best_eff + 1e-9) {
-      best_eff = eff;
-      best = K;
+// Occupancy-aware launch plan.  For each CTA size NT (64 or 128 threads) and
+// cluster size K, the grid is C = K * ceil(n_local / (NT * Q)) CTAs.  Score =
+//   balance   (C/S) / ceil(C/S), S = SM count (equal-work CTAs on S SMs)
+// x issue    measured FP32 issue efficiency of the scalar Q=4 loop vs warps/SM
+//            (tools/probe_fp32x2.cu on B200: 8 -> 0.80, 16 -> 0.87, 32 -> 0.88)
+// x chunk    per-CTA fixed cost (ring fill, merge, epilogue ~ 256 candidates)
+// Ties go to the smaller K (less merge work).
+static double issue_eff(double warps_per_sm) {
+  if (warps_per_sm >= 24) return 0.88;
+  if (warps_per_sm >= 16) return 0.866 + (warps_per_sm - 16) * (0.014 / 8);
+  if (warps_per_sm >= 8) return 0.80 + (warps_per_sm - 8) * (0.066 / 8);
+  return 0.80 * warps_per_sm / 8;
+}
+
+struct Plan {
+  int nt, k;
+};
+
+static Plan plan_launch(int64_t total_candidates, int64_t nloc, int sm_count, int forced_k) {
+  static const int resident[2] = {8, 4};  // CTAs/SM for NT = 64, 128 (~120 registers, ptxas -v)
+  const int64_t tiles = total_candidates / CT;
+  Plan best{128, 1};
+  double best_score = -1.0;
+  for (int ni = 0; ni < 2; ++ni) {
+    const int nt = ni == 0 ? 64 : 128;
+    const int64_t nqb = (nloc + nt * Q - 1) / (nt * Q);
+    for (int K = 1; K <= 16; K *= 2) {
+      if (forced_k && K != forced_k) continue;
+      if (K > 1 && tiles / K < 1) break;
+      const double C = (double)(nqb * K), S = (double)sm_count;
+      const double per_sm = std::ceil(C / S);
+      const double balance = (C / S) / per_sm;
+      const double warps = std::min<double>(per_sm, resident[ni]) * nt / 32.0;
+      const double cand = (double)total_candidates / K;
+      const double score = balance * issue_eff(warps) * cand / (cand + 256.0);
+      if (score > best_score * (1.0 + 1e-6)) {
+        best_score = score;
+        best = Plan{nt, K};
+      }
     }
   }
   return best;
 }
 
+int fused_auto_cluster(int64_t total_candidates, int64_t nloc, int sm_count) {
+  return plan_launch(total_candidates, nloc, sm_count, 0).k;
+}
+
 cudaError_t launch_fused(const StepArgs& a, int cluster, cudaStream_t s) {
   if (a.nloc <= 0) return cudaSuccess;
-  int64_t total = (int64_t)a.world * a.m;
-  int64_t tiles = total / CT;
-  int64_t nqb = (a.nloc + QB - 1) / QB;
+  const int64_t total = (int64_t)a.world * a.m;
+  const int64_t tiles = total / CT;
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  int K = cluster > 0 ? cluster : fused_auto_cluster(total, a.nloc, sms);
-  while (K > 1 && tiles / K < 1) K /= 2;
-  switch (K) {
-    case 1: return launch_k<1>(a, tiles, nqb, s);
-    case 2: return launch_k<2>(a, tiles, nqb, s);
-    case 4: return launch_k<4>(a, tiles, nqb, s);
-    case 8: return launch_k<8>(a, tiles, nqb, s);
-    default: return launch_k<16>(a, tiles, nqb, s);
-  }
+  Plan p = plan_launch(total, a.nloc, sms, cluster);
+  while (p.k > 1 && tiles / p.k < 1) p.k /= 2;
+  return p.nt == 64 ? launch_nt<64>(a, p.k, tiles, s) : launch_nt<128>(a, p.k, tiles, s);
 }
 
 }  // namespace boids
