@@ -86,6 +86,9 @@ typedef struct boids_info_t {
   int32_t kernel;    /* brute-force kernel variant in use (BOIDS_KERNEL_*) */
   int32_t cluster;   /* candidate split (CTAs per cluster) of the fused kernel */
   int64_t launches;  /* number of kernels this handle has launched so far */
+  int64_t slow_groups; /* fused kernel, cumulative: vote groups (U candidates x Q queries x 32
+                          lanes) that took the insertion path ... */
+  int64_t vote_groups; /* ... out of this many (diagnostics; boids_info synchronises) */
 } boids_info_t;
 
 #define BOIDS_KERNEL_FUSED 0  /* default: one fused search+steer+modify kernel per step */
@@ -96,6 +99,11 @@ typedef struct boids_info_t {
 #define BOIDS_OPT_KERNEL 2          /* BOIDS_KERNEL_* */
 #define BOIDS_OPT_PROFILE 3         /* 1: bracket each kernel launch with CUDA events (boids_get_profile) */
 #define BOIDS_OPT_CLUSTER 4         /* 0 = automatic, else force the fused kernel's cluster size (1..16) */
+#define BOIDS_OPT_RESORT 6          /* refresh the spatial order of the fused kernel's query blocks every
+                                       `value` steps (default 8; results never depend on it) */
+#define BOIDS_OPT_VOTE_U 7          /* fused kernel: candidates per warp vote, 4 (default) or 8 */
+#define BOIDS_OPT_PHASES 5          /* diagnostics: value = max CTAs; the fused kernel records per-CTA
+                                       %globaltimer stamps (read with boids_get_phases); 0 = off */
 
 BOIDS_API void boids_default_params(boids_params* out);
 
@@ -153,6 +161,7 @@ BOIDS_API int boids_get_steering(boids_ctx* ctx, float* force3);
 /* Wait for all enqueued work; returns the first pending CUDA error. */
 BOIDS_API int boids_sync(boids_ctx* ctx);
 
+/* Describe the handle (synchronises: it reads the device-side counters). */
 BOIDS_API int boids_info(boids_ctx* ctx, boids_info_t* out);
 
 /* Accumulated kernel time (ms) and launch count per kernel class since the last
@@ -160,6 +169,9 @@ BOIDS_API int boids_info(boids_ctx* ctx, boids_info_t* out);
  * Classes: 0 fused/search, 1 update, 2 binning, 3 grid search.  Synchronises. */
 #define BOIDS_PROF_CLASSES 4
 BOIDS_API int boids_get_profile(boids_ctx* ctx, double* ms, int64_t* launches, int32_t reset);
+
+/* Diagnostics: copy `count` u64 phase stamps (8 per CTA) of the last fused step to host. */
+BOIDS_API int boids_get_phases(boids_ctx* ctx, uint64_t* out, int64_t count);
 
 BOIDS_API void boids_destroy(boids_ctx* ctx);
 

@@ -20,7 +20,8 @@ BOIDS_OK, BOIDS_EINVAL, BOIDS_ECUDA, BOIDS_ENCCL, BOIDS_ENOMEM = 0, -1, -2, -3, 
 BOIDS_BRUTE, BOIDS_GRID = 0, 1
 BOIDS_INIT_OPENSTEER, BOIDS_INIT_WORLD = 0, 1
 BOIDS_KERNEL_FUSED, BOIDS_KERNEL_SIMPLE = 0, 1
-BOIDS_OPT_RECORD_STEERING, BOIDS_OPT_KERNEL, BOIDS_OPT_PROFILE, BOIDS_OPT_CLUSTER = 1, 2, 3, 4
+BOIDS_OPT_RECORD_STEERING, BOIDS_OPT_KERNEL, BOIDS_OPT_PROFILE, BOIDS_OPT_CLUSTER, BOIDS_OPT_PHASES = 1, 2, 3, 4, 5
+BOIDS_OPT_RESORT, BOIDS_OPT_VOTE_U = 6, 7
 BOIDS_PROF_CLASSES = 4
 PROF_NAMES = ("fused_or_search", "update", "binning", "grid_search")
 
@@ -29,7 +30,7 @@ EXPORTS = (
     "boids_default_params", "boids_create", "boids_create_shard", "boids_set_stream",
     "boids_set_option", "boids_step", "boids_step_shard", "boids_shard_buffers",
     "boids_get_state", "boids_set_state", "boids_get_neighbors", "boids_get_steering",
-    "boids_sync", "boids_info", "boids_get_profile", "boids_destroy", "boids_last_error",
+    "boids_sync", "boids_info", "boids_get_profile", "boids_get_phases", "boids_destroy", "boids_last_error",
 )
 
 
@@ -53,7 +54,7 @@ class boids_info_t(C.Structure):
     _fields_ = [
         ("n", C.c_int64), ("lo", C.c_int64), ("hi", C.c_int64), ("slice", C.c_int64),
         ("rank", C.c_int32), ("world", C.c_int32), ("kernel", C.c_int32), ("cluster", C.c_int32),
-        ("launches", C.c_int64),
+        ("launches", C.c_int64), ("slow_groups", C.c_int64), ("vote_groups", C.c_int64),
     ]
 
 
@@ -88,6 +89,7 @@ def load(path: str = LIB_PATH):
         "boids_sync": (C.c_int, [vp]),
         "boids_info": (C.c_int, [vp, C.POINTER(boids_info_t)]),
         "boids_get_profile": (C.c_int, [vp, C.POINTER(C.c_double), C.POINTER(i64), i32]),
+        "boids_get_phases": (C.c_int, [vp, C.POINTER(C.c_uint64), i64]),
         "boids_destroy": (None, [vp]),
         "boids_last_error": (C.c_char_p, []),
     }
@@ -167,9 +169,19 @@ def boids_info(h: int) -> boids_info_t:
     return info
 
 
+_spans: dict = {}
+
+
+def _count(h: int) -> int:
+    """Owned agents of a handle (hi - lo); cached -- a handle's span never changes."""
+    if h not in _spans:
+        k = boids_info(h)
+        _spans[h] = k.hi - k.lo
+    return _spans[h]
+
+
 def boids_get_state(h: int, out: dict | None = None) -> dict:
-    k = boids_info(h)
-    cnt = k.hi - k.lo
+    cnt = _count(h)
     out = out or dict(pos=np.empty((cnt, 3), np.float32), fwd=np.empty((cnt, 3), np.float32),
                       up=np.empty((cnt, 3), np.float32), side=np.empty((cnt, 3), np.float32),
                       speed=np.empty(cnt, np.float32))
@@ -179,8 +191,7 @@ def boids_get_state(h: int, out: dict | None = None) -> dict:
 
 
 def boids_set_state(h: int, state: dict):
-    k = boids_info(h)
-    cnt = k.hi - k.lo
+    cnt = _count(h)
     pos = _f32(state["pos"], (cnt, 3))
     fwd = _f32(state["fwd"], (cnt, 3))
     up = _f32(state["up"], (cnt, 3))
@@ -190,8 +201,7 @@ def boids_set_state(h: int, state: dict):
 
 
 def boids_get_neighbors(h: int):
-    k = boids_info(h)
-    cnt = k.hi - k.lo
+    cnt = _count(h)
     idx = np.empty((cnt, 7), np.int32)
     c = np.empty(cnt, np.int32)
     _check(load().boids_get_neighbors(h, _iptr(idx), _iptr(c)))
@@ -199,8 +209,7 @@ def boids_get_neighbors(h: int):
 
 
 def boids_get_steering(h: int):
-    k = boids_info(h)
-    F = np.empty((k.hi - k.lo, 3), np.float32)
+    F = np.empty((_count(h), 3), np.float32)
     _check(load().boids_get_steering(h, _fptr(F)))
     return F
 
@@ -216,8 +225,15 @@ def boids_get_profile(h: int, reset: bool = True):
     return {PROF_NAMES[i]: (ms[i], n[i]) for i in range(BOIDS_PROF_CLASSES)}
 
 
+def boids_get_phases(h: int, ctas: int):
+    out = np.zeros((ctas, 8), np.uint64)
+    _check(load().boids_get_phases(h, out.ctypes.data_as(C.POINTER(C.c_uint64)), ctas * 8))
+    return out
+
+
 def boids_destroy(h: int):
     if h:
+        _spans.pop(h, None)
         load().boids_destroy(h)
 
 

@@ -55,6 +55,17 @@ struct boids_ctx {
   int cur = 0;
   float4 *up4 = nullptr, *side4 = nullptr, *force4 = nullptr;
   int32_t *nbr = nullptr, *cnt = nullptr;
+  // spatial binning (k_bin.cu): locality grid of the brute-force step
+  BinGrid loc_grid{};
+  int2* cellrank = nullptr;
+  int32_t *bcnt = nullptr, *bstart = nullptr, *qperm = nullptr;
+  float4* cand = nullptr;
+  int64_t ncand = 0;
+  unsigned long long* stats = nullptr;  // fused-kernel insertion-path counters (device)
+  unsigned long long* phase = nullptr;  // diagnostics (BOIDS_OPT_PHASES): per-CTA timestamps
+  int vote_u = 4;          // fused kernel: candidates per warp vote
+  int resort_every = 8;    // refresh the spatial query order every this many steps
+  int64_t since_sort = -1; // steps since the last refresh (-1: never sorted)
   bool warm = false;
   bool record_steering = false, steering_valid = false;
   int kernel = BOIDS_KERNEL_FUSED;
@@ -109,6 +120,13 @@ void free_ctx(boids_ctx* c) {
   cudaFree(c->force4);
   cudaFree(c->nbr);
   cudaFree(c->cnt);
+  cudaFree(c->cellrank);
+  cudaFree(c->bcnt);
+  cudaFree(c->bstart);
+  cudaFree(c->qperm);
+  cudaFree(c->cand);
+  cudaFree(c->stats);
+  cudaFree(c->phase);
   for (auto& r : c->recs) {
     cudaEventDestroy(r.a);
     cudaEventDestroy(r.b);
@@ -130,7 +148,7 @@ cudaEvent_t get_event(boids_ctx* c) {
 
 // Launch wrapper: counts launches and, when profiling, brackets with events.
 template <class F>
-int launch(boids_ctx* c, int cls, F&& f) {
+int launch(boids_ctx* c, int cls, F&& f, int kernels = 1) {
   cudaEvent_t a = nullptr, b = nullptr;
   if (c->profile) {
     a = get_event(c);
@@ -138,7 +156,7 @@ int launch(boids_ctx* c, int cls, F&& f) {
     CK(cudaEventRecord(a, c->stream));
   }
   CK(f());
-  c->launches++;
+  c->launches += kernels;
   if (c->profile) {
     CK(cudaEventRecord(b, c->stream));
     c->recs.push_back({cls, a, b});
@@ -188,6 +206,18 @@ int create_impl(int64_t n, const boids_params* p, uint64_t seed, int32_t rank, i
     free_ctx(c);
     return rc;
   }
+  const int64_t slots = shard ? (int64_t)world * m : m;
+  c->loc_grid = make_locality_grid(n, *p);
+  c->ncand = (n + TILE - 1) / TILE * TILE;
+  if ((rc = alloc((void**)&c->cellrank, slots * sizeof(int2))) ||
+      (rc = alloc((void**)&c->bcnt, c->loc_grid.cells * sizeof(int32_t))) ||
+      (rc = alloc((void**)&c->bstart, (c->loc_grid.cells + 1) * sizeof(int32_t))) ||
+      (rc = alloc((void**)&c->qperm, m * sizeof(int32_t))) ||
+      (rc = alloc((void**)&c->cand, c->ncand * sizeof(float4))) ||
+      (rc = alloc((void**)&c->stats, 2 * sizeof(unsigned long long)))) {
+    free_ctx(c);
+    return rc;
+  }
   cudaStream_t s = c->stream;
   cudaError_t e = cudaSuccess;
   // phantoms in every segment of every buffer; then the owned agents
@@ -197,6 +227,9 @@ int create_impl(int64_t n, const boids_params* p, uint64_t seed, int32_t rank, i
   if (e == cudaSuccess) e = cudaMemsetAsync(c->nbr, 0xFF, m * 7 * sizeof(int32_t), s);
   if (e == cudaSuccess) e = cudaMemsetAsync(c->up4, 0, m * sizeof(float4), s);
   if (e == cudaSuccess) e = cudaMemsetAsync(c->side4, 0, m * sizeof(float4), s);
+  if (e == cudaSuccess) e = cudaMemsetAsync(c->bcnt, 0, c->loc_grid.cells * sizeof(int32_t), s);
+  if (e == cudaSuccess) e = launch_fill_nan(c->cand, c->ncand, s);  // entries >= n stay NaN
+  if (e == cudaSuccess) e = cudaMemsetAsync(c->stats, 0, 2 * sizeof(unsigned long long), s);
   if (e == cudaSuccess)
     e = launch_fill_phantoms(c->buf[0], m, shard ? 0 : c->nloc, shard ? world : 1, s);
   if (e == cudaSuccess) e = launch_fill_phantoms(c->buf[1], m, c->nloc, 1, s);
@@ -229,6 +262,12 @@ StepArgs make_args(boids_ctx* c, float dt) {
   a.warm = c->warm ? 1 : 0;
   a.dt = dt;
   a.p = c->p;
+  a.cand = c->cand;
+  a.ncand = c->ncand;
+  a.qperm = c->qperm;
+  a.stats = c->stats;
+  a.phase = c->phase;
+  a.vote_u = c->vote_u;
   return a;
 }
 
@@ -239,6 +278,18 @@ int one_step(boids_ctx* c, float dt) {
     if ((rc = launch(c, 0, [&] { return launch_search_simple(a, c->stream); }))) return rc;
     if ((rc = launch(c, 1, [&] { return launch_update(a, c->stream); }))) return rc;
   } else {
+    // a2: spatial (Morton) order of the owned queries, so the 128 queries of a
+    // warp are spatially coherent.  It is only a permutation of the work (results
+    // never depend on it), so it is refreshed every resort_every steps.
+    if (c->since_sort < 0 || c->since_sort >= c->resort_every) {
+      if ((rc = launch(c, 2, [&] {
+             return launch_bin(a.full, c->m, c->lo, c->nloc, c->loc_grid, c->cellrank, c->bcnt, c->bstart,
+                               nullptr, c->qperm, (int)c->lo, c->stream, nullptr);
+           }, 3)))
+        return rc;
+      c->since_sort = 0;
+    }
+    c->since_sort++;
     int cl = c->cluster_opt;
     if ((rc = launch(c, 0, [&] { return launch_fused(a, cl, c->stream); }))) return rc;
   }
@@ -315,6 +366,25 @@ BOIDS_API int boids_set_option(boids_ctx* c, int32_t opt, int64_t v) {
       return BOIDS_OK;
     case BOIDS_OPT_PROFILE:
       c->profile = v != 0;
+      return BOIDS_OK;
+    case BOIDS_OPT_VOTE_U:
+      if (v != 4 && v != 8) return fail(BOIDS_EINVAL, "vote width must be 4 or 8");
+      c->vote_u = (int)v;
+      return BOIDS_OK;
+    case BOIDS_OPT_RESORT:
+      if (v < 1) return fail(BOIDS_EINVAL, "resort interval must be >= 1");
+      c->resort_every = (int)v;
+      c->since_sort = -1;
+      return BOIDS_OK;
+    case BOIDS_OPT_PHASES:
+      if (v && !c->phase) {
+        CK(cudaMalloc((void**)&c->phase, (size_t)v * 8 * sizeof(unsigned long long)));
+        CK(cudaMemset(c->phase, 0, (size_t)v * 8 * sizeof(unsigned long long)));
+      }
+      if (!v && c->phase) {
+        cudaFree(c->phase);
+        c->phase = nullptr;
+      }
       return BOIDS_OK;
     case BOIDS_OPT_CLUSTER:
       if (v < 0 || v > 16 || (v & (v - 1))) return fail(BOIDS_EINVAL, "cluster must be 0 or a power of two <= 16");
@@ -451,9 +521,13 @@ BOIDS_API int boids_info(boids_ctx* c, boids_info_t* o) {
   o->rank = c->rank;
   o->world = c->world;
   o->kernel = c->kernel;
-  o->cluster = c->cluster_opt ? c->cluster_opt
-                              : fused_auto_cluster((int64_t)(c->shard ? c->world : 1) * c->m, c->nloc, c->sm_count);
+  o->cluster = c->cluster_opt ? c->cluster_opt : fused_auto_cluster(c->ncand, c->nloc, c->sm_count);
   o->launches = c->launches;
+  unsigned long long st[2] = {0, 0};
+  CK(cudaMemcpyAsync(st, c->stats, sizeof(st), cudaMemcpyDeviceToHost, c->stream));
+  CK(cudaStreamSynchronize(c->stream));
+  o->slow_groups = (int64_t)st[0];
+  o->vote_groups = (int64_t)st[1];
   return BOIDS_OK;
 }
 
@@ -478,6 +552,15 @@ BOIDS_API int boids_get_profile(boids_ctx* c, double* ms, int64_t* launches, int
       c->prof_n[k] = 0;
     }
   }
+  return BOIDS_OK;
+}
+
+BOIDS_API int boids_get_phases(boids_ctx* c, uint64_t* out, int64_t count) {
+  if (!c || !out) return fail(BOIDS_EINVAL, "NULL argument");
+  if (!c->phase) return fail(BOIDS_EINVAL, "phases not enabled (BOIDS_OPT_PHASES)");
+  DeviceGuard g(c->dev);
+  CK(cudaMemcpyAsync(out, c->phase, count * sizeof(uint64_t), cudaMemcpyDeviceToHost, c->stream));
+  CK(cudaStreamSynchronize(c->stream));
   return BOIDS_OK;
 }
 

@@ -70,6 +70,19 @@ cudaError_t launch_fill_phantoms(float4* base, int64_t m, int64_t nloc, int64_t 
   return cudaGetLastError();
 }
 
+__global__ void k_fill_nan(float4* p, int64_t count) {
+  int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (k >= count) return;
+  float nan = __int_as_float(0x7fc00000);
+  p[k] = make_float4(nan, nan, nan, __int_as_float(-1));
+}
+
+cudaError_t launch_fill_nan(float4* p, int64_t count, cudaStream_t s) {
+  if (count <= 0) return cudaSuccess;
+  k_fill_nan<<<(unsigned)((count + 255) / 256), 256, 0, s>>>(p, count);
+  return cudaGetLastError();
+}
+
 // ------------------------------------------------------- simple search ----
 // One thread per owned agent; candidate positions staged through shared memory
 // one TILE at a time (the thesis's version-2 structure, Listing 6.2), register

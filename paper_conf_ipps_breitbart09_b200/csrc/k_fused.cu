@@ -21,7 +21,8 @@
 //  * Warm threshold: t0 = max d2 to the previous step's 7 neighbours at the
 //    current positions is an upper bound on the true 7th key, so only
 //    candidates with d2 <= t0 can enter (identical result, far fewer inserts).
-//    The per-pair test is one compare against lim = min(r2, next(t0), worst).
+//    Per query lim = min(r2, next(t0), worst held); the fast test is a min
+//    tree over the Q*U distances against the thread's max lim.
 //  * The hot loop is warp-uniform: a vote over U candidates x Q queries takes
 //    the (rare) insertion path only when some lane needs it (the SIMD branching
 //    issue of sec 6.3.1).
@@ -41,7 +42,7 @@ namespace {
 
 constexpr int Q = 4;        // queries per thread (4 independent distance chains)
 constexpr int CT = 256;     // candidates per tile (4 KB)
-constexpr int STAGES = 4;   // TMA ring depth
+constexpr int STAGES = 2;   // TMA ring depth (a tile takes ~10-25 us to consume; TMA latency ~1 us)
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
   return (uint32_t)__cvta_generic_to_shared(p);
@@ -74,6 +75,14 @@ __device__ __forceinline__ void tma_load_1d(void* dst, const void* src, uint32_t
       "l"(src), "r"(bytes), "r"(smem_u32(bar))
       : "memory");
 }
+__device__ __forceinline__ void stamp(const StepArgs& a, int k) {
+  if (a.phase && threadIdx.x == 0) {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    a.phase[blockIdx.x * 8 + k] = t;
+  }
+}
+
 __device__ __forceinline__ void cluster_arrive() {
   asm volatile("barrier.cluster.arrive.release.aligned;" ::: "memory");
 }
@@ -84,17 +93,34 @@ __device__ __forceinline__ void cluster_wait() {
 template <int NT>
 struct __align__(16) Smem {
   static constexpr int QB = NT * Q;
-  static constexpr int RING = STAGES * CT * (int)sizeof(float4);
-  static constexpr int LISTS = 7 * QB * (int)sizeof(key_t);
-  // candidate ring during the scan, then the partial lists [7][QB] (k-major) for the merge
-  __align__(128) unsigned char buf[RING > LISTS ? RING : LISTS];
-  float t0[QB];  // warm thresholds (each cluster rank fills its share)
+  float4 ring[STAGES][CT];  // candidate tiles (TMA destination)
+  key_t lists[7 * QB];      // sorted top-7 per query, k-major [7][QB]; touched only on inserts
+  float t0[QB];             // warm thresholds (each cluster rank fills its share)
   uint64_t full[STAGES];
   uint64_t empty[STAGES];
 };
 
+// Insert (d2, j) into the shared-memory list of query slot ql; returns the new
+// worst d2 (+inf while fewer than 7 are held).  Out of line: it runs rarely and
+// one copy keeps the hot loop small in the instruction cache.
+__device__ __noinline__ float insert_list(key_t* lists, int qb, int ql, float d2, int j) {
+  key_t L[7];
+#pragma unroll
+  for (int s = 0; s < 7; ++s) L[s] = lists[s * qb + ql];
+  insert7(L, make_key(d2, j));
+#pragma unroll
+  for (int s = 0; s < 7; ++s) lists[s * qb + ql] = L[s];
+  return key_d2(L[6]);
+}
+
 __device__ __forceinline__ const float4* tile_src(const StepArgs& a, int64_t tile) {
   return pos_of(a.full, a.m, tile * CT);  // m % CT == 0: a tile never straddles a slice
+}
+
+// local query index held by block slot qs (>= nloc: inactive slot)
+__device__ __forceinline__ int64_t query_of(const StepArgs& a, int64_t qs) {
+  if (qs >= a.nloc) return a.nloc;
+  return a.qperm ? (int64_t)__ldg(a.qperm + qs) : qs;
 }
 
 // t0 for local query ql (returns +inf when there is no valid warm list).
@@ -135,13 +161,15 @@ __global__ void __launch_bounds__(NT) k_fused(StepArgs a, int64_t tiles_total) {
   constexpr int QPC = QB / K;   // queries owned (merged + finished) by each cluster rank
   constexpr int NW = NT / 32;
   __shared__ Smem<NT> sm;
-  float4(*ring)[CT] = reinterpret_cast<float4(*)[CT]>(sm.buf);
+  float4(*ring)[CT] = sm.ring;
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int r = K > 1 ? (int)cg::this_cluster().block_rank() : 0;
   const int64_t q_base = (int64_t)(blockIdx.x / K) * QB;  // local index of the block's first query
-  const int64_t t_lo = tiles_total * r / K, t_hi = tiles_total * (r + 1) / K;
-  const int nt = (int)(t_hi - t_lo);
+  // cluster rank r scans tiles r, r + K, r + 2K, ...: strided, so the hits of a
+  // spatially coherent query block are spread evenly over the cluster's CTAs
+  const int nt = (int)((tiles_total - r + K - 1) / K);
 
+  stamp(a, 0);
   if (tid == 0) {
 #pragma unroll
     for (int s = 0; s < STAGES; ++s) {
@@ -154,69 +182,103 @@ __global__ void __launch_bounds__(NT) k_fused(StepArgs a, int64_t tiles_total) {
   if (tid == 0) {  // prologue: fill the ring
     for (int t = 0; t < STAGES && t < nt; ++t) {
       mbar_arrive_expect_tx(&sm.full[t], CT * sizeof(float4));
-      tma_load_1d(ring[t], tile_src(a, t_lo + t), CT * sizeof(float4), &sm.full[t]);
+      tma_load_1d(ring[t], tile_src(a, r + (int64_t)t * K), CT * sizeof(float4), &sm.full[t]);
     }
   }
   // warm thresholds of this rank's share of the queries, exchanged through DSMEM
-  for (int k = tid; k < QPC; k += NT) sm.t0[r * QPC + k] = warm_t0(a, q_base + r * QPC + k);
+  for (int k = tid; k < QPC; k += NT) sm.t0[r * QPC + k] = warm_t0(a, query_of(a, q_base + r * QPC + k));
   if constexpr (K > 1) cg::this_cluster().sync();
   else __syncthreads();
+  stamp(a, 1);
 
   const float r2 = __fmul_rn(a.p.search_radius, a.p.search_radius);
+  const float r2_in = __uint_as_float(__float_as_uint(r2) - 1u);  // largest float < r2 (r2 > 0)
   float px[Q], py[Q], pz[Q], lim[Q];
-  int64_t gq[Q];
-  key_t L[Q][7];
+  int gq[Q];  // global index of each query (n < 2^31)
+  {
+    // Query coordinates are staged through shared memory as (0, x, y, z) so the
+    // LDS.128 that reads them back leaves x, y, z in odd/even/odd registers --
+    // the opposite register-bank parity of a candidate's x, y, z (even/odd/even
+    // from the tile's LDS.128), so the subtractions never read two registers of
+    // one bank (measured: ~8% dispatch stalls otherwise).  The list area is free
+    // until it is initialised below.
+    float4* qscratch = reinterpret_cast<float4*>(sm.lists) + tid * Q;
+#pragma unroll
+    for (int q = 0; q < Q; ++q) {
+      const int ql = warp * 32 * Q + q * 32 + lane;  // query slot within the block
+      const int64_t qi = query_of(a, q_base + ql);
+      gq[q] = (int)(a.lo + qi);
+      float4 me = qi < a.nloc ? __ldg(pos_of(a.full, a.m, a.lo + qi))
+                              : make_float4(__int_as_float(0x7fc00000), 0.f, 0.f, 0.f);
+      qscratch[q] = make_float4(0.f, me.x, me.y, me.z);
+    }
+#pragma unroll
+    for (int q = 0; q < Q; ++q) {
+      volatile float4* vq = qscratch + q;
+      float4 v = make_float4(vq->x, vq->y, vq->z, vq->w);
+      px[q] = v.y;
+      py[q] = v.z;
+      pz[q] = v.w;
+    }
+    __syncthreads();  // every thread has read its coordinates before the lists are initialised
+  }
 #pragma unroll
   for (int q = 0; q < Q; ++q) {
-    const int ql = warp * 32 * Q + q * 32 + lane;  // query slot within the block
-    const int64_t qi = q_base + ql;
-    gq[q] = a.lo + qi;
-    float4 me = qi < a.nloc ? __ldg(pos_of(a.full, a.m, a.lo + qi))
-                            : make_float4(__int_as_float(0x7fc00000), 0.f, 0.f, 0.f);
-    px[q] = me.x;
-    py[q] = me.y;
-    pz[q] = me.z;
+    const int ql = warp * 32 * Q + q * 32 + lane;
     float t0;
     if constexpr (K > 1) t0 = *cg::this_cluster().map_shared_rank(&sm.t0[ql], ql / QPC);
     else t0 = sm.t0[ql];
-    // accept d2 <= t0 (inclusive: ties at t0 are kept) and d2 < r2
-    float nt0 = t0 < __int_as_float(0x7f800000) ? __uint_as_float(__float_as_uint(t0) + 1u) : t0;
-    lim[q] = fminf(r2, nt0);
+    // inclusive limit: accept d2 <= t0 (ties at t0 kept) and d2 < r2, i.e. d2 <= prev(r2)
+    lim[q] = fminf(r2_in, t0);
 #pragma unroll
-    for (int s = 0; s < 7; ++s) L[q][s] = KEY_EMPTY;
+    for (int s = 0; s < 7; ++s) sm.lists[s * QB + ql] = KEY_EMPTY;
   }
+  __syncwarp();
 
   // ------------------------------------------------------------ scan ----
+  // Limits are INCLUSIVE (d2 <= lim): candidates arrive in spatial, not index,
+  // order, so a candidate tying the held 7th d2 may still win on its index; the
+  // exact (d2, index) comparison is insert7's.  Fast test per U candidates: min
+  // over all Q*U distances (an FMNMX3 tree) against limc = max_q lim[q] --
+  // conservative, so it never misses a pair that passes its own query's limit;
+  // the exact per-query test, the self exclusion and the insertion run only in
+  // the rare warp-uniform slow path.
+  float limc = fmaxf(fmaxf(lim[0], lim[1]), fmaxf(lim[2], lim[3]));
+  unsigned slow_groups = 0;
   for (int t = 0; t < nt; ++t) {
     const int s = t % STAGES;
     mbar_wait(&sm.full[s], (uint32_t)((t / STAGES) & 1));
     const float4* tile = ring[s];
-    const int64_t jb = (t_lo + t) * CT;
+    const int jb = (int)((r + (int64_t)t * K) * CT);
 #pragma unroll 2
     for (int c = 0; c < CT; c += U) {
       float4 cc[U];
 #pragma unroll
       for (int u = 0; u < U; ++u) cc[u] = tile[c + u];
       float d[Q][U];
-      bool hit = false;
 #pragma unroll
       for (int u = 0; u < U; ++u)
 #pragma unroll
-        for (int q = 0; q < Q; ++q) {
-          d[q][u] = dist2(px[q], py[q], pz[q], cc[u]);
-          hit |= d[q][u] < lim[q];
-        }
-      if (__any_sync(0xffffffffu, hit)) {  // rare, warp-uniform
+        for (int q = 0; q < Q; ++q) d[q][u] = dist2(px[q], py[q], pz[q], cc[u]);
+      float mq[Q];
+#pragma unroll
+      for (int q = 0; q < Q; ++q) {
+        mq[q] = d[q][0];
+#pragma unroll
+        for (int u = 1; u < U; ++u) mq[q] = fminf(mq[q], d[q][u]);
+      }
+      const float m = fminf(fminf(mq[0], mq[1]), fminf(mq[2], mq[3]));  // NaN (phantoms) ignored
+      if (__any_sync(0xffffffffu, m <= limc)) {  // rare, warp-uniform
+        ++slow_groups;
 #pragma unroll
         for (int u = 0; u < U; ++u)
 #pragma unroll
           for (int q = 0; q < Q; ++q) {
-            const int64_t j = jb + c + u;
-            if (d[q][u] < lim[q] && j != gq[q]) {
-              insert7(L[q], make_key(d[q][u], (int)j));
-              lim[q] = fminf(lim[q], key_d2(L[q][6]));
-            }
+            const int j = jb + c + u;
+            if (d[q][u] <= lim[q] && j != gq[q])
+              lim[q] = fminf(lim[q], insert_list(sm.lists, QB, warp * 32 * Q + q * 32 + lane, d[q][u], j));
           }
+        limc = fmaxf(fmaxf(lim[0], lim[1]), fmaxf(lim[2], lim[3]));
       }
     }
     __syncwarp();
@@ -225,25 +287,32 @@ __global__ void __launch_bounds__(NT) k_fused(StepArgs a, int64_t tiles_total) {
     if (tid == 0 && t + STAGES < nt) {
       mbar_wait(&sm.empty[s], (uint32_t)((t / STAGES) & 1));
       mbar_arrive_expect_tx(&sm.full[s], CT * sizeof(float4));
-      tma_load_1d(ring[s], tile_src(a, t_lo + t + STAGES), CT * sizeof(float4), &sm.full[s]);
+      tma_load_1d(ring[s], tile_src(a, r + (int64_t)(t + STAGES) * K), CT * sizeof(float4), &sm.full[s]);
     }
   }
 
+  stamp(a, 2);
+  if (a.stats && lane == 0) {
+    atomicAdd(a.stats, (unsigned long long)slow_groups);
+    atomicAdd(a.stats + 1, (unsigned long long)nt * (CT / U));
+  }
+
   // ------------------------------------------- split merge + epilogue ----
+  key_t* lists = sm.lists;  // [7][QB]
   if constexpr (K == 1) {
-#pragma unroll
-    for (int q = 0; q < Q; ++q) finish_query(a, q_base + warp * 32 * Q + q * 32 + lane, L[q]);
-  } else {
-    key_t* lists = reinterpret_cast<key_t*>(sm.buf);  // [7][QB]
-    __syncthreads();  // every warp is done reading the ring
+    __syncwarp();
 #pragma unroll
     for (int q = 0; q < Q; ++q) {
       const int ql = warp * 32 * Q + q * 32 + lane;
+      key_t A[7];
 #pragma unroll
-      for (int s = 0; s < 7; ++s) lists[s * QB + ql] = L[q][s];
+      for (int s = 0; s < 7; ++s) A[s] = lists[s * QB + ql];
+      finish_query(a, query_of(a, q_base + ql), A);
     }
+  } else {
     cg::cluster_group cl = cg::this_cluster();
     cl.sync();  // all partial lists of the cluster are in shared memory
+    stamp(a, 3);
     if constexpr (QPC >= NT) {
       // K <= Q: each thread owns QPC / NT queries and merges all K lists of each.
       constexpr int QPT = QPC / NT;
@@ -266,9 +335,12 @@ __global__ void __launch_bounds__(NT) k_fused(StepArgs a, int64_t tiles_total) {
         }
       }
       cluster_arrive();  // done reading peers' shared memory
+      stamp(a, 4);
 #pragma unroll
-      for (int w = 0; w < QPT; ++w) finish_query(a, q_base + r * QPC + w * NT + tid, A[w]);
+      for (int w = 0; w < QPT; ++w) finish_query(a, query_of(a, q_base + r * QPC + w * NT + tid), A[w]);
+      stamp(a, 5);
       cluster_wait();
+      stamp(a, 6);
     } else {
       // K > Q: LP = K / Q lanes per query; each lane merges Q of the K lists,
       // then a shuffle butterfly over the LP lanes.
@@ -290,6 +362,7 @@ __global__ void __launch_bounds__(NT) k_fused(StepArgs a, int64_t tiles_total) {
         }
       }
       cluster_arrive();  // done reading peers' shared memory
+      stamp(a, 4);
 #pragma unroll
       for (int w = 1; w < LP; w <<= 1) {
         key_t B[7];
@@ -297,15 +370,16 @@ __global__ void __launch_bounds__(NT) k_fused(StepArgs a, int64_t tiles_total) {
         for (int s = 0; s < 7; ++s) B[s] = __shfl_xor_sync(0xffffffffu, A[s], w);
         merge7(A, B);
       }
-      if (sub == 0) finish_query(a, q_base + my_q, A);
+      if (sub == 0) finish_query(a, query_of(a, q_base + my_q), A);
+      stamp(a, 5);
       cluster_wait();
+      stamp(a, 6);
     }
   }
 }
 
-template <int NT, int K>
+template <int NT, int K, int U>
 cudaError_t launch_k(const StepArgs& a, int64_t tiles, cudaStream_t s) {
-  constexpr int U = 2;
   auto kern = k_fused<NT, K, U>;
   if (K > 8) {
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
@@ -327,14 +401,14 @@ cudaError_t launch_k(const StepArgs& a, int64_t tiles, cudaStream_t s) {
   return cudaLaunchKernelEx(&cfg, kern, a, tiles);
 }
 
-template <int NT>
+template <int NT, int U>
 cudaError_t launch_nt(const StepArgs& a, int K, int64_t tiles, cudaStream_t s) {
   switch (K) {
-    case 1: return launch_k<NT, 1>(a, tiles, s);
-    case 2: return launch_k<NT, 2>(a, tiles, s);
-    case 4: return launch_k<NT, 4>(a, tiles, s);
-    case 8: return launch_k<NT, 8>(a, tiles, s);
-    default: return launch_k<NT, 16>(a, tiles, s);
+    case 1: return launch_k<NT, 1, U>(a, tiles, s);
+    case 2: return launch_k<NT, 2, U>(a, tiles, s);
+    case 4: return launch_k<NT, 4, U>(a, tiles, s);
+    case 8: return launch_k<NT, 8, U>(a, tiles, s);
+    default: return launch_k<NT, 16, U>(a, tiles, s);
   }
 }
 
@@ -359,7 +433,7 @@ struct Plan {
 };
 
 static Plan plan_launch(int64_t total_candidates, int64_t nloc, int sm_count, int forced_k) {
-  static const int resident[2] = {8, 4};  // CTAs/SM for NT = 64, 128 (~120 registers, ptxas -v)
+  static const int resident[2] = {9, 5};  // CTAs/SM for NT = 64, 128 (96 registers; 24 / 39 KB smem)
   const int64_t tiles = total_candidates / CT;
   Plan best{128, 1};
   double best_score = -1.0;
@@ -397,7 +471,8 @@ cudaError_t launch_fused(const StepArgs& a, int cluster, cudaStream_t s) {
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   Plan p = plan_launch(total, a.nloc, sms, cluster);
   while (p.k > 1 && tiles / p.k < 1) p.k /= 2;
-  return p.nt == 64 ? launch_nt<64>(a, p.k, tiles, s) : launch_nt<128>(a, p.k, tiles, s);
+  if (a.vote_u == 8) return p.nt == 64 ? launch_nt<64, 8>(a, p.k, tiles, s) : launch_nt<128, 8>(a, p.k, tiles, s);
+  return p.nt == 64 ? launch_nt<64, 4>(a, p.k, tiles, s) : launch_nt<128, 4>(a, p.k, tiles, s);
 }
 
 }  // namespace boids
