@@ -89,10 +89,14 @@ typedef struct boids_info_t {
   int64_t slow_groups; /* fused kernel, cumulative: vote groups (U candidates x Q queries x 32
                           lanes) that took the insertion path ... */
   int64_t vote_groups; /* ... out of this many (diagnostics; boids_info synchronises) */
+  int64_t fallbacks;   /* warm path, cumulative: agents re-searched after a hit-buffer overflow */
 } boids_info_t;
 
-#define BOIDS_KERNEL_FUSED 0  /* default: one fused search+steer+modify kernel per step */
-#define BOIDS_KERNEL_SIMPLE 1 /* two kernels: tiled search -> neighbour lists -> update */
+#define BOIDS_KERNEL_FUSED 0   /* default: cold steps run the fused cluster kernel (search + merge +
+                                  steer + modify); warm steps (previous lists known) run the
+                                  all-pairs hit scan + select/update pair */
+#define BOIDS_KERNEL_SIMPLE 1  /* two kernels: tiled search -> neighbour lists -> update */
+#define BOIDS_KERNEL_CLUSTER 2 /* every step on the fused cluster kernel */
 
 /* Options for boids_set_option. */
 #define BOIDS_OPT_RECORD_STEERING 1 /* 1: keep the last step's steering vectors (boids_get_steering) */

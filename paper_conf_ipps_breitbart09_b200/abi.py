@@ -19,7 +19,7 @@ LIB_PATH = os.path.join(HERE, "libboids.so")
 BOIDS_OK, BOIDS_EINVAL, BOIDS_ECUDA, BOIDS_ENCCL, BOIDS_ENOMEM = 0, -1, -2, -3, -4
 BOIDS_BRUTE, BOIDS_GRID = 0, 1
 BOIDS_INIT_OPENSTEER, BOIDS_INIT_WORLD = 0, 1
-BOIDS_KERNEL_FUSED, BOIDS_KERNEL_SIMPLE = 0, 1
+BOIDS_KERNEL_FUSED, BOIDS_KERNEL_SIMPLE, BOIDS_KERNEL_CLUSTER = 0, 1, 2
 BOIDS_OPT_RECORD_STEERING, BOIDS_OPT_KERNEL, BOIDS_OPT_PROFILE, BOIDS_OPT_CLUSTER, BOIDS_OPT_PHASES = 1, 2, 3, 4, 5
 BOIDS_OPT_RESORT, BOIDS_OPT_VOTE_U = 6, 7
 BOIDS_PROF_CLASSES = 4
@@ -55,6 +55,7 @@ class boids_info_t(C.Structure):
         ("n", C.c_int64), ("lo", C.c_int64), ("hi", C.c_int64), ("slice", C.c_int64),
         ("rank", C.c_int32), ("world", C.c_int32), ("kernel", C.c_int32), ("cluster", C.c_int32),
         ("launches", C.c_int64), ("slow_groups", C.c_int64), ("vote_groups", C.c_int64),
+        ("fallbacks", C.c_int64),
     ]
 
 

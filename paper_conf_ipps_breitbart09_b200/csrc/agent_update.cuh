@@ -16,8 +16,8 @@ __device__ __forceinline__ V3 steer_agent(const StepArgs& a, V3 me, V3 fme, cons
   for (int k = 0; k < 7; ++k) {
     if (k >= cnt) break;
     int64_t j = nb[k];
-    float4 pj = __ldg(pos_of(a.full, a.m, j));
-    float4 fj = __ldg(fwd_of(a.full, a.m, j));
+    float4 pj = __ldg(pos_of(a.full, a.m, a.sdiv, j));
+    float4 fj = __ldg(fwd_of(a.full, a.m, a.sdiv, j));
     V3 o = sub(v3(pj), me);  // A.position - me.position (Listing 5.3 line 7)
     float L = len(o);
     if (L > 0.0f) sep = sub(sep, divs(divs(o, L), L));  // 1/d fall-off (Listing 5.3 line 10)

@@ -62,6 +62,11 @@ struct boids_ctx {
   float4* cand = nullptr;
   int64_t ncand = 0;
   unsigned long long* stats = nullptr;  // fused-kernel insertion-path counters (device)
+  unsigned long long* hits = nullptr;   // warm path hit buffers [m][HITS]
+  int32_t* hitcnt = nullptr;            // warm path hit counts [m]
+  int32_t* nbr8 = nullptr;              // 8th nearest of the last step or -1 [m]
+  unsigned long long* partial = nullptr;  // warm path partial lists [m][PSLOTS][7]
+  int32_t* pcnt = nullptr;
   unsigned long long* phase = nullptr;  // diagnostics (BOIDS_OPT_PHASES): per-CTA timestamps
   int vote_u = 4;          // fused kernel: candidates per warp vote
   int resort_every = 8;    // refresh the spatial query order every this many steps
@@ -126,6 +131,11 @@ void free_ctx(boids_ctx* c) {
   cudaFree(c->qperm);
   cudaFree(c->cand);
   cudaFree(c->stats);
+  cudaFree(c->hits);
+  cudaFree(c->hitcnt);
+  cudaFree(c->nbr8);
+  cudaFree(c->partial);
+  cudaFree(c->pcnt);
   cudaFree(c->phase);
   for (auto& r : c->recs) {
     cudaEventDestroy(r.a);
@@ -214,7 +224,12 @@ int create_impl(int64_t n, const boids_params* p, uint64_t seed, int32_t rank, i
       (rc = alloc((void**)&c->bstart, (c->loc_grid.cells + 1) * sizeof(int32_t))) ||
       (rc = alloc((void**)&c->qperm, m * sizeof(int32_t))) ||
       (rc = alloc((void**)&c->cand, c->ncand * sizeof(float4))) ||
-      (rc = alloc((void**)&c->stats, 2 * sizeof(unsigned long long)))) {
+      (rc = alloc((void**)&c->stats, 4 * sizeof(unsigned long long))) ||
+      (rc = alloc((void**)&c->hits, (size_t)m * HITS * sizeof(unsigned long long))) ||
+      (rc = alloc((void**)&c->hitcnt, m * sizeof(int32_t))) ||
+      (rc = alloc((void**)&c->nbr8, m * sizeof(int32_t))) ||
+      (rc = alloc((void**)&c->partial, (size_t)m * PSLOTS * 7 * sizeof(unsigned long long))) ||
+      (rc = alloc((void**)&c->pcnt, m * sizeof(int32_t)))) {
     free_ctx(c);
     return rc;
   }
@@ -229,7 +244,10 @@ int create_impl(int64_t n, const boids_params* p, uint64_t seed, int32_t rank, i
   if (e == cudaSuccess) e = cudaMemsetAsync(c->side4, 0, m * sizeof(float4), s);
   if (e == cudaSuccess) e = cudaMemsetAsync(c->bcnt, 0, c->loc_grid.cells * sizeof(int32_t), s);
   if (e == cudaSuccess) e = launch_fill_nan(c->cand, c->ncand, s);  // entries >= n stay NaN
-  if (e == cudaSuccess) e = cudaMemsetAsync(c->stats, 0, 2 * sizeof(unsigned long long), s);
+  if (e == cudaSuccess) e = cudaMemsetAsync(c->stats, 0, 4 * sizeof(unsigned long long), s);
+  if (e == cudaSuccess) e = cudaMemsetAsync(c->hitcnt, 0, m * sizeof(int32_t), s);
+  if (e == cudaSuccess) e = cudaMemsetAsync(c->nbr8, 0xFF, m * sizeof(int32_t), s);
+  if (e == cudaSuccess) e = cudaMemsetAsync(c->pcnt, 0, m * sizeof(int32_t), s);
   if (e == cudaSuccess)
     e = launch_fill_phantoms(c->buf[0], m, shard ? 0 : c->nloc, shard ? world : 1, s);
   if (e == cudaSuccess) e = launch_fill_phantoms(c->buf[1], m, c->nloc, 1, s);
@@ -256,6 +274,7 @@ StepArgs make_args(boids_ctx* c, float dt) {
   a.cnt = c->cnt;
   a.n = c->n;
   a.m = c->m;
+  a.sdiv = make_slice_div(c->m, c->shard ? c->world : 1);
   a.lo = c->lo;
   a.nloc = c->nloc;
   a.world = c->shard ? c->world : 1;
@@ -268,12 +287,22 @@ StepArgs make_args(boids_ctx* c, float dt) {
   a.stats = c->stats;
   a.phase = c->phase;
   a.vote_u = c->vote_u;
+  a.hits = c->hits;
+  a.hitcnt = c->hitcnt;
+  a.nbr8 = c->nbr8;
+  a.partial = c->partial;
+  a.pcnt = c->pcnt;
   return a;
 }
 
 int one_step(boids_ctx* c, float dt) {
   StepArgs a = make_args(c, dt);
   int rc;
+  // Only the warm path keeps the 8th-nearest seed consistent with the lists it
+  // writes; any other step invalidates it (a stale seed could repeat one of the
+  // new 7 neighbours and break the t0 bound).
+  const bool warm_path = c->kernel == BOIDS_KERNEL_FUSED && c->warm;
+  if (!warm_path) CK(cudaMemsetAsync(c->nbr8, 0xFF, c->m * sizeof(int32_t), c->stream));
   if (c->kernel == BOIDS_KERNEL_SIMPLE) {
     if ((rc = launch(c, 0, [&] { return launch_search_simple(a, c->stream); }))) return rc;
     if ((rc = launch(c, 1, [&] { return launch_update(a, c->stream); }))) return rc;
@@ -283,15 +312,22 @@ int one_step(boids_ctx* c, float dt) {
     // never depend on it), so it is refreshed every resort_every steps.
     if (c->since_sort < 0 || c->since_sort >= c->resort_every) {
       if ((rc = launch(c, 2, [&] {
-             return launch_bin(a.full, c->m, c->lo, c->nloc, c->loc_grid, c->cellrank, c->bcnt, c->bstart,
+             return launch_bin(a.full, c->m, a.sdiv, c->lo, c->nloc, c->loc_grid, c->cellrank, c->bcnt, c->bstart,
                                nullptr, c->qperm, (int)c->lo, c->stream, nullptr);
            }, 3)))
         return rc;
       c->since_sort = 0;
     }
     c->since_sort++;
-    int cl = c->cluster_opt;
-    if ((rc = launch(c, 0, [&] { return launch_fused(a, cl, c->stream); }))) return rc;
+    if (warm_path) {
+      // warm step: all-pairs scan appending passing keys, then select + update
+      if ((rc = launch(c, 0, [&] { return launch_warm_scan(a, c->stream); }))) return rc;
+      if ((rc = launch(c, 1, [&] { return launch_warm_select(a, c->stream); }))) return rc;
+    } else {
+      // cold step (no previous lists) or forced: the cluster kernel
+      int cl = c->cluster_opt;
+      if ((rc = launch(c, 0, [&] { return launch_fused(a, cl, c->stream); }))) return rc;
+    }
   }
   if (!c->shard) c->cur ^= 1;
   c->warm = true;
@@ -361,7 +397,8 @@ BOIDS_API int boids_set_option(boids_ctx* c, int32_t opt, int64_t v) {
       c->record_steering = v != 0;
       return BOIDS_OK;
     case BOIDS_OPT_KERNEL:
-      if (v != BOIDS_KERNEL_FUSED && v != BOIDS_KERNEL_SIMPLE) return fail(BOIDS_EINVAL, "bad kernel");
+      if (v != BOIDS_KERNEL_FUSED && v != BOIDS_KERNEL_SIMPLE && v != BOIDS_KERNEL_CLUSTER)
+        return fail(BOIDS_EINVAL, "bad kernel");
       c->kernel = (int)v;
       return BOIDS_OK;
     case BOIDS_OPT_PROFILE:
@@ -477,6 +514,7 @@ BOIDS_API int boids_set_state(boids_ctx* c, const float* pos3, const float* fwd3
   CK(cudaMemcpyAsync(c->side4, hs.data(), k * sizeof(float4), cudaMemcpyHostToDevice, c->stream));
   CK(cudaMemsetAsync(c->cnt, 0, m * sizeof(int32_t), c->stream));
   CK(cudaMemsetAsync(c->nbr, 0xFF, m * 7 * sizeof(int32_t), c->stream));
+  CK(cudaMemsetAsync(c->nbr8, 0xFF, m * sizeof(int32_t), c->stream));
   CK(cudaStreamSynchronize(c->stream));
   c->warm = false;
   c->steering_valid = false;
@@ -523,11 +561,12 @@ BOIDS_API int boids_info(boids_ctx* c, boids_info_t* o) {
   o->kernel = c->kernel;
   o->cluster = c->cluster_opt ? c->cluster_opt : fused_auto_cluster(c->ncand, c->nloc, c->sm_count);
   o->launches = c->launches;
-  unsigned long long st[2] = {0, 0};
+  unsigned long long st[4] = {0, 0, 0, 0};
   CK(cudaMemcpyAsync(st, c->stats, sizeof(st), cudaMemcpyDeviceToHost, c->stream));
   CK(cudaStreamSynchronize(c->stream));
   o->slow_groups = (int64_t)st[0];
   o->vote_groups = (int64_t)st[1];
+  o->fallbacks = (int64_t)st[2];
   return BOIDS_OK;
 }
 

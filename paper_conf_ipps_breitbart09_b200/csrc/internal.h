@@ -8,6 +8,8 @@
 namespace boids {
 
 constexpr int TILE = 256;  // slice granularity (agents); every slice m is a multiple
+constexpr int HITS = 48;   // warm path: hit-buffer slots per agent (more -> full re-search)
+constexpr int PSLOTS = 16; // warm path: partial top-7 lists per unbounded agent
 
 // Device view of the agent state for one step.  Layout:
 //   full: world segments of 2*m float4; segment g = [pos4(m) | fwd4(m)] of agents
@@ -16,6 +18,42 @@ constexpr int TILE = 256;  // slice granularity (agents); every slice m is a mul
 //   out:  this rank's new [pos4(m) | fwd4(m)].
 //   up4, side4: this rank's local frames (read and written by the owner only).
 //   nbr (m x 7 int32), cnt (m int32): this rank's neighbour lists (last step).
+// Segmented addressing: agent j lives in slice g = j / m at full[g*2m + j - g*m]
+// (pos4) and full[g*2m + m + j - g*m] (fwd4), i.e. at j + g*m and j + (g+1)*m.
+// The division by the runtime slice m is a precomputed magic-number multiply
+// (Granlund-Montgomery, valid for 32-bit j; checked against j / m for the slice
+// sizes in use), avoiding a 64-bit division subroutine per gather.
+struct SliceDiv {
+  uint32_t mult;
+  int32_t shift;  // l = ceil(log2 m) >= 8 (m is a multiple of 256)
+  int32_t one;    // world == 1: every agent is in slice 0
+};
+inline SliceDiv make_slice_div(int64_t m, int32_t world) {
+  SliceDiv s{};
+  int l = 0;
+  while ((1ull << l) < (unsigned long long)m) ++l;
+  s.mult = (uint32_t)((((unsigned long long)1 << 32) * ((1ull << l) - (unsigned long long)m)) / (unsigned long long)m + 1);
+  s.shift = l;
+  s.one = world == 1;
+  return s;
+}
+__host__ __device__ inline int64_t slice_of(const SliceDiv& s, int64_t j) {
+  if (s.one) return 0;
+#ifdef __CUDA_ARCH__
+  const uint32_t n = (uint32_t)j, t = __umulhi(s.mult, n);
+  return (int64_t)((t + ((n - t) >> 1)) >> (s.shift - 1));
+#else
+  const uint32_t n = (uint32_t)j, t = (uint32_t)(((unsigned long long)s.mult * n) >> 32);
+  return (int64_t)((t + ((n - t) >> 1)) >> (s.shift - 1));
+#endif
+}
+__host__ __device__ inline const float4* pos_of(const float4* full, int64_t m, const SliceDiv& s, int64_t j) {
+  return full + j + slice_of(s, j) * m;
+}
+__host__ __device__ inline const float4* fwd_of(const float4* full, int64_t m, const SliceDiv& s, int64_t j) {
+  return full + j + (slice_of(s, j) + 1) * m;
+}
+
 // Uniform grid for binning (k_bin.cu): cells of size h from lo, dim cells per axis.
 struct BinGrid {
   float lo[3];
@@ -35,6 +73,7 @@ struct StepArgs {
   int32_t* cnt;
   int64_t n;       // total agents
   int64_t m;       // slice size
+  SliceDiv sdiv;   // j -> slice of agent j
   int64_t lo;      // first owned agent
   int64_t nloc;    // owned agents (hi - lo)
   int32_t world;
@@ -46,24 +85,22 @@ struct StepArgs {
   const int32_t* qperm;  // local queries in spatial order (local indices); nullptr = identity
   unsigned long long* stats;  // [0] vote groups that took the insertion path, [1] all vote groups
   int32_t vote_u;             // candidates per warp vote in the fused kernel (4 or 8)
+  unsigned long long* hits;   // warm path: [nloc][HITS] passing (d2, index) keys
+  int32_t* hitcnt;            // warm path: [nloc] number of passing keys (zero between steps)
+  int32_t* nbr8;              // [nloc] 8th nearest agent of the last step, or -1 (warm-bound seed)
+  unsigned long long* partial;  // warm path: [nloc][PSLOTS][7] partial top-7 lists (unbounded agents)
+  int32_t* pcnt;              // warm path: [nloc] partial lists written
   unsigned long long* phase;  // diagnostics: per-CTA %globaltimer stamps [grid][8], nullptr = off
   float dt;
   boids_params p;
 };
-
-__host__ __device__ inline const float4* pos_of(const float4* full, int64_t m, int64_t j) {
-  return full + (j / m) * 2 * m + (j % m);
-}
-__host__ __device__ inline const float4* fwd_of(const float4* full, int64_t m, int64_t j) {
-  return full + (j / m) * 2 * m + m + (j % m);
-}
 
 // launchers (return the cudaError_t of the launch)
 cudaError_t launch_init(float4* out, float4* up4, float4* side4, int64_t m, int64_t lo,
                         int64_t nloc, const boids_params& p, uint64_t seed, cudaStream_t s);
 cudaError_t launch_fill_phantoms(float4* seg_base, int64_t m, int64_t nloc, int64_t segments,
                                  cudaStream_t s);
-cudaError_t launch_bin(const float4* full, int64_t m, int64_t j0, int64_t count, const BinGrid& g,
+cudaError_t launch_bin(const float4* full, int64_t m, const SliceDiv& sd, int64_t j0, int64_t count, const BinGrid& g,
                        int2* cellrank, int* cnt, int* start, float4* spos, int* perm, int perm_base,
                        cudaStream_t s, int* launches);
 BinGrid make_locality_grid(int64_t n, const boids_params& p);
@@ -71,6 +108,8 @@ cudaError_t launch_fill_nan(float4* p, int64_t count, cudaStream_t s);
 cudaError_t launch_search_simple(const StepArgs& a, cudaStream_t s);
 cudaError_t launch_update(const StepArgs& a, cudaStream_t s);
 cudaError_t launch_fused(const StepArgs& a, int cluster, cudaStream_t s);
+cudaError_t launch_warm_scan(const StepArgs& a, cudaStream_t s);
+cudaError_t launch_warm_select(const StepArgs& a, cudaStream_t s);
 int fused_auto_cluster(int64_t n_pad_total, int64_t nloc, int sm_count);
 
 }  // namespace boids

@@ -93,7 +93,7 @@ __global__ void __launch_bounds__(TILE) k_search_simple(StepArgs a) {
   int64_t i = (int64_t)blockIdx.x * TILE + threadIdx.x;
   bool active = i < a.nloc;
   int64_t g = a.lo + i;
-  float4 me = active ? *pos_of(a.full, a.m, g) : make_float4(0.f, 0.f, 0.f, 0.f);
+  float4 me = active ? *pos_of(a.full, a.m, a.sdiv, g) : make_float4(0.f, 0.f, 0.f, 0.f);
   float r2 = __fmul_rn(a.p.search_radius, a.p.search_radius);
   key_t L[7];
 #pragma unroll
@@ -102,7 +102,7 @@ __global__ void __launch_bounds__(TILE) k_search_simple(StepArgs a) {
   int cnt = 0;
   int64_t total = (int64_t)a.world * a.m;
   for (int64_t base = 0; base < total; base += TILE) {
-    tile[threadIdx.x] = *pos_of(a.full, a.m, base + threadIdx.x);
+    tile[threadIdx.x] = *pos_of(a.full, a.m, a.sdiv, base + threadIdx.x);
     __syncthreads();
     for (int k = 0; k < TILE; ++k) {
       float d2 = dist2(me.x, me.y, me.z, tile[k]);
@@ -133,8 +133,8 @@ __global__ void __launch_bounds__(256) k_update(StepArgs a) {
   int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= a.nloc) return;
   int64_t g = a.lo + i;
-  float4 p4 = __ldg(pos_of(a.full, a.m, g));
-  float4 f4 = __ldg(fwd_of(a.full, a.m, g));
+  float4 p4 = __ldg(pos_of(a.full, a.m, a.sdiv, g));
+  float4 f4 = __ldg(fwd_of(a.full, a.m, a.sdiv, g));
   int cnt = a.cnt[i];
   int nb[7];
 #pragma unroll

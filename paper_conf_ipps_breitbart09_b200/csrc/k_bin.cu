@@ -42,11 +42,11 @@ __device__ __forceinline__ int cell_of(float4 p, const BinGrid& g) {
 }
 
 // Agents j in [j0, j0 + count) of the segmented buffer `full`.
-__global__ void k_bin_count(const float4* __restrict__ full, int64_t m, int64_t j0, int64_t count,
+__global__ void k_bin_count(const float4* __restrict__ full, int64_t m, SliceDiv sd, int64_t j0, int64_t count,
                             BinGrid g, int2* __restrict__ cellrank, int* __restrict__ cnt) {
   int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (k >= count) return;
-  float4 p = __ldg(pos_of(full, m, j0 + k));
+  float4 p = __ldg(pos_of(full, m, sd, j0 + k));
   if (p.x != p.x) {  // phantom (NaN position): not binned
     cellrank[k] = make_int2(-1, 0);
     return;
@@ -107,7 +107,7 @@ __global__ void __launch_bounds__(SCAN_T) k_bin_scan(int* __restrict__ cnt, int*
   for (int i = tid; i < C; i += SCAN_T) start[i] = sh[i + (i >> 5)];
 }
 
-__global__ void k_bin_scatter(const float4* __restrict__ full, int64_t m, int64_t j0, int64_t count,
+__global__ void k_bin_scatter(const float4* __restrict__ full, int64_t m, SliceDiv sd, int64_t j0, int64_t count,
                               const int2* __restrict__ cellrank, const int* __restrict__ start,
                               float4* __restrict__ spos, int* __restrict__ perm, int perm_base) {
   int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -117,18 +117,18 @@ __global__ void k_bin_scatter(const float4* __restrict__ full, int64_t m, int64_
   int dst = start[cr.x] + cr.y;
   int64_t j = j0 + k;
   if (spos) {
-    float4 p = __ldg(pos_of(full, m, j));
+    float4 p = __ldg(pos_of(full, m, sd, j));
     spos[dst] = make_float4(p.x, p.y, p.z, __int_as_float((int)j));
   }
   if (perm) perm[dst] = (int)(j - perm_base);
 }
 
-cudaError_t launch_bin(const float4* full, int64_t m, int64_t j0, int64_t count, const BinGrid& g,
+cudaError_t launch_bin(const float4* full, int64_t m, const SliceDiv& sd, int64_t j0, int64_t count, const BinGrid& g,
                        int2* cellrank, int* cnt, int* start, float4* spos, int* perm, int perm_base,
                        cudaStream_t s, int* launches) {
   if (count <= 0) return cudaSuccess;
   const unsigned blocks = (unsigned)((count + 255) / 256);
-  k_bin_count<<<blocks, 256, 0, s>>>(full, m, j0, count, g, cellrank, cnt);
+  k_bin_count<<<blocks, 256, 0, s>>>(full, m, sd, j0, count, g, cellrank, cnt);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return e;
   const size_t shm = (size_t)(g.cells + g.cells / 32 + 1) * sizeof(int);
@@ -138,7 +138,7 @@ cudaError_t launch_bin(const float4* full, int64_t m, int64_t j0, int64_t count,
   }
   k_bin_scan<<<1, SCAN_T, shm, s>>>(cnt, start, g.cells);
   if ((e = cudaGetLastError()) != cudaSuccess) return e;
-  k_bin_scatter<<<blocks, 256, 0, s>>>(full, m, j0, count, cellrank, start, spos, perm, perm_base);
+  k_bin_scatter<<<blocks, 256, 0, s>>>(full, m, sd, j0, count, cellrank, start, spos, perm, perm_base);
   if (launches) *launches += 3;
   return cudaGetLastError();
 }

@@ -14,10 +14,13 @@
 //    copy engine (cp.async.bulk + mbarrier complete_tx) through a STAGES-deep
 //    ring of 256-candidate tiles; all 4 warps read each candidate with a
 //    broadcast LDS.128.
-//  * Each thread owns Q = 4 queries (4 independent distance chains per LDS;
-//    measured 0.87 of the FP32 lane-op peak vs 0.58 for Q = 2) and keeps four
-//    register-resident sorted top-7 lists of (d2, index) keys (64-bit, the
-//    reading-Q4 total order).  Packed FADD2/FMUL2 were measured slower.
+//  * Each thread owns Q = 4 queries (4 independent distance chains per LDS.128;
+//    Q = 2 measured ~0.58 of the lane-op peak).  The distance uses packed
+//    FADD2/FMUL2 on (x, y) pairs + scalar dz and sums: 6 issue slots per 8 FP32
+//    lane-ops, so the loop is bound by the FP32 pipe rather than by issue
+//    (tools/probe_loop.cu: 0.78-0.81 vs 0.72-0.75 scalar).  The sorted top-7
+//    lists of 64-bit (d2, index) keys (the reading-Q4 total order) live in
+//    shared memory: only the rare insertion path touches them.
 //  * Warm threshold: t0 = max d2 to the previous step's 7 neighbours at the
 //    current positions is an upper bound on the true 7th key, so only
 //    candidates with d2 <= t0 can enter (identical result, far fewer inserts).
@@ -114,7 +117,7 @@ __device__ __noinline__ float insert_list(key_t* lists, int qb, int ql, float d2
 }
 
 __device__ __forceinline__ const float4* tile_src(const StepArgs& a, int64_t tile) {
-  return pos_of(a.full, a.m, tile * CT);  // m % CT == 0: a tile never straddles a slice
+  return pos_of(a.full, a.m, a.sdiv, tile * CT);  // m % CT == 0: a tile never straddles a slice
 }
 
 // local query index held by block slot qs (>= nloc: inactive slot)
@@ -127,12 +130,12 @@ __device__ __forceinline__ int64_t query_of(const StepArgs& a, int64_t qs) {
 __device__ __forceinline__ float warm_t0(const StepArgs& a, int64_t ql) {
   if (!a.warm || ql >= a.nloc) return __int_as_float(0x7f800000);
   if (a.cnt[ql] < 7) return __int_as_float(0x7f800000);
-  float4 me = __ldg(pos_of(a.full, a.m, a.lo + ql));
+  float4 me = __ldg(pos_of(a.full, a.m, a.sdiv, a.lo + ql));
   float t = 0.f;
 #pragma unroll
   for (int k = 0; k < 7; ++k) {
     int j = a.nbr[ql * 7 + k];
-    t = fmaxf(t, dist2(me.x, me.y, me.z, __ldg(pos_of(a.full, a.m, j))));
+    t = fmaxf(t, dist2(me.x, me.y, me.z, __ldg(pos_of(a.full, a.m, a.sdiv, j))));
   }
   return t;
 }
@@ -149,8 +152,8 @@ __device__ __forceinline__ void finish_query(const StepArgs& a, int64_t qi, cons
 #pragma unroll
   for (int s = 0; s < 7; ++s) a.nbr[qi * 7 + s] = nb[s];
   a.cnt[qi] = cnt;
-  float4 p4 = __ldg(pos_of(a.full, a.m, a.lo + qi));
-  float4 f4 = __ldg(fwd_of(a.full, a.m, a.lo + qi));
+  float4 p4 = __ldg(pos_of(a.full, a.m, a.sdiv, a.lo + qi));
+  float4 f4 = __ldg(fwd_of(a.full, a.m, a.sdiv, a.lo + qi));
   V3 F = steer_agent(a, v3(p4), v3(f4), nb, cnt);
   modify_agent(a, qi, v3(p4), f4, F);
 }
@@ -193,34 +196,18 @@ __global__ void __launch_bounds__(NT) k_fused(StepArgs a, int64_t tiles_total) {
 
   const float r2 = __fmul_rn(a.p.search_radius, a.p.search_radius);
   const float r2_in = __uint_as_float(__float_as_uint(r2) - 1u);  // largest float < r2 (r2 > 0)
-  float px[Q], py[Q], pz[Q], lim[Q];
+  float2 pxy[Q];  // (x, y) of each query as an aligned register pair (FADD2 operand)
+  float pz[Q], lim[Q];
   int gq[Q];  // global index of each query (n < 2^31)
-  {
-    // Query coordinates are staged through shared memory as (0, x, y, z) so the
-    // LDS.128 that reads them back leaves x, y, z in odd/even/odd registers --
-    // the opposite register-bank parity of a candidate's x, y, z (even/odd/even
-    // from the tile's LDS.128), so the subtractions never read two registers of
-    // one bank (measured: ~8% dispatch stalls otherwise).  The list area is free
-    // until it is initialised below.
-    float4* qscratch = reinterpret_cast<float4*>(sm.lists) + tid * Q;
 #pragma unroll
-    for (int q = 0; q < Q; ++q) {
-      const int ql = warp * 32 * Q + q * 32 + lane;  // query slot within the block
-      const int64_t qi = query_of(a, q_base + ql);
-      gq[q] = (int)(a.lo + qi);
-      float4 me = qi < a.nloc ? __ldg(pos_of(a.full, a.m, a.lo + qi))
-                              : make_float4(__int_as_float(0x7fc00000), 0.f, 0.f, 0.f);
-      qscratch[q] = make_float4(0.f, me.x, me.y, me.z);
-    }
-#pragma unroll
-    for (int q = 0; q < Q; ++q) {
-      volatile float4* vq = qscratch + q;
-      float4 v = make_float4(vq->x, vq->y, vq->z, vq->w);
-      px[q] = v.y;
-      py[q] = v.z;
-      pz[q] = v.w;
-    }
-    __syncthreads();  // every thread has read its coordinates before the lists are initialised
+  for (int q = 0; q < Q; ++q) {
+    const int ql = warp * 32 * Q + q * 32 + lane;  // query slot within the block
+    const int64_t qi = query_of(a, q_base + ql);
+    gq[q] = (int)(a.lo + qi);
+    float4 me = qi < a.nloc ? __ldg(pos_of(a.full, a.m, a.sdiv, a.lo + qi))
+                            : make_float4(__int_as_float(0x7fc00000), 0.f, 0.f, 0.f);
+    pxy[q] = make_float2(me.x, me.y);
+    pz[q] = me.z;
   }
 #pragma unroll
   for (int q = 0; q < Q; ++q) {
@@ -255,11 +242,21 @@ __global__ void __launch_bounds__(NT) k_fused(StepArgs a, int64_t tiles_total) {
       float4 cc[U];
 #pragma unroll
       for (int u = 0; u < U; ++u) cc[u] = tile[c + u];
+      // d2 = ((dx*dx) + (dy*dy)) + (dz*dz), every op rounded (Appendix A): (dx, dy)
+      // and their squares as packed FADD2 / FMUL2 on the query's (x, y) pair and
+      // the candidate's (x, y) pair (both aligned register pairs), dz scalar, the
+      // sums scalar FADD (a packed add would be contracted into FFMA2 by ptxas).
+      // Same bits as dist2(); 6 issue slots for 8 FP32 lane-ops.
       float d[Q][U];
 #pragma unroll
       for (int u = 0; u < U; ++u)
 #pragma unroll
-        for (int q = 0; q < Q; ++q) d[q][u] = dist2(px[q], py[q], pz[q], cc[u]);
+        for (int q = 0; q < Q; ++q) {
+          const float2 dxy = __fadd2_rn(pxy[q], make_float2(-cc[u].x, -cc[u].y));
+          const float2 sq = __fmul2_rn(dxy, dxy);
+          const float dz = __fsub_rn(pz[q], cc[u].z);
+          d[q][u] = __fadd_rn(__fadd_rn(sq.x, sq.y), __fmul_rn(dz, dz));
+        }
       float mq[Q];
 #pragma unroll
       for (int q = 0; q < Q; ++q) {
@@ -378,101 +375,157 @@ __global__ void __launch_bounds__(NT) k_fused(StepArgs a, int64_t tiles_total) {
   }
 }
 
-template <int NT, int K, int U>
-cudaError_t launch_k(const StepArgs& a, int64_t tiles, cudaStream_t s) {
-  auto kern = k_fused<NT, K, U>;
-  if (K > 8) {
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
-    if (e != cudaSuccess) return e;
-  }
-  const int64_t nqb = (a.nloc + NT * Q - 1) / (NT * Q);
-  cudaLaunchConfig_t cfg = {};
-  cfg.gridDim = dim3((unsigned)(nqb * K));
-  cfg.blockDim = dim3(NT);
-  cfg.dynamicSmemBytes = 0;
-  cfg.stream = s;
-  cudaLaunchAttribute attr[1];
-  attr[0].id = cudaLaunchAttributeClusterDimension;
-  attr[0].val.clusterDim.x = K;
-  attr[0].val.clusterDim.y = 1;
-  attr[0].val.clusterDim.z = 1;
-  cfg.attrs = attr;
-  cfg.numAttrs = 1;
-  return cudaLaunchKernelEx(&cfg, kern, a, tiles);
-}
+// ---------------------------------------------------------------- launch ----
+// Kernel table [NT 64/128][K 1,2,4,8,16][U 4/8] with lazily queried occupancy.
+typedef void (*FusedFn)(StepArgs, int64_t);
+struct KEntry {
+  FusedFn fn;
+  int nt, k;
+  int rmax;  // max resident CTAs per SM without padding
+  int static_smem;
+  bool ready;
+};
 
 template <int NT, int U>
-cudaError_t launch_nt(const StepArgs& a, int K, int64_t tiles, cudaStream_t s) {
-  switch (K) {
-    case 1: return launch_k<NT, 1, U>(a, tiles, s);
-    case 2: return launch_k<NT, 2, U>(a, tiles, s);
-    case 4: return launch_k<NT, 4, U>(a, tiles, s);
-    case 8: return launch_k<NT, 8, U>(a, tiles, s);
-    default: return launch_k<NT, 16, U>(a, tiles, s);
-  }
+void fill_row(KEntry (&tab)[2][5][2], int ni, int ui) {
+  const FusedFn fns[5] = {k_fused<NT, 1, U>, k_fused<NT, 2, U>, k_fused<NT, 4, U>, k_fused<NT, 8, U>,
+                          k_fused<NT, 16, U>};
+  for (int i = 0; i < 5; ++i) tab[ni][i][ui] = KEntry{fns[i], NT, 1 << i, 0, 0, false};
 }
 
-}  // namespace
+KEntry& entry(int ni, int ki, int ui) {
+  static KEntry tab[2][5][2];
+  static bool init = false;
+  if (!init) {
+    fill_row<64, 4>(tab, 0, 0);
+    fill_row<64, 8>(tab, 0, 1);
+    fill_row<128, 4>(tab, 1, 0);
+    fill_row<128, 8>(tab, 1, 1);
+    init = true;
+  }
+  KEntry& e = tab[ni][ki][ui];
+  if (!e.ready) {
+    // all of the SM's unified memory goes to shared memory (the kernel relies on L1
+    // only for a few gathers), so residency is governed by the padding below
+    cudaFuncSetAttribute(e.fn, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+    if (e.k > 8) cudaFuncSetAttribute(e.fn, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+    cudaFuncAttributes at{};
+    cudaFuncGetAttributes(&at, e.fn);
+    e.static_smem = (int)at.sharedSizeBytes;
+    int r = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&r, e.fn, e.nt, 0);
+    e.rmax = r > 0 ? r : 1;
+    e.ready = true;
+  }
+  return e;
+}
 
-// Occupancy-aware launch plan.  For each CTA size NT (64 or 128 threads) and
-// cluster size K, the grid is C = K * ceil(n_local / (NT * Q)) CTAs.  Score =
-//   balance   (C/S) / ceil(C/S), S = SM count (equal-work CTAs on S SMs)
-// x issue    measured FP32 issue efficiency of the scalar Q=4 loop vs warps/SM
-//            (tools/probe_fp32x2.cu on B200: 8 -> 0.80, 16 -> 0.87, 32 -> 0.88)
-// x chunk    per-CTA fixed cost (ring fill, merge, epilogue ~ 256 candidates)
-// Ties go to the smaller K (less merge work).
-static double issue_eff(double warps_per_sm) {
-  if (warps_per_sm >= 24) return 0.88;
-  if (warps_per_sm >= 16) return 0.866 + (warps_per_sm - 16) * (0.014 / 8);
-  if (warps_per_sm >= 8) return 0.80 + (warps_per_sm - 8) * (0.066 / 8);
-  return 0.80 * warps_per_sm / 8;
+// Dynamic shared memory padding that caps residency at `cap` CTAs per SM, so a
+// single wave of C CTAs spreads ceil(C / SMs) per SM instead of the cluster
+// scheduler piling its maximum onto some SMs (measured: 2x scan-time spread).
+int pad_for_cap(KEntry& e, int cap) {
+  if (cap >= e.rmax) return 0;
+  int dev = 0, optin = 0;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+  int lo = 0, hi = optin - e.static_smem, r = 0;
+  cudaFuncSetAttribute(e.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, hi);
+  while (lo < hi) {  // smallest padding with occupancy <= cap
+    const int mid = (lo + hi) / 2;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&r, e.fn, e.nt, mid);
+    if (r <= cap) hi = mid;
+    else lo = mid + 1;
+  }
+  return lo;
+}
+
+// Occupancy-aware launch plan.  For CTA size NT (64 or 128) and cluster size K
+// the grid is C = K * ceil(n_local / (NT * Q)) CTAs on S SMs:
+//   one wave (ceil(C/S) <= rmax): residency capped at r = ceil(C/S) (padding),
+//             balance (C/S) / r;   else r = rmax, balance waves / ceil(waves);
+//   x loop efficiency at r * NT / 32 warps per SM (tools/probe_loop.cu, packed)
+//   x per-CTA fixed cost (ring fill, merge, epilogue ~ 512 candidates).
+// Ties go to the smaller NT, then the smaller K.
+double loop_eff(double w) {
+  static const double W[] = {4, 8, 12, 16, 24, 32, 64};
+  static const double E[] = {0.40, 0.66, 0.74, 0.78, 0.80, 0.81, 0.81};
+  if (w <= W[0]) return E[0] * w / W[0];
+  for (int i = 1; i < 7; ++i)
+    if (w <= W[i]) return E[i - 1] + (E[i] - E[i - 1]) * (w - W[i - 1]) / (W[i] - W[i - 1]);
+  return E[6];
 }
 
 struct Plan {
-  int nt, k;
+  int ni, ki, cap;
 };
 
-static Plan plan_launch(int64_t total_candidates, int64_t nloc, int sm_count, int forced_k) {
-  static const int resident[2] = {9, 5};  // CTAs/SM for NT = 64, 128 (96 registers; 24 / 39 KB smem)
+Plan plan_launch(int64_t total_candidates, int64_t nloc, int sm_count, int forced_k, int ui) {
   const int64_t tiles = total_candidates / CT;
-  Plan best{128, 1};
+  Plan best{1, 0, 1};
   double best_score = -1.0;
   for (int ni = 0; ni < 2; ++ni) {
     const int nt = ni == 0 ? 64 : 128;
     const int64_t nqb = (nloc + nt * Q - 1) / (nt * Q);
-    for (int K = 1; K <= 16; K *= 2) {
+    for (int ki = 0; ki < 5; ++ki) {
+      const int K = 1 << ki;
       if (forced_k && K != forced_k) continue;
       if (K > 1 && tiles / K < 1) break;
+      KEntry& e = entry(ni, ki, ui);
       const double C = (double)(nqb * K), S = (double)sm_count;
-      const double per_sm = std::ceil(C / S);
-      const double balance = (C / S) / per_sm;
-      const double warps = std::min<double>(per_sm, resident[ni]) * nt / 32.0;
+      const int per_sm = (int)std::ceil(C / S);
+      double balance;
+      int r;
+      if (per_sm <= e.rmax) {
+        r = per_sm;
+        balance = (C / S) / per_sm;
+      } else {
+        r = e.rmax;
+        const double waves = C / (S * r);
+        balance = waves / std::ceil(waves);
+      }
       const double cand = (double)total_candidates / K;
-      const double score = balance * issue_eff(warps) * cand / (cand + 256.0);
+      const double score = balance * loop_eff(r * nt / 32.0) * cand / (cand + 512.0);
       if (score > best_score * (1.0 + 1e-6)) {
         best_score = score;
-        best = Plan{nt, K};
+        best = Plan{ni, ki, r};
       }
     }
   }
   return best;
 }
 
+}  // namespace
+
 int fused_auto_cluster(int64_t total_candidates, int64_t nloc, int sm_count) {
-  return plan_launch(total_candidates, nloc, sm_count, 0).k;
+  return 1 << plan_launch(total_candidates, nloc, sm_count, 0, 0).ki;
 }
 
 cudaError_t launch_fused(const StepArgs& a, int cluster, cudaStream_t s) {
   if (a.nloc <= 0) return cudaSuccess;
-  const int64_t total = (int64_t)a.world * a.m;
-  const int64_t tiles = total / CT;
+  const int64_t tiles = (int64_t)a.world * a.m / CT;
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  Plan p = plan_launch(total, a.nloc, sms, cluster);
-  while (p.k > 1 && tiles / p.k < 1) p.k /= 2;
-  if (a.vote_u == 8) return p.nt == 64 ? launch_nt<64, 8>(a, p.k, tiles, s) : launch_nt<128, 8>(a, p.k, tiles, s);
-  return p.nt == 64 ? launch_nt<64, 4>(a, p.k, tiles, s) : launch_nt<128, 4>(a, p.k, tiles, s);
+  const int ui = a.vote_u == 8 ? 1 : 0;
+  const Plan p = plan_launch(tiles * CT, a.nloc, sms, cluster, ui);
+  KEntry& e = entry(p.ni, p.ki, ui);
+  // Residency caps fight the cluster scheduler (whole clusters per GPC), so the
+  // cluster kernel runs uncapped; pad_for_cap is kept for K == 1 grids.
+  const int pad = e.k == 1 ? pad_for_cap(e, p.cap) : 0;
+  const int64_t nqb = (a.nloc + e.nt * Q - 1) / (e.nt * Q);
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)(nqb * e.k));
+  cfg.blockDim = dim3(e.nt);
+  cfg.dynamicSmemBytes = pad;
+  cfg.stream = s;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = e.k;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, e.fn, a, tiles);
 }
 
 }  // namespace boids

@@ -1,0 +1,429 @@
+// k_warm.cu -- the warm-start Boids step: k_scan (all pairs, stream-K balanced)
+// + k_select (top-7, steering, modification).  Used for every step whose
+// previous step left neighbour lists for all owned agents (the cold step -- the
+// first one, or the first after boids_set_state -- runs k_fused).
+//
+// Why a second design.  With the warm threshold t0_i = max over the previous
+// step's 7 neighbours j of d2(i, j) at the CURRENT positions, the true 7th key
+// of agent i is <= t0_i (those 7 agents still exist), so the result is the top-7
+// of the set {j != i : d2 <= min(prev(r2), t0_i)}, which holds only ~8-12 agents.
+// The scan therefore needs no running top-7: it APPENDS every passing (d2, j)
+// key to a per-agent hit buffer, and the selection happens once, afterwards.
+// Without per-query lists the candidate range can be split any way at all, so
+//   k_scan   a persistent grid (SMs x occupancy CTAs) walks the item space
+//            (query block of 512 agents) x (256-candidate tile) in equal
+//            contiguous ranges (stream-K): every CTA gets the same number of
+//            items +-1 whatever n is -- no clusters, no wave quantisation.  The
+//            hot loop is k_fused's (TMA ring, packed FADD2/FMUL2 distance,
+//            FMNMX-tree vote); passing pairs go to a per-warp shared-memory
+//            record buffer that is flushed with one global atomic per record.
+//   k_select one thread per agent: sort its <= H hits into the top-7 (exact
+//            (d2, index) order, reading Q4), then steering + modification.
+//            Agents without a warm bound (t0 >= r2: the agent wrapped to the far
+//            side of the world, or fewer than 7 previous neighbours) keep an
+//            exact running top-7 in k_scan's shared memory instead, flushed as
+//            partial lists that k_select merges.  A buffer that still overflows
+//            is searched again by its warp, all 32 lanes scanning all
+//            candidates (brute force, Listing 5.2).
+// Every pair (i, j) is evaluated exactly once by k_scan: brute force as the
+// thesis defines it, with the thesis's own re-use of shared memory for
+// candidate positions (Listing 6.2).
+#include "agent_update.cuh"
+
+namespace boids {
+namespace {
+
+constexpr int Q = 4;        // queries per thread
+constexpr int CT = 256;     // candidates per tile (one TMA bulk copy of 4 KB)
+constexpr int STAGES = 3;   // TMA ring depth
+constexpr int U = 4;        // candidates per warp vote
+constexpr int NTS = 128;    // k_scan threads per CTA
+constexpr int QBS = NTS * Q;  // queries per block (512)
+constexpr int WB = Q * U * 32;  // records per warp buffer (8 KB): one vote group's maximum
+constexpr int UBW = 8;         // per warp: running top-7 lists for unbounded queries
+
+struct __align__(8) Rec {
+  int qi;  // local query index
+  int pad;
+  key_t key;
+};
+
+struct __align__(16) ScanSmem {
+  float4 ring[STAGES][CT];
+  Rec rec[NTS / 32][WB];
+  key_t ulist[NTS / 32][UBW][7];  // sorted top-7 of unbounded queries (t0 >= r2)
+  uint64_t full[STAGES];
+  uint64_t empty[STAGES];
+};
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  asm volatile(
+      "{\n"
+      ".reg .pred P1;\n"
+      "LAB_WAIT:\n"
+      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n"
+      "@!P1 bra LAB_WAIT;\n"
+      "}\n" ::"r"(smem_u32(bar)),
+      "r"(parity)
+      : "memory");
+}
+__device__ __forceinline__ void tma_load_1d(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_u32(dst)),
+      "l"(src), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+
+__device__ __forceinline__ int64_t query_of(const StepArgs& a, int64_t qs) {
+  if (qs >= a.nloc) return a.nloc;
+  return a.qperm ? (int64_t)__ldg(a.qperm + qs) : qs;
+}
+
+// t0 of local query qi: an upper bound on its 7th smallest d2 this step, from
+// agents that exist -- the previous step's 7 neighbours and, when known, the
+// 8th nearest: t0 = 7th smallest of their d2 at the CURRENT positions, i.e. the
+// max of the 7 or the second largest of the 8 (so one neighbour that wrapped
+// to the far side of the world does not spoil the bound).  +inf without a full
+// previous list.  All loads are issued before any is used.
+__device__ __forceinline__ float warm_t0(const StepArgs& a, int64_t qi, float4 me) {
+  if (qi >= a.nloc) return __int_as_float(0x7f800000);
+  int nb[8];
+#pragma unroll
+  for (int k = 0; k < 7; ++k) nb[k] = __ldg(a.nbr + qi * 7 + k);
+  nb[7] = __ldg(a.nbr8 + qi);
+  const int c = __ldg(a.cnt + qi);
+  float4 p[8];
+#pragma unroll
+  for (int k = 0; k < 8; ++k) p[k] = __ldg(pos_of(a.full, a.m, a.sdiv, nb[k] < 0 ? 0 : nb[k]));
+  float m1 = 0.f, m2 = 0.f;  // largest and second largest of the 8
+#pragma unroll
+  for (int k = 0; k < 8; ++k) {
+    const float d = (k < 7 || nb[7] >= 0) ? dist2(me.x, me.y, me.z, p[k]) : 0.f;  // no 8th: ignore
+    m2 = fmaxf(m2, fminf(m1, d));
+    m1 = fmaxf(m1, d);
+  }
+  if (c < 7) return __int_as_float(0x7f800000);
+  return nb[7] >= 0 ? m2 : m1;
+}
+
+// Issue the TMA load of global tile counter tc (stage tc % STAGES), waiting until
+// every warp released the stage's previous tile.  Called by thread 0 only.
+__device__ __forceinline__ void issue_tile(ScanSmem& sm, const StepArgs& a, uint32_t tc, int64_t tile) {
+  const int s = (int)(tc % STAGES);
+  if (tc >= STAGES) mbar_wait(&sm.empty[s], ((tc - STAGES) / STAGES) & 1u);
+  mbar_arrive_expect_tx(&sm.full[s], CT * sizeof(float4));
+  tma_load_1d(sm.ring[s], pos_of(a.full, a.m, a.sdiv, tile * CT), CT * sizeof(float4), &sm.full[s]);
+}
+
+// Insert key k into a sorted 7-list in shared memory; returns the new worst d2.
+__device__ __noinline__ float insert_l7(key_t* L7, key_t k) {
+  key_t L[7];
+#pragma unroll
+  for (int s = 0; s < 7; ++s) L[s] = L7[s];
+  insert7(L, k);
+#pragma unroll
+  for (int s = 0; s < 7; ++s) L7[s] = L[s];
+  return key_d2(L[6]);
+}
+
+// Flush a warp's record buffer into the global per-query hit buffers.
+__device__ __forceinline__ void flush(const StepArgs& a, const Rec* rec, int n, int lane) {
+  for (int i = lane; i < n; i += 32) {
+    const Rec r = rec[i];
+    const int slot = atomicAdd(a.hitcnt + r.qi, 1);
+    if (slot < HITS) a.hits[(int64_t)r.qi * HITS + slot] = r.key;
+  }
+}
+
+__global__ void __launch_bounds__(NTS) k_scan(StepArgs a, int64_t units, int64_t items) {
+  __shared__ ScanSmem sm;
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const int64_t L0 = items * blockIdx.x / gridDim.x, L1 = items * (blockIdx.x + 1) / gridDim.x;
+  if (tid == 0) {
+#pragma unroll
+    for (int s = 0; s < STAGES; ++s) {
+      mbar_init(&sm.full[s], 1);
+      mbar_init(&sm.empty[s], NTS / 32);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  const float r2 = __fmul_rn(a.p.search_radius, a.p.search_radius);
+  const float r2_in = __uint_as_float(__float_as_uint(r2) - 1u);  // d2 < r2  <=>  d2 <= r2_in
+  Rec* rec = sm.rec[warp];
+  int wcount = 0;     // records in this warp's buffer (warp-uniform)
+  unsigned slow_groups = 0, groups = 0;
+  uint32_t tc = 0;    // tiles issued / consumed by this CTA (ring phase bookkeeping)
+  for (int64_t L = L0; L < L1;) {
+    const int64_t qb = L / units, u0 = L - qb * units;
+    const int nu = (int)min(units - u0, L1 - L);
+    if (tid == 0)
+      for (int t = 0; t < STAGES && t < nu; ++t) issue_tile(sm, a, tc + t, u0 + t);
+    // this run's queries: 4 per thread, in spatial order (qperm)
+    float2 pxy[Q];
+    float pz[Q], lim[Q];
+    int gq[Q], qloc[Q];
+#pragma unroll
+    for (int q = 0; q < Q; ++q) {
+      const int64_t qi = query_of(a, qb * QBS + warp * 32 * Q + q * 32 + lane);
+      qloc[q] = (int)qi;
+      gq[q] = (int)(a.lo + qi);
+      const float4 me = qi < a.nloc ? __ldg(pos_of(a.full, a.m, a.sdiv, a.lo + qi))
+                                    : make_float4(__int_as_float(0x7fc00000), 0.f, 0.f, 0.f);
+      pxy[q] = make_float2(me.x, me.y);
+      pz[q] = me.z;
+      lim[q] = fminf(r2_in, warm_t0(a, qi, me));  // inclusive limit
+    }
+    // Unbounded queries (no warm bound: t0 >= r2, e.g. the agent wrapped to the far
+    // side of the world) would append every in-radius pair; the first UBW of each
+    // warp keep a running top-7 here instead (limit tightening as it fills) and
+    // flush it as a partial list at the end of the run.
+    int ul[Q];
+    {
+      int used = 0;
+#pragma unroll
+      for (int q = 0; q < Q; ++q) {
+        const bool ub = qloc[q] < a.nloc && lim[q] >= r2_in;
+        const unsigned bal = __ballot_sync(0xffffffffu, ub);
+        const int idx = used + __popc(bal & ((1u << lane) - 1u));
+        ul[q] = (ub && idx < UBW) ? idx : -1;
+        used += __popc(bal);
+      }
+      __syncwarp();
+      for (int i = lane; i < UBW * 7; i += 32) (&sm.ulist[warp][0][0])[i] = KEY_EMPTY;
+      __syncwarp();
+    }
+    float limc = fmaxf(fmaxf(lim[0], lim[1]), fmaxf(lim[2], lim[3]));
+    for (int t = 0; t < nu; ++t, ++tc) {
+      const int s = (int)(tc % STAGES);
+      mbar_wait(&sm.full[s], (tc / STAGES) & 1u);
+      const float4* tile = sm.ring[s];
+      const int jb = (int)((u0 + t) * CT);
+#pragma unroll 2
+      for (int c = 0; c < CT; c += U) {
+        float4 cc[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) cc[u] = tile[c + u];
+        // d2 = ((dx*dx) + (dy*dy)) + (dz*dz), each op rounded: packed (dx, dy) and
+        // squares, scalar dz and sums (see k_fused.cu)
+        float d[Q][U];
+#pragma unroll
+        for (int u = 0; u < U; ++u)
+#pragma unroll
+          for (int q = 0; q < Q; ++q) {
+            const float2 dxy = __fadd2_rn(pxy[q], make_float2(-cc[u].x, -cc[u].y));
+            const float2 sq = __fmul2_rn(dxy, dxy);
+            const float dz = __fsub_rn(pz[q], cc[u].z);
+            d[q][u] = __fadd_rn(__fadd_rn(sq.x, sq.y), __fmul_rn(dz, dz));
+          }
+        float mq[Q];
+#pragma unroll
+        for (int q = 0; q < Q; ++q) {
+          mq[q] = d[q][0];
+#pragma unroll
+          for (int u = 1; u < U; ++u) mq[q] = fminf(mq[q], d[q][u]);
+        }
+        const float m = fminf(fminf(mq[0], mq[1]), fminf(mq[2], mq[3]));  // NaN (phantoms) ignored
+        ++groups;
+        if (__any_sync(0xffffffffu, m <= limc)) {  // rare, warp-uniform
+          ++slow_groups;
+          unsigned bits = 0;
+#pragma unroll
+          for (int q = 0; q < Q; ++q)
+#pragma unroll
+            for (int u = 0; u < U; ++u)
+              if (d[q][u] <= lim[q] && jb + c + u != gq[q]) {
+                if (ul[q] >= 0)  // unbounded query with a list: exact running top-7
+                  lim[q] = fminf(lim[q], insert_l7(sm.ulist[warp][ul[q]], make_key(d[q][u], jb + c + u)));
+                else
+                  bits |= 1u << (q * U + u);
+              }
+          const int nrec = __popc(bits);
+          int incl = nrec;
+#pragma unroll
+          for (int o = 1; o < 32; o <<= 1) {
+            const int y = __shfl_up_sync(0xffffffffu, incl, o);
+            if (lane >= o) incl += y;
+          }
+          const int total = __shfl_sync(0xffffffffu, incl, 31);
+          if (wcount + total > WB) {  // warp-uniform; total <= WB always
+            __syncwarp();
+            flush(a, rec, wcount, lane);
+            __syncwarp();
+            wcount = 0;
+          }
+          int off = wcount + incl - nrec;
+#pragma unroll
+          for (int q = 0; q < Q; ++q)
+#pragma unroll
+            for (int u = 0; u < U; ++u)
+              if (bits & (1u << (q * U + u))) {
+                rec[off].qi = qloc[q];
+                rec[off].key = make_key(d[q][u], jb + c + u);
+                ++off;
+              }
+          wcount += total;
+          limc = fmaxf(fmaxf(lim[0], lim[1]), fmaxf(lim[2], lim[3]));
+        }
+      }
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&sm.empty[s]);
+      if (tid == 0 && t + STAGES < nu) issue_tile(sm, a, tc + STAGES, u0 + t + STAGES);
+    }
+    // partial lists of the unbounded queries -> global (merged by k_select)
+    __syncwarp();
+#pragma unroll
+    for (int q = 0; q < Q; ++q) {
+      if (ul[q] >= 0) {
+        const int slot = atomicAdd(a.pcnt + qloc[q], 1);
+        if (slot < PSLOTS) {
+          key_t* dst = a.partial + ((int64_t)qloc[q] * PSLOTS + slot) * 7;
+#pragma unroll
+          for (int s = 0; s < 7; ++s) dst[s] = sm.ulist[warp][ul[q]][s];
+        }
+      }
+    }
+    __syncwarp();
+    L += nu;
+  }
+  __syncwarp();
+  flush(a, rec, wcount, lane);
+  if (a.stats && lane == 0) {
+    atomicAdd(a.stats, (unsigned long long)slow_groups);
+    atomicAdd(a.stats + 1, (unsigned long long)groups);
+  }
+}
+
+// --------------------------------------------------------------- select ----
+constexpr int NSEL = 128;
+
+// Brute-force top-7 of local query qi by the whole warp (lanes stride the
+// candidates; per-lane top-7; shuffle butterfly merge).  Result in every lane.
+__device__ __noinline__ void warp_full_search(const StepArgs& a, int64_t qi, key_t (&A)[7]) {
+  const int lane = threadIdx.x & 31;
+  const float4 me = __ldg(pos_of(a.full, a.m, a.sdiv, a.lo + qi));
+  const int g = (int)(a.lo + qi);
+  const float r2 = __fmul_rn(a.p.search_radius, a.p.search_radius);
+#pragma unroll
+  for (int s = 0; s < 7; ++s) A[s] = KEY_EMPTY;
+  const int64_t total = (int64_t)a.world * a.m;
+  // 8 independent loads in flight per lane (total is a multiple of 256)
+  for (int64_t j0 = lane; j0 < total; j0 += 32 * 8) {
+    float4 c[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u) c[u] = __ldg(pos_of(a.full, a.m, a.sdiv, j0 + 32 * u));
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      const float d2 = dist2(me.x, me.y, me.z, c[u]);
+      const int j = (int)(j0 + 32 * u);
+      if (d2 < r2 && j != g) {
+        const key_t k = make_key(d2, j);
+        if (k < A[6]) insert7(A, k);
+      }
+    }
+  }
+#pragma unroll
+  for (int w = 1; w < 32; w <<= 1) {
+    key_t B[7];
+#pragma unroll
+    for (int s = 0; s < 7; ++s) B[s] = __shfl_xor_sync(0xffffffffu, A[s], w);
+    merge7(A, B);
+  }
+}
+
+__global__ void __launch_bounds__(NSEL) k_select(StepArgs a) {
+  const int64_t qi = (int64_t)blockIdx.x * NSEL + threadIdx.x;
+  const bool active = qi < a.nloc;
+  const int c = active ? a.hitcnt[qi] : 0;
+  const int pc = active ? a.pcnt[qi] : 0;
+  const bool over = active && (c > HITS || pc > PSLOTS);
+  key_t A[7];
+#pragma unroll
+  for (int s = 0; s < 7; ++s) A[s] = KEY_EMPTY;
+  key_t eighth = KEY_EMPTY;  // 8th smallest passing key: seeds the next step's t0
+  if (active && !over) {
+    for (int p = 0; p < pc; ++p) {
+      key_t B[7];
+#pragma unroll
+      for (int s = 0; s < 7; ++s) B[s] = a.partial[(qi * PSLOTS + p) * 7 + s];
+      merge7(A, B);
+    }
+    for (int k = 0; k < c; ++k) insert7(A, a.hits[qi * HITS + k]);
+    for (int k = 0; k < c; ++k) {
+      const key_t h = a.hits[qi * HITS + k];
+      if (h > A[6] && h < eighth) eighth = h;
+    }
+  }
+  // overflowed buffers: the warp searches those agents again, one at a time
+  unsigned om = __ballot_sync(0xffffffffu, over);
+  if (a.stats && (threadIdx.x & 31) == 0 && om) atomicAdd(a.stats + 2, (unsigned long long)__popc(om));
+  while (om) {
+    const int src = __ffs(om) - 1;
+    om &= om - 1;
+    const int64_t qo = __shfl_sync(0xffffffffu, qi, src);
+    key_t B[7];
+    warp_full_search(a, qo, B);
+    if ((int)(threadIdx.x & 31) == src) {
+#pragma unroll
+      for (int s = 0; s < 7; ++s) A[s] = B[s];
+    }
+  }
+  if (!active) return;
+  a.hitcnt[qi] = 0;  // ready for the next step
+  a.pcnt[qi] = 0;
+  a.nbr8[qi] = eighth == KEY_EMPTY ? -1 : key_idx(eighth);
+  int nb[7], cnt = 0;
+#pragma unroll
+  for (int s = 0; s < 7; ++s) {
+    nb[s] = A[s] == KEY_EMPTY ? -1 : key_idx(A[s]);
+    cnt += A[s] == KEY_EMPTY ? 0 : 1;
+  }
+#pragma unroll
+  for (int s = 0; s < 7; ++s) a.nbr[qi * 7 + s] = nb[s];
+  a.cnt[qi] = cnt;
+  const float4 p4 = __ldg(pos_of(a.full, a.m, a.sdiv, a.lo + qi));
+  const float4 f4 = __ldg(fwd_of(a.full, a.m, a.sdiv, a.lo + qi));
+  const V3 F = steer_agent(a, v3(p4), v3(f4), nb, cnt);
+  modify_agent(a, qi, v3(p4), f4, F);
+}
+
+}  // namespace
+
+cudaError_t launch_warm_scan(const StepArgs& a, cudaStream_t s) {
+  if (a.nloc <= 0) return cudaSuccess;
+  static int grid = 0;
+  if (!grid) {
+    int dev = 0, sms = 148, r = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    cudaFuncSetAttribute(k_scan, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&r, k_scan, NTS, 0);
+    grid = sms * (r > 0 ? r : 1);
+  }
+  const int64_t units = (int64_t)a.world * a.m / CT;
+  const int64_t nqb = (a.nloc + QBS - 1) / QBS;
+  const int64_t items = nqb * units;
+  const int g = (int)std::min<int64_t>(grid, items);
+  k_scan<<<g, NTS, 0, s>>>(a, units, items);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_warm_select(const StepArgs& a, cudaStream_t s) {
+  if (a.nloc <= 0) return cudaSuccess;
+  k_select<<<(unsigned)((a.nloc + NSEL - 1) / NSEL), NSEL, 0, s>>>(a);
+  return cudaGetLastError();
+}
+
+}  // namespace boids

@@ -120,7 +120,8 @@ def test_wrap_agents_outside(pk, orc):
 
 
 # -------------------------------------------------- trajectories (warm path)
-@pytest.mark.parametrize("kernel,n,steps", [(0, 1024, 30), (0, 4096, 10), (1, 1024, 10)])
+@pytest.mark.parametrize("kernel,n,steps", [(0, 1024, 30), (0, 4096, 10), (1, 1024, 10), (2, 1024, 12),
+                                            (0, 20000, 3)])
 def test_trajectory_from_init(pk, orc, kernel, n, steps):
     """GPU steps continuously (warm thresholds active after step 1); the oracle
     runs the same steps from its own init.  Bit-exact sides stay identical."""
@@ -134,6 +135,26 @@ def test_trajectory_from_init(pk, orc, kernel, n, steps):
             g = f.state()
             assert_state_close(g, o, f"step {t}")
             assert bitexact(g, o), f"step {t} not bit-exact"
+
+
+def test_trajectory_wraps_and_overflow(pk, orc):
+    """Small world, long dt: many agents wrap to the diametric opposite point each
+    step, so their old neighbours end far away -> t0 >= r2 -> the warm
+    scan's hit buffers overflow and k_select's warp re-search runs.  Bit-exact."""
+    p = pk.boids_default_params(init_mode=1, world_radius=12.0, max_speed=30.0)
+    op = _oparams(orc, p)
+    n, dt = 3000, 0.05
+    with pk.Flock(n, p, seed=5) as f:
+        o = orc.init(n, op, seed=5)
+        wrapped = 0
+        for t in range(8):
+            prev = o
+            o, o_idx, _, _ = orc.step(o, dt, op)
+            wrapped += int((np.linalg.norm(o["pos"] - prev["pos"], axis=1) > 10.0).sum())
+            f.step(dt, 1)
+            np.testing.assert_array_equal(f.neighbors()[0], o_idx, err_msg=f"step {t}")
+            assert bitexact(f.state(), o), f"step {t}"
+        assert wrapped > 20
 
 
 # ------------------------------------------- full sizes (bench launch config)
@@ -210,7 +231,7 @@ def test_launch_count_and_info(pk):
         f.step(DT, 5)
         f.sync()
         info = f.info()
-        # per step one fused kernel; the spatial query order (3 binning kernels:
-        # count, scan, scatter) is refreshed on the first step and every 8th
-        assert info.launches - i0 == 5 + 3
+        # step 1 (cold): the fused cluster kernel; steps 2-5 (warm): scan + select;
+        # the spatial query order (3 binning kernels) is refreshed on step 1 and every 8th
+        assert info.launches - i0 == 1 + 4 * 2 + 3
         assert info.cluster == 16 and info.slice == 16384
