@@ -173,6 +173,7 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--cpu-seconds", type=float, default=10.0, help="oracle sample size (seconds of CPU work)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true", help="skip the e2e leg (profiling runs)")
     ap.add_argument("--kernel", type=int, default=0, help="0 fused (default), 1 two-kernel simple path")
     args = ap.parse_args()
     cfg = W.CONFIGS[args.workload]
@@ -264,7 +265,7 @@ def main():
             traffic = json.load(open(summ)).get(cfg.name, {}).get("dram_bytes_per_launch")
         except Exception:
             traffic = None
-    roofline = {"bound": "alu", "kernel": "k_fused (search+merge+steer+modify)",
+    roofline = {"bound": "alu", "kernel": "k_scan (warm-step all-pairs search; k_fused on cold steps)",
                 "achieved": achieved, "peak": peak, "unit": "TFLOP/s", "frac": achieved / peak,
                 "traffic": traffic,
                 "peak_note": f"FP32 SIMT lane-ops: 148 SM x 128 lanes x {sm_max:.0f} MHz "
@@ -276,25 +277,31 @@ def main():
 
     # ---------------- e2e through the C ABI with host buffers ----------------
     e2e = None
-    st = abi.boids_get_state(h)
+    if args.no_e2e:
+        args_e2e = False
+    else:
+        args_e2e = True
+    st = abi.boids_get_state(h) if args_e2e else {}
     host = {k: np.ascontiguousarray(v) for k, v in st.items()}
     h2d = nloc * 4 * 16  # set_state uploads pos4, fwd4 (+speed), up4, side4
     d2h = nloc * 4 * 16  # get_state downloads pos4, fwd4, up4, side4
-    barrier()
-    t0 = time.perf_counter()
-    for _ in range(args.steps):
-        abi.boids_set_state(h, host)
-        step()
-        abi.boids_get_state(h, host)
-    t1 = time.perf_counter()
-    e2e_s = t1 - t0
-    if dist is not None:
-        t = torch.tensor([e2e_s], device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        e2e_s = float(t.item())
-    e2e = {"value": cfg.n * args.steps / e2e_s, "unit": UNIT, "h2d_bytes_per_step": h2d * world,
-           "d2h_bytes_per_step": d2h * world,
-           "note": "boids_set_state (host AoS -> device) + step + boids_get_state (device -> host AoS), wall clock"}
+    if args_e2e:
+        barrier()
+        t0 = time.perf_counter()
+        for _ in range(args.steps):
+            abi.boids_set_state(h, host)
+            step()
+            abi.boids_get_state(h, host)
+        t1 = time.perf_counter()
+        e2e_s = t1 - t0
+        if dist is not None:
+            t = torch.tensor([e2e_s], device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            e2e_s = float(t.item())
+        e2e = {"value": cfg.n * args.steps / e2e_s, "unit": UNIT, "h2d_bytes_per_step": h2d * world,
+               "d2h_bytes_per_step": d2h * world,
+               "note": "boids_set_state (host AoS -> device) + step + boids_get_state (device -> host AoS), "
+                       "wall clock"}
 
     # ---------------- CPU oracle baseline (rank 0, N=1) ----------------
     cpu = None

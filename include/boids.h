@@ -148,7 +148,8 @@ BOIDS_API int boids_get_state(boids_ctx* ctx, float* pos3, float* fwd3, float* u
                     float* speed);
 
 /* Overwrite the owned agents' state from host AoS arrays (count = hi - lo).
- * side is recomputed by the next step; warm-start neighbour data is invalidated.
+ * side is recomputed by the next step.  The last step's neighbour lists are kept
+ * as the seed of the next step's search bound (valid for any new positions).
  * pos3, fwd3, up3, speed must be non-NULL; side3 may be NULL (then zero).  Synchronises. */
 BOIDS_API int boids_set_state(boids_ctx* ctx, const float* pos3, const float* fwd3, const float* up3,
                     const float* side3, const float* speed);

@@ -512,11 +512,12 @@ BOIDS_API int boids_set_state(boids_ctx* c, const float* pos3, const float* fwd3
   CK(cudaMemcpyAsync(L + m, hf.data(), k * sizeof(float4), cudaMemcpyHostToDevice, c->stream));
   CK(cudaMemcpyAsync(c->up4, hu.data(), k * sizeof(float4), cudaMemcpyHostToDevice, c->stream));
   CK(cudaMemcpyAsync(c->side4, hs.data(), k * sizeof(float4), cudaMemcpyHostToDevice, c->stream));
-  CK(cudaMemsetAsync(c->cnt, 0, m * sizeof(int32_t), c->stream));
-  CK(cudaMemsetAsync(c->nbr, 0xFF, m * 7 * sizeof(int32_t), c->stream));
-  CK(cudaMemsetAsync(c->nbr8, 0xFF, m * sizeof(int32_t), c->stream));
+  // The previous neighbour lists are KEPT: the warm bound they seed (the 7th
+  // smallest current distance to 7-8 distinct existing agents) is an upper bound
+  // on the 7th neighbour distance for ANY positions, so the next step stays exact;
+  // a poor bound only costs time.  boids_get_neighbors still reports the lists of
+  // the last step until the next step.
   CK(cudaStreamSynchronize(c->stream));
-  c->warm = false;
   c->steering_valid = false;
   return BOIDS_OK;
 }

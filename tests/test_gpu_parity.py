@@ -137,6 +137,24 @@ def test_trajectory_from_init(pk, orc, kernel, n, steps):
             assert bitexact(g, o), f"step {t} not bit-exact"
 
 
+@pytest.mark.parametrize("new", ["ball", "lattice", "coincident"])
+def test_set_state_keeps_exact_with_stale_lists(pk, orc, new):
+    """boids_set_state keeps the previous neighbour lists as the seed of the warm
+    bound; it must stay exact for an unrelated new state (loose bounds, ties)."""
+    n = 1000
+    gen = {"ball": lambda: W.ball_flock(n, seed=77, radius=14.0),
+           "lattice": lambda: W.lattice_flock(10, 1.0, seed=3),
+           "coincident": lambda: W.coincident_flock(n, groups=6, seed=8)}[new]
+    s = gen()
+    with pk.Flock(n, seed=1, record_steering=True) as f:
+        f.step(DT, 3)  # warm lists of an unrelated flock
+        f.set_state(s)
+        f.step(DT, 1)
+        o_state, o_idx, o_cnt, o_F = orc.step(orc.State(s), DT)
+        np.testing.assert_array_equal(f.neighbors()[0], o_idx)
+        assert bitexact(f.state(), o_state) and np.array_equal(f.steering(), o_F)
+
+
 def test_trajectory_wraps_and_overflow(pk, orc):
     """Small world, long dt: many agents wrap to the diametric opposite point each
     step, so their old neighbours end far away -> t0 >= r2 -> the warm
