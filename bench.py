@@ -226,7 +226,8 @@ def main():
     # ---------------- timed region: K steps, L2 flushed before each ----------------
     abi.boids_set_option(h, abi.BOIDS_OPT_PROFILE, 1)
     abi.boids_get_profile(h, reset=True)
-    launches0 = abi.boids_info(h).launches
+    info0 = abi.boids_info(h)
+    launches0 = info0.launches
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
     barrier()
     torch.cuda.synchronize()
@@ -238,7 +239,8 @@ def main():
             ev[k][1].record(stream)
         torch.cuda.synchronize()
         barrier()
-    launches = abi.boids_info(h).launches - launches0
+    info1 = abi.boids_info(h)
+    launches = info1.launches - launches0
     prof = abi.boids_get_profile(h, reset=True)
     abi.boids_set_option(h, abi.BOIDS_OPT_PROFILE, 0)
     ms = float(sum(a.elapsed_time(b) for a, b in ev))
@@ -249,10 +251,14 @@ def main():
     value = cfg.n * args.steps / (ms / 1e3)
 
     # ---------------- roofline of the dominant kernel ----------------
-    kname = "fused_or_search"
+    grid = cfg.search_mode == 1
+    kname = "grid_search" if grid else "fused_or_search"
     k_ms, k_n = prof[kname]
     k_ms_per = k_ms / max(k_n, 1)
-    pairs_per_launch = float(nloc) * float(cfg.n)
+    if grid:  # algorithmic work of the grid search: pairs over the 27-cell stencils (device counter)
+        pairs_per_launch = float(info1.grid_pairs - info0.grid_pairs) / max(k_n, 1)
+    else:
+        pairs_per_launch = float(nloc) * float(cfg.n)
     achieved = OPS_PER_PAIR * pairs_per_launch / (k_ms_per / 1e3) / 1e12  # T lane-op/s
     pk_ = peaks()
     sm_max = float(pk_.get("sm_max_mhz", 1965.0))
@@ -265,12 +271,15 @@ def main():
             traffic = json.load(open(summ)).get(cfg.name, {}).get("dram_bytes_per_launch")
         except Exception:
             traffic = None
-    roofline = {"bound": "alu", "kernel": "k_scan (warm-step all-pairs search; k_fused on cold steps)",
+    roofline = {"bound": "alu",
+                "kernel": ("k_grid (binned search + steer + modify)" if grid else
+                           "k_scan (warm-step all-pairs search; k_fused on cold steps)"),
                 "achieved": achieved, "peak": peak, "unit": "TFLOP/s", "frac": achieved / peak,
                 "traffic": traffic,
                 "peak_note": f"FP32 SIMT lane-ops: 148 SM x 128 lanes x {sm_max:.0f} MHz "
                              f"(sm_max_mhz of MEASURED_PEAKS.json; each add/sub/mul counted once, no FMA)",
-                "work_per_launch": f"{OPS_PER_PAIR} lane-ops x {pairs_per_launch:.4g} pairs",
+                "work_per_launch": f"{OPS_PER_PAIR} lane-ops x {pairs_per_launch:.4g} pairs"
+                                   + (" (27-cell stencil candidates, device counter)" if grid else " (n_local x n)"),
                 "kernel_ms_per_launch": k_ms_per, "kernel_share_of_step": k_ms / ms if ms else None,
                 "frac_at_measured_clock": (achieved / (148 * LANES_PER_SM * clocks["sm_mhz"] * 1e6 / 1e12))
                 if clocks.get("sm_mhz") else None}

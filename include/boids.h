@@ -90,6 +90,8 @@ typedef struct boids_info_t {
                           lanes) that took the insertion path ... */
   int64_t vote_groups; /* ... out of this many (diagnostics; boids_info synchronises) */
   int64_t fallbacks;   /* warm path, cumulative: agents re-searched after a hit-buffer overflow */
+  int64_t grid_pairs;  /* grid mode, cumulative: (query, candidate) pairs evaluated over the
+                          27-cell stencils -- the grid search's algorithmic work */
 } boids_info_t;
 
 #define BOIDS_KERNEL_FUSED 0   /* default: cold steps run the fused cluster kernel (search + merge +

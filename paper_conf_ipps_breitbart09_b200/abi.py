@@ -55,7 +55,7 @@ class boids_info_t(C.Structure):
         ("n", C.c_int64), ("lo", C.c_int64), ("hi", C.c_int64), ("slice", C.c_int64),
         ("rank", C.c_int32), ("world", C.c_int32), ("kernel", C.c_int32), ("cluster", C.c_int32),
         ("launches", C.c_int64), ("slow_groups", C.c_int64), ("vote_groups", C.c_int64),
-        ("fallbacks", C.c_int64),
+        ("fallbacks", C.c_int64), ("grid_pairs", C.c_int64),
     ]
 
 

@@ -68,6 +68,11 @@ struct boids_ctx {
   unsigned long long* partial = nullptr;  // warm path partial lists [m][PSLOTS][7]
   int32_t* pcnt = nullptr;
   unsigned long long* phase = nullptr;  // diagnostics (BOIDS_OPT_PHASES): per-CTA timestamps
+  // grid mode (BOIDS_GRID): search grid and its binning buffers
+  BinGrid sgrid{};
+  int2* gcellrank = nullptr;
+  int32_t *gcnt = nullptr, *gstart = nullptr, *gqstart = nullptr, *item_start = nullptr, *counter = nullptr;
+  float4* spos = nullptr;
   int vote_u = 4;          // fused kernel: candidates per warp vote
   int resort_every = 8;    // refresh the spatial query order every this many steps
   int64_t since_sort = -1; // steps since the last refresh (-1: never sorted)
@@ -136,6 +141,13 @@ void free_ctx(boids_ctx* c) {
   cudaFree(c->nbr8);
   cudaFree(c->partial);
   cudaFree(c->pcnt);
+  cudaFree(c->gcellrank);
+  cudaFree(c->gcnt);
+  cudaFree(c->gstart);
+  cudaFree(c->gqstart);
+  cudaFree(c->item_start);
+  cudaFree(c->counter);
+  cudaFree(c->spos);
   cudaFree(c->phase);
   for (auto& r : c->recs) {
     cudaEventDestroy(r.a);
@@ -225,11 +237,27 @@ int create_impl(int64_t n, const boids_params* p, uint64_t seed, int32_t rank, i
       (rc = alloc((void**)&c->qperm, m * sizeof(int32_t))) ||
       (rc = alloc((void**)&c->cand, c->ncand * sizeof(float4))) ||
       (rc = alloc((void**)&c->stats, 4 * sizeof(unsigned long long))) ||
-      (rc = alloc((void**)&c->hits, (size_t)m * HITS * sizeof(unsigned long long))) ||
-      (rc = alloc((void**)&c->hitcnt, m * sizeof(int32_t))) ||
-      (rc = alloc((void**)&c->nbr8, m * sizeof(int32_t))) ||
-      (rc = alloc((void**)&c->partial, (size_t)m * PSLOTS * 7 * sizeof(unsigned long long))) ||
-      (rc = alloc((void**)&c->pcnt, m * sizeof(int32_t)))) {
+      (rc = alloc((void**)&c->nbr8, m * sizeof(int32_t)))) {
+    free_ctx(c);
+    return rc;
+  }
+  if (p->search_mode == BOIDS_GRID) {
+    c->sgrid = make_search_grid(*p);
+    const int C = c->sgrid.cells;
+    if ((rc = alloc((void**)&c->gcellrank, slots * sizeof(int2))) ||
+        (rc = alloc((void**)&c->gcnt, C * sizeof(int32_t))) ||
+        (rc = alloc((void**)&c->gstart, (C + 1) * sizeof(int32_t))) ||
+        (rc = alloc((void**)&c->gqstart, (C + 1) * sizeof(int32_t))) ||
+        (rc = alloc((void**)&c->item_start, (C + 1) * sizeof(int32_t))) ||
+        (rc = alloc((void**)&c->counter, sizeof(int32_t))) ||
+        (rc = alloc((void**)&c->spos, (size_t)n * sizeof(float4)))) {
+      free_ctx(c);
+      return rc;
+    }
+  } else if ((rc = alloc((void**)&c->hits, (size_t)m * HITS * sizeof(unsigned long long))) ||
+             (rc = alloc((void**)&c->hitcnt, m * sizeof(int32_t))) ||
+             (rc = alloc((void**)&c->partial, (size_t)m * PSLOTS * 7 * sizeof(unsigned long long))) ||
+             (rc = alloc((void**)&c->pcnt, m * sizeof(int32_t)))) {
     free_ctx(c);
     return rc;
   }
@@ -245,9 +273,10 @@ int create_impl(int64_t n, const boids_params* p, uint64_t seed, int32_t rank, i
   if (e == cudaSuccess) e = cudaMemsetAsync(c->bcnt, 0, c->loc_grid.cells * sizeof(int32_t), s);
   if (e == cudaSuccess) e = launch_fill_nan(c->cand, c->ncand, s);  // entries >= n stay NaN
   if (e == cudaSuccess) e = cudaMemsetAsync(c->stats, 0, 4 * sizeof(unsigned long long), s);
-  if (e == cudaSuccess) e = cudaMemsetAsync(c->hitcnt, 0, m * sizeof(int32_t), s);
+  if (e == cudaSuccess && c->hitcnt) e = cudaMemsetAsync(c->hitcnt, 0, m * sizeof(int32_t), s);
   if (e == cudaSuccess) e = cudaMemsetAsync(c->nbr8, 0xFF, m * sizeof(int32_t), s);
-  if (e == cudaSuccess) e = cudaMemsetAsync(c->pcnt, 0, m * sizeof(int32_t), s);
+  if (e == cudaSuccess && c->pcnt) e = cudaMemsetAsync(c->pcnt, 0, m * sizeof(int32_t), s);
+  if (e == cudaSuccess && c->gcnt) e = cudaMemsetAsync(c->gcnt, 0, c->sgrid.cells * sizeof(int32_t), s);
   if (e == cudaSuccess)
     e = launch_fill_phantoms(c->buf[0], m, shard ? 0 : c->nloc, shard ? world : 1, s);
   if (e == cudaSuccess) e = launch_fill_phantoms(c->buf[1], m, c->nloc, 1, s);
@@ -301,9 +330,34 @@ int one_step(boids_ctx* c, float dt) {
   // Only the warm path keeps the 8th-nearest seed consistent with the lists it
   // writes; any other step invalidates it (a stale seed could repeat one of the
   // new 7 neighbours and break the t0 bound).
-  const bool warm_path = c->kernel == BOIDS_KERNEL_FUSED && c->warm;
+  const bool grid = c->p.search_mode == BOIDS_GRID;
+  const bool warm_path = !grid && c->kernel == BOIDS_KERNEL_FUSED && c->warm;
   if (!warm_path) CK(cudaMemsetAsync(c->nbr8, 0xFF, c->m * sizeof(int32_t), c->stream));
-  if (c->kernel == BOIDS_KERNEL_SIMPLE) {
+  if (grid) {
+    // a2: bin all agents (candidates) and the owned ones (queries) by search cell
+    const bool one = !c->shard || c->world == 1;
+    const int64_t slots = c->shard ? (int64_t)c->world * c->m : c->m;
+    const int chunk = grid_chunk();
+    if ((rc = launch(c, 2, [&] {
+           cudaError_t e = launch_bin(a.full, c->m, a.sdiv, 0, slots, c->sgrid, c->gcellrank, c->gcnt, c->gstart,
+                                      c->spos, one ? c->qperm : nullptr, 0, c->stream, nullptr,
+                                      one ? c->item_start : nullptr, chunk, one ? c->counter : nullptr);
+           if (e == cudaSuccess && !one)
+             e = launch_bin(a.full, c->m, a.sdiv, c->lo, c->nloc, c->sgrid, c->gcellrank, c->gcnt, c->gqstart,
+                            nullptr, c->qperm, (int)c->lo, c->stream, nullptr, c->item_start, chunk, c->counter);
+           return e;
+         }, one ? 3 : 6)))
+      return rc;
+    GridArgs g;
+    g.spos = c->spos;
+    g.cstart = c->gstart;
+    g.qstart = one ? c->gstart : c->gqstart;
+    g.qperm = c->qperm;
+    g.item_start = c->item_start;
+    g.counter = c->counter;
+    g.grid = c->sgrid;
+    if ((rc = launch(c, 3, [&] { return launch_grid(a, g, c->stream); }))) return rc;
+  } else if (c->kernel == BOIDS_KERNEL_SIMPLE) {
     if ((rc = launch(c, 0, [&] { return launch_search_simple(a, c->stream); }))) return rc;
     if ((rc = launch(c, 1, [&] { return launch_update(a, c->stream); }))) return rc;
   } else {
@@ -568,6 +622,7 @@ BOIDS_API int boids_info(boids_ctx* c, boids_info_t* o) {
   o->slow_groups = (int64_t)st[0];
   o->vote_groups = (int64_t)st[1];
   o->fallbacks = (int64_t)st[2];
+  o->grid_pairs = (int64_t)st[3];
   return BOIDS_OK;
 }
 

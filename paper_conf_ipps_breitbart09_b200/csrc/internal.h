@@ -95,6 +95,17 @@ struct StepArgs {
   boids_params p;
 };
 
+// Grid-mode inputs of k_grid (k_grid.cu), produced by the binning passes.
+struct GridArgs {
+  const float4* spos;     // all agents sorted by search cell: x, y, z, original index (int bits)
+  const int* cstart;      // [cells + 1] start of each cell in spos
+  const int* qstart;      // [cells + 1] start of each cell in qperm (owned agents)
+  const int* qperm;       // owned agents (local indices) sorted by cell
+  const int* item_start;  // [cells + 1] first work item (cell, chunk of 512 owned agents) per cell
+  int* counter;           // work-queue counter (reset by the binning scan)
+  BinGrid grid;
+};
+
 // launchers (return the cudaError_t of the launch)
 cudaError_t launch_init(float4* out, float4* up4, float4* side4, int64_t m, int64_t lo,
                         int64_t nloc, const boids_params& p, uint64_t seed, cudaStream_t s);
@@ -102,13 +113,17 @@ cudaError_t launch_fill_phantoms(float4* seg_base, int64_t m, int64_t nloc, int6
                                  cudaStream_t s);
 cudaError_t launch_bin(const float4* full, int64_t m, const SliceDiv& sd, int64_t j0, int64_t count, const BinGrid& g,
                        int2* cellrank, int* cnt, int* start, float4* spos, int* perm, int perm_base,
-                       cudaStream_t s, int* launches);
+                       cudaStream_t s, int* launches, int* item_start = nullptr, int chunk = 1,
+                       int* counter = nullptr);
 BinGrid make_locality_grid(int64_t n, const boids_params& p);
+BinGrid make_search_grid(const boids_params& p);
 cudaError_t launch_fill_nan(float4* p, int64_t count, cudaStream_t s);
 cudaError_t launch_search_simple(const StepArgs& a, cudaStream_t s);
 cudaError_t launch_update(const StepArgs& a, cudaStream_t s);
 cudaError_t launch_fused(const StepArgs& a, int cluster, cudaStream_t s);
 cudaError_t launch_warm_scan(const StepArgs& a, cudaStream_t s);
+cudaError_t launch_grid(const StepArgs& a, const GridArgs& g, cudaStream_t s);
+int grid_chunk();
 cudaError_t launch_warm_select(const StepArgs& a, cudaStream_t s);
 int fused_auto_cluster(int64_t n_pad_total, int64_t nloc, int sm_count);
 

@@ -56,20 +56,12 @@ __global__ void k_bin_count(const float4* __restrict__ full, int64_t m, SliceDiv
   cellrank[k] = make_int2(c, r);
 }
 
-// Exclusive scan of cnt[0..C) into start[0..C], start[C] = total; zeroes cnt.
-// One CTA: counts are staged through shared memory with coalesced global
-// accesses (padded by one word per 32 so each thread's contiguous run is
-// bank-conflict free), scanned per thread, then across the block.
 constexpr int SCAN_T = 1024;
-__global__ void __launch_bounds__(SCAN_T) k_bin_scan(int* __restrict__ cnt, int* __restrict__ start, int C) {
-  extern __shared__ int sh[];  // C + C / 32 words
-  __shared__ int warp_sums[SCAN_T / 32];
+
+// Block-wide exclusive scan of the padded shared array v[0..C) (index i at
+// i + i/32: each thread's contiguous run is bank-conflict free); returns total.
+__device__ __forceinline__ int block_scan_runs(int* sh, int C, int* warp_sums) {
   const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
-  for (int i = tid; i < C; i += SCAN_T) {
-    sh[i + (i >> 5)] = cnt[i];
-    cnt[i] = 0;
-  }
-  __syncthreads();
   const int per = (C + SCAN_T - 1) / SCAN_T;  // contiguous run per thread
   const int b = tid * per;
   int local = 0;
@@ -102,9 +94,49 @@ __global__ void __launch_bounds__(SCAN_T) k_bin_scan(int* __restrict__ cnt, int*
       excl += c;
     }
   }
-  if (tid == SCAN_T - 1) start[C] = excl;
+  const int total = warp_sums[SCAN_T / 32 - 1];
   __syncthreads();
+  return total;
+}
+
+// Exclusive scan of cnt[0..C) into start[0..C], start[C] = total; zeroes cnt.
+// One CTA; counts are staged through shared memory with coalesced accesses.
+// With item_start: also the work items of the grid search -- ceil(count / chunk)
+// per cell -- scanned into item_start[0..C] (item_start[C] = number of items),
+// and the grid kernel's work counter is reset.
+__global__ void __launch_bounds__(SCAN_T) k_bin_scan(int* __restrict__ cnt, int* __restrict__ start, int C,
+                                                    int* __restrict__ item_start, int chunk,
+                                                    int* __restrict__ counter) {
+  extern __shared__ int sh[];  // C + C / 32 words
+  __shared__ int warp_sums[SCAN_T / 32];
+  const int tid = threadIdx.x;
+  for (int i = tid; i < C; i += SCAN_T) {
+    sh[i + (i >> 5)] = cnt[i];
+    cnt[i] = 0;
+  }
+  __syncthreads();
+  const int total = block_scan_runs(sh, C, warp_sums);
   for (int i = tid; i < C; i += SCAN_T) start[i] = sh[i + (i >> 5)];
+  if (tid == 0) start[C] = total;
+  if (!item_start) return;
+  __syncthreads();
+  for (int i = tid; i < C; i += SCAN_T) {  // chunks per cell from the starts
+    const int s0 = sh[i + (i >> 5)];
+    const int s1 = i + 1 < C ? sh[(i + 1) + ((i + 1) >> 5)] : total;
+    cnt[i] = (s1 - s0 + chunk - 1) / chunk;  // cnt is scratch here (re-zeroed below)
+  }
+  __syncthreads();
+  for (int i = tid; i < C; i += SCAN_T) sh[i + (i >> 5)] = cnt[i];
+  __syncthreads();
+  const int items = block_scan_runs(sh, C, warp_sums);
+  for (int i = tid; i < C; i += SCAN_T) {
+    item_start[i] = sh[i + (i >> 5)];
+    cnt[i] = 0;
+  }
+  if (tid == 0) {
+    item_start[C] = items;
+    *counter = 0;
+  }
 }
 
 __global__ void k_bin_scatter(const float4* __restrict__ full, int64_t m, SliceDiv sd, int64_t j0, int64_t count,
@@ -125,9 +157,14 @@ __global__ void k_bin_scatter(const float4* __restrict__ full, int64_t m, SliceD
 
 cudaError_t launch_bin(const float4* full, int64_t m, const SliceDiv& sd, int64_t j0, int64_t count, const BinGrid& g,
                        int2* cellrank, int* cnt, int* start, float4* spos, int* perm, int perm_base,
-                       cudaStream_t s, int* launches) {
-  if (count <= 0) return cudaSuccess;
+                       cudaStream_t s, int* launches, int* item_start, int chunk, int* counter) {
   const unsigned blocks = (unsigned)((count + 255) / 256);
+  if (count <= 0) {  // still publish an empty binning (starts, items, counter)
+    const size_t shm0 = (size_t)(g.cells + g.cells / 32 + 1) * sizeof(int);
+    if (shm0 > 48 * 1024) cudaFuncSetAttribute(k_bin_scan, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)shm0);
+    k_bin_scan<<<1, SCAN_T, shm0, s>>>(cnt, start, g.cells, item_start, chunk, counter);
+    return cudaGetLastError();
+  }
   k_bin_count<<<blocks, 256, 0, s>>>(full, m, sd, j0, count, g, cellrank, cnt);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return e;
@@ -136,11 +173,37 @@ cudaError_t launch_bin(const float4* full, int64_t m, const SliceDiv& sd, int64_
     e = cudaFuncSetAttribute(k_bin_scan, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)shm);
     if (e != cudaSuccess) return e;
   }
-  k_bin_scan<<<1, SCAN_T, shm, s>>>(cnt, start, g.cells);
+  k_bin_scan<<<1, SCAN_T, shm, s>>>(cnt, start, g.cells, item_start, chunk, counter);
   if ((e = cudaGetLastError()) != cudaSuccess) return e;
   k_bin_scatter<<<blocks, 256, 0, s>>>(full, m, sd, j0, count, cellrank, start, spos, perm, perm_base);
   if (launches) *launches += 3;
   return cudaGetLastError();
+}
+
+// Search grid of BOIDS_GRID: cells of size h = r (1 + 2^-10) (a margin far above
+// the fp32 rounding of the cell coordinate and of d2 < r2), row-major over the
+// world box [-B, B]^3, B = max(world, init radius) * 1.02; agents outside are
+// clamped into boundary cells, which keeps every pair closer than r in the same
+// or adjacent cells (clamping is monotone and 1-Lipschitz on cell coordinates).
+// The 27-cell stencil of a cell is then 9 contiguous x-runs of the sorted array.
+BinGrid make_search_grid(const boids_params& p) {
+  BinGrid g{};
+  const float B = fmaxf(p.world_radius, p.init_radius) * 1.02f;
+  g.h = p.search_radius * (1.0f + 1.0f / 1024.0f);
+  int dim = (int)ceilf(2.f * B / g.h);
+  if (dim < 1) dim = 1;
+  if (dim > 1024) {  // huge world vs radius: cap the table (cells grow, still >= r)
+    dim = 1024;
+    g.h = 2.f * B / dim;
+  }
+  for (int d = 0; d < 3; ++d) {
+    g.lo[d] = -B;
+    g.dim[d] = dim;
+  }
+  g.inv_h = 1.f / g.h;
+  g.cells = dim * dim * dim;
+  g.morton = 0;
+  return g;
 }
 
 // Morton locality grid for the brute-force step: 2^L cells per dimension over

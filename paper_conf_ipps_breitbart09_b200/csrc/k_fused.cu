@@ -37,6 +37,7 @@
 #include <cooperative_groups.h>
 
 #include "agent_update.cuh"
+#include "tma.cuh"
 
 namespace cg = cooperative_groups;
 
@@ -47,37 +48,6 @@ constexpr int Q = 4;        // queries per thread (4 independent distance chains
 constexpr int CT = 256;     // candidates per tile (4 KB)
 constexpr int STAGES = 2;   // TMA ring depth (a tile takes ~10-25 us to consume; TMA latency ~1 us)
 
-__device__ __forceinline__ uint32_t smem_u32(const void* p) {
-  return (uint32_t)__cvta_generic_to_shared(p);
-}
-__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
-}
-__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
-               : "memory");
-}
-__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
-  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
-}
-__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
-  asm volatile(
-      "{\n"
-      ".reg .pred P1;\n"
-      "LAB_WAIT:\n"
-      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n"
-      "@!P1 bra LAB_WAIT;\n"
-      "}\n" ::"r"(smem_u32(bar)),
-      "r"(parity)
-      : "memory");
-}
-__device__ __forceinline__ void tma_load_1d(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
-  asm volatile(
-      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
-          smem_u32(dst)),
-      "l"(src), "r"(bytes), "r"(smem_u32(bar))
-      : "memory");
-}
 __device__ __forceinline__ void stamp(const StepArgs& a, int k) {
   if (a.phase && threadIdx.x == 0) {
     unsigned long long t;
@@ -179,7 +149,7 @@ __global__ void __launch_bounds__(NT) k_fused(StepArgs a, int64_t tiles_total) {
       mbar_init(&sm.full[s], 1);
       mbar_init(&sm.empty[s], NW);
     }
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    mbar_fence_init();
   }
   __syncthreads();
   if (tid == 0) {  // prologue: fill the ring

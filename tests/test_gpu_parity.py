@@ -253,3 +253,70 @@ def test_launch_count_and_info(pk):
         # the spatial query order (3 binning kernels) is refreshed on step 1 and every 8th
         assert info.launches - i0 == 1 + 4 * 2 + 3
         assert info.cluster == 16 and info.slice == 16384
+
+
+# ------------------------------------------------------- grid mode (BOIDS_GRID)
+def _grid(pk, **kw):
+    return pk.boids_default_params(search_mode=1, **kw)
+
+
+@pytest.mark.parametrize("n", [1, 2, 7, 257, 1000, 3000])
+def test_grid_step_ball(pk, orc, n):
+    s = W.ball_flock(n, seed=n + 11, radius=max(3.0, 20.0 * (n / 16384) ** (1 / 3) * 2))
+    check_step(pk, orc, s, params=_grid(pk))
+
+
+@pytest.mark.parametrize("case", ["lattice9", "lattice_r", "coincident", "shell", "outside"])
+def test_grid_edge_cases(pk, orc, case):
+    s = {"lattice9": lambda: W.lattice_flock(10, 3.0, seed=1),   # spacing 3 -> d2 = 81 = r2 ties at cell edges
+         "lattice_r": lambda: W.lattice_flock(8, 9.0, seed=2),   # neighbours exactly at r (excluded)
+         "coincident": lambda: W.coincident_flock(700, groups=4, seed=3),
+         "shell": lambda: W.radius_shell_flock(9.0),
+         "outside": lambda: W.ball_flock(1500, seed=9, radius=70.0)}[case]()  # clamped into boundary cells
+    check_step(pk, orc, s, params=_grid(pk), dt=0.05)
+
+
+@pytest.mark.parametrize("n,steps,world", [(4096, 10, 50.0), (3000, 8, 12.0)])
+def test_grid_trajectory(pk, orc, n, steps, world):
+    p = _grid(pk, init_mode=1, world_radius=world)
+    op = _oparams(orc, p)
+    with pk.Flock(n, p, seed=4) as f:
+        o = orc.init(n, op, seed=4)
+        for t in range(steps):
+            o, o_idx, _, _ = orc.step(o, 0.05, op)
+            f.step(0.05, 1)
+            np.testing.assert_array_equal(f.neighbors()[0], o_idx, err_msg=f"step {t}")
+            assert bitexact(f.state(), o), f"step {t}"
+
+
+def test_grid_equals_brute_gpu(pk):
+    """Variant equivalence at scale: grid and brute force give bit-identical lists and states."""
+    n = 120000
+    pg = pk.boids_default_params(init_mode=1, search_mode=1)
+    pb = pk.boids_default_params(init_mode=1, search_mode=0)
+    with pk.Flock(n, pg, seed=2) as fg, pk.Flock(n, pb, seed=2) as fb:
+        for t in range(3):
+            fg.step(DT, 1)
+            fb.step(DT, 1)
+            assert np.array_equal(fg.neighbors()[0], fb.neighbors()[0]), f"step {t}"
+            sg, sb = fg.state(), fb.state()
+            assert all(np.array_equal(sg[k], sb[k]) for k in KEYS), f"step {t}"
+
+
+def test_config_c5_sampled(pk, orc):
+    """C5 (n = 1M, grid) at full size: one step from init, 256 sampled agents
+    checked one by one against the oracle (each an O(n) brute-force search)."""
+    c = W.CONFIGS["c5"]
+    p = pk.boids_default_params(init_mode=c.init_mode, search_mode=c.search_mode)
+    op = _oparams(orc, p)
+    ag = W.sample_agents(c.n, 256)
+    with pk.Flock(c.n, p, seed=1, record_steering=True) as f:
+        s0 = orc.init(c.n, op, seed=1)
+        f.step(DT, 1)
+        g = f.state()
+        g_idx, _ = f.neighbors()
+        o, o_idx, _, o_F = orc.step_sample(s0, ag, DT, op)
+        np.testing.assert_array_equal(g_idx[ag], o_idx)
+        np.testing.assert_allclose(f.steering()[ag], o_F, rtol=RTOL, atol=ATOL)
+        for k in KEYS:
+            np.testing.assert_array_equal(g[k][ag], o[k])
