@@ -175,6 +175,8 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true", help="skip the e2e leg (profiling runs)")
     ap.add_argument("--kernel", type=int, default=0, help="0 fused (default), 1 two-kernel simple path")
+    ap.add_argument("--force-shard", action="store_true",
+                    help="use the multi-GPU code path (NCCL process group + sharded handles) even at N=1")
     args = ap.parse_args()
     cfg = W.CONFIGS[args.workload]
     if args.warmup < 3:
@@ -190,10 +192,12 @@ def main():
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     dist = None
-    if world > 1:
+    if world > 1 or args.force_shard:
         import torch.distributed as dist
 
-        dist.init_process_group("nccl", device_id=dev)
+        if "MASTER_ADDR" not in os.environ:
+            os.environ["MASTER_ADDR"], os.environ["MASTER_PORT"] = "127.0.0.1", "29533"
+        dist.init_process_group("nccl", rank=rank, world_size=world, device_id=dev)
 
     import paper_conf_ipps_breitbart09_b200 as pk
     from paper_conf_ipps_breitbart09_b200 import abi
@@ -201,7 +205,7 @@ def main():
 
     params = pk.boids_default_params(init_mode=cfg.init_mode, search_mode=cfg.search_mode)
     dt = float(W.DT)
-    if world > 1:
+    if dist is not None:
         fl = ShardedFlock(cfg.n, params, seed=1, kernel=args.kernel)
         h = fl.h
         step = lambda: fl.step(dt, 1)  # noqa: E731

@@ -1,0 +1,105 @@
+"""Multi-GPU path on one GPU (the pool gives one GPU per call).
+
+* Shard emulation: G shard handles (boids_create_shard, ranks
+  0..G-1) in one process; the per-step NCCL all-gather is emulated by device
+  copies of every rank's send slice into every rank's full buffer (the exact
+  layout all_gather_into_tensor produces).  The gathered state after k steps
+  must be bit-identical to one single-rank handle: same per-agent arithmetic,
+  same (d2, index) order, whatever the partition.
+* ShardedFlock over a real NCCL process group of size 1 (torch.distributed,
+  all_gather_into_tensor on zero-copy views of the library's buffers).
+"""
+import os
+import socket
+
+import numpy as np
+import pytest
+
+import workloads as W
+
+pytestmark = pytest.mark.gpu
+KEYS = ("pos", "fwd", "up", "side", "speed")
+DT = float(W.DT)
+
+
+def _emulated_run(pk, n, world, params, steps, seed=1):
+    import torch
+
+    from paper_conf_ipps_breitbart09_b200 import abi
+    from paper_conf_ipps_breitbart09_b200.shard import device_view
+
+    dev = torch.device("cuda", 0)
+    hs = [abi.boids_create_shard(n, params, seed, r, world) for r in range(world)]
+    try:
+        stream = torch.cuda.current_stream().cuda_stream
+        views = []
+        for h in hs:
+            abi.boids_set_stream(h, stream)
+            send, full, nbytes = abi.boids_shard_buffers(h)
+            views.append((device_view(send, nbytes, dev), device_view(full, nbytes * world, dev), nbytes // 4))
+        for _ in range(steps):
+            for r, (send, _, nf) in enumerate(views):  # all-gather: rank r's slice -> every full buffer
+                for (_, full, _) in views:
+                    full[r * nf:(r + 1) * nf].copy_(send)
+            for h in hs:
+                abi.boids_step_shard(h, DT)
+        torch.cuda.synchronize()
+        parts = [abi.boids_get_state(h) for h in hs]
+        nbrs = [abi.boids_get_neighbors(h)[0] for h in hs]
+        return {k: np.concatenate([p[k] for p in parts]) for k in KEYS}, np.concatenate(nbrs)
+    finally:
+        for h in hs:
+            abi.boids_destroy(h)
+
+
+@pytest.mark.parametrize("mode,n,world", [(0, 3000, 2), (0, 5000, 3), (0, 1000, 8), (1, 20000, 4), (1, 777, 2)])
+def test_shard_emulation_bitidentical(boidslib, mode, n, world):
+    import paper_conf_ipps_breitbart09_b200 as pk
+
+    p = pk.boids_default_params(init_mode=1, search_mode=mode, world_radius=20.0)
+    steps = 4
+    got, got_nbr = _emulated_run(pk, n, world, p, steps)
+    with pk.Flock(n, p, seed=1) as f:
+        f.step(DT, steps)
+        ref = f.state()
+        ref_nbr = f.neighbors()[0]
+    assert np.array_equal(got_nbr, ref_nbr)
+    for k in KEYS:
+        assert np.array_equal(got[k], ref[k]), k
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def test_sharded_flock_nccl_single_rank(boidslib):
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_ipps_breitbart09_b200 as pk
+    from paper_conf_ipps_breitbart09_b200.shard import ShardedFlock
+
+    os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+    os.environ["MASTER_PORT"] = str(_free_port())
+    torch.cuda.set_device(0)
+    dist.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda", 0))
+    try:
+        p = pk.boids_default_params(init_mode=1)
+        n = 4000
+        sf = ShardedFlock(n, p, seed=3)
+        sf.step(DT, 5)
+        got = sf.state()
+        got_nbr = sf.neighbors()[0]
+        sf.close()
+        with pk.Flock(n, p, seed=3) as f:
+            f.step(DT, 5)
+            ref = f.state()
+            assert np.array_equal(got_nbr, f.neighbors()[0])
+        for k in KEYS:
+            assert np.array_equal(got[k], ref[k]), k
+    finally:
+        dist.destroy_process_group()
