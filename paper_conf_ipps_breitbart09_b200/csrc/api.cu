@@ -66,6 +66,7 @@ struct boids_ctx {
   int32_t* hitcnt = nullptr;            // warm path hit counts [m]
   int32_t* nbr8 = nullptr;              // 8th nearest of the last step or -1 [m]
   unsigned long long* partial = nullptr;  // warm path partial lists [m][PSLOTS][7]
+  float* qlim = nullptr;                  // warm path search limits [m]
   int32_t* pcnt = nullptr;
   unsigned long long* phase = nullptr;  // diagnostics (BOIDS_OPT_PHASES): per-CTA timestamps
   // grid mode (BOIDS_GRID): search grid and its binning buffers
@@ -141,6 +142,7 @@ void free_ctx(boids_ctx* c) {
   cudaFree(c->nbr8);
   cudaFree(c->partial);
   cudaFree(c->pcnt);
+  cudaFree(c->qlim);
   cudaFree(c->gcellrank);
   cudaFree(c->gcnt);
   cudaFree(c->gstart);
@@ -257,7 +259,8 @@ int create_impl(int64_t n, const boids_params* p, uint64_t seed, int32_t rank, i
   } else if ((rc = alloc((void**)&c->hits, (size_t)m * HITS * sizeof(unsigned long long))) ||
              (rc = alloc((void**)&c->hitcnt, m * sizeof(int32_t))) ||
              (rc = alloc((void**)&c->partial, (size_t)m * PSLOTS * 7 * sizeof(unsigned long long))) ||
-             (rc = alloc((void**)&c->pcnt, m * sizeof(int32_t)))) {
+             (rc = alloc((void**)&c->pcnt, m * sizeof(int32_t))) ||
+             (rc = alloc((void**)&c->qlim, m * sizeof(float)))) {
     free_ctx(c);
     return rc;
   }
@@ -321,6 +324,7 @@ StepArgs make_args(boids_ctx* c, float dt) {
   a.nbr8 = c->nbr8;
   a.partial = c->partial;
   a.pcnt = c->pcnt;
+  a.qlim = c->qlim;
   return a;
 }
 
@@ -375,7 +379,7 @@ int one_step(boids_ctx* c, float dt) {
     c->since_sort++;
     if (warm_path) {
       // warm step: all-pairs scan appending passing keys, then select + update
-      if ((rc = launch(c, 0, [&] { return launch_warm_scan(a, c->stream); }))) return rc;
+      if ((rc = launch(c, 0, [&] { return launch_warm_scan(a, c->stream); }, 2))) return rc;
       if ((rc = launch(c, 1, [&] { return launch_warm_select(a, c->stream); }))) return rc;
     } else {
       // cold step (no previous lists) or forced: the cluster kernel

@@ -90,6 +90,7 @@ struct StepArgs {
   int32_t* nbr8;              // [nloc] 8th nearest agent of the last step, or -1 (warm-bound seed)
   unsigned long long* partial;  // warm path: [nloc][PSLOTS][7] partial top-7 lists (unbounded agents)
   int32_t* pcnt;              // warm path: [nloc] partial lists written
+  float* qlim;                // warm path: [nloc] inclusive search limit min(prev(r2), t0) (k_bound)
   unsigned long long* phase;  // diagnostics: per-CTA %globaltimer stamps [grid][8], nullptr = off
   float dt;
   boids_params p;

@@ -35,11 +35,13 @@ namespace boids {
 namespace {
 
 constexpr int Q = 4;        // queries per thread
-constexpr int CT = 256;     // candidates per tile (one TMA bulk copy of 4 KB)
-constexpr int STAGES = 3;   // TMA ring depth
+constexpr int CT = 128;     // candidates per tile (one TMA bulk copy of 2 KB; fine stream-K granularity)
+constexpr int STAGES = 4;   // TMA ring depth
 constexpr int U = 4;        // candidates per warp vote
-constexpr int NTS = 128;    // k_scan threads per CTA
-constexpr int QBS = NTS * Q;  // queries per block (512)
+// k_scan CTA shapes: 512 threads (one CTA per SM; its 16 warps share the TMA
+// ring, so a warp that runs ahead waits on the ring instead of leaving the SM
+// to a lone straggler -- measured 1.7-2x per-CTA spread with 3 small CTAs per
+// SM) for large n, 128 threads when there are too few items for 148 CTAs.
 constexpr int WB = Q * U * 32;  // records per warp buffer (8 KB): one vote group's maximum
 constexpr int UBW = 8;         // per warp: running top-7 lists for unbounded queries
 
@@ -49,10 +51,11 @@ struct __align__(8) Rec {
   key_t key;
 };
 
+template <int NT>
 struct __align__(16) ScanSmem {
   float4 ring[STAGES][CT];
-  Rec rec[NTS / 32][WB];
-  key_t ulist[NTS / 32][UBW][7];  // sorted top-7 of unbounded queries (t0 >= r2)
+  Rec rec[NT / 32][WB];
+  key_t ulist[NT / 32][UBW][7];  // sorted top-7 of unbounded queries (t0 >= r2)
   uint64_t full[STAGES];
   uint64_t empty[STAGES];
 };
@@ -92,11 +95,23 @@ __device__ __forceinline__ float warm_t0(const StepArgs& a, int64_t qi, float4 m
 
 // Issue the TMA load of global tile counter tc (stage tc % STAGES), waiting until
 // every warp released the stage's previous tile.  Called by thread 0 only.
-__device__ __forceinline__ void issue_tile(ScanSmem& sm, const StepArgs& a, uint32_t tc, int64_t tile) {
+// Tile k of a run over candidates [c0, c1): [tb, te), CT-aligned inside the run.
+__device__ __forceinline__ void run_tile(int64_t c0, int64_t c1, int k, int64_t& tb, int64_t& te) {
+  const int64_t base = c0 / CT + k;
+  tb = k == 0 ? c0 : base * CT;
+  te = min(c1, (base + 1) * CT);
+}
+
+// Issue the TMA load of candidates [tb, te) as global tile counter tc (stage tc %
+// STAGES), after every warp released the stage's previous tile.  Thread 0 only.
+// The range never straddles a slice (m % CT == 0); any multiple of 16 bytes.
+template <class SM>
+__device__ __forceinline__ void issue_tile(SM& sm, const StepArgs& a, uint32_t tc, int64_t tb, int64_t te) {
   const int s = (int)(tc % STAGES);
   if (tc >= STAGES) mbar_wait(&sm.empty[s], ((tc - STAGES) / STAGES) & 1u);
-  mbar_arrive_expect_tx(&sm.full[s], CT * sizeof(float4));
-  tma_load_1d(sm.ring[s], pos_of(a.full, a.m, a.sdiv, tile * CT), CT * sizeof(float4), &sm.full[s]);
+  const uint32_t bytes = (uint32_t)(te - tb) * (uint32_t)sizeof(float4);
+  mbar_arrive_expect_tx(&sm.full[s], bytes);
+  tma_load_1d(sm.ring[s], pos_of(a.full, a.m, a.sdiv, tb), bytes, &sm.full[s]);
 }
 
 // Insert key k into a sorted 7-list in shared memory; returns the new worst d2.
@@ -111,18 +126,42 @@ __device__ __noinline__ float insert_l7(key_t* L7, key_t k) {
 }
 
 // Flush a warp's record buffer into the global per-query hit buffers.
+// 8 records per lane per round: the atomics' round trips overlap.
 __device__ __forceinline__ void flush(const StepArgs& a, const Rec* rec, int n, int lane) {
-  for (int i = lane; i < n; i += 32) {
-    const Rec r = rec[i];
-    const int slot = atomicAdd(a.hitcnt + r.qi, 1);
-    if (slot < HITS) a.hits[(int64_t)r.qi * HITS + slot] = r.key;
+  for (int i0 = 0; i0 < n; i0 += 32 * 8) {
+    Rec r[8];
+    int slot[8];
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      const int i = i0 + k * 32 + lane;
+      r[k] = i < n ? rec[i] : Rec{-1, 0, 0ull};
+    }
+#pragma unroll
+    for (int k = 0; k < 8; ++k) slot[k] = r[k].qi >= 0 ? atomicAdd(a.hitcnt + r[k].qi, 1) : HITS;
+#pragma unroll
+    for (int k = 0; k < 8; ++k)
+      if (slot[k] < HITS) a.hits[(int64_t)r[k].qi * HITS + slot[k]] = r[k].key;
   }
 }
 
-__global__ void __launch_bounds__(NTS) k_scan(StepArgs a, int64_t units, int64_t items) {
-  __shared__ ScanSmem sm;
+__device__ __forceinline__ void stamp_k(const StepArgs& a, int k) {
+  if (a.phase && threadIdx.x == 0) {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    a.phase[blockIdx.x * 8 + k] = t;
+  }
+}
+
+template <int NTS>
+__global__ void __launch_bounds__(NTS, NTS == 128 ? 4 : 1) k_scan(StepArgs a, int64_t ncand, int64_t items) {
+  constexpr int QBS = NTS * Q;
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  ScanSmem<NTS>& sm = *reinterpret_cast<ScanSmem<NTS>*>(smem_raw);
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-  const int64_t L0 = items * blockIdx.x / gridDim.x, L1 = items * (blockIdx.x + 1) / gridDim.x;
+  stamp_k(a, 0);
+  // equal shares of the (query block, candidate) space, boundaries on multiples of
+  // U (ncand % U == 0), so every tile holds whole vote groups
+  const int64_t L0 = items * blockIdx.x / gridDim.x / U * U, L1 = items * (blockIdx.x + 1) / gridDim.x / U * U;
   if (tid == 0) {
 #pragma unroll
     for (int s = 0; s < STAGES; ++s) {
@@ -132,6 +171,7 @@ __global__ void __launch_bounds__(NTS) k_scan(StepArgs a, int64_t units, int64_t
     mbar_fence_init();
   }
   __syncthreads();
+  stamp_k(a, 4);
   const float r2 = __fmul_rn(a.p.search_radius, a.p.search_radius);
   const float r2_in = __uint_as_float(__float_as_uint(r2) - 1u);  // d2 < r2  <=>  d2 <= r2_in
   Rec* rec = sm.rec[warp];
@@ -139,10 +179,12 @@ __global__ void __launch_bounds__(NTS) k_scan(StepArgs a, int64_t units, int64_t
   unsigned slow_groups = 0, groups = 0;
   uint32_t tc = 0;    // tiles issued / consumed by this CTA (ring phase bookkeeping)
   for (int64_t L = L0; L < L1;) {
-    const int64_t qb = L / units, u0 = L - qb * units;
-    const int nu = (int)min(units - u0, L1 - L);
-    if (tid == 0)
-      for (int t = 0; t < STAGES && t < nu; ++t) issue_tile(sm, a, tc + t, u0 + t);
+    // run = one query block x candidates [c0, c1): the CTA's range is an exact
+    // 1/grid share of (query blocks x candidates), so every CTA has the same work
+    const int64_t qb = L / ncand, c0 = L - qb * ncand;
+    const int64_t c1 = min(ncand, c0 + (L1 - L));
+    const int nu = (int)((c1 - 1) / CT - c0 / CT + 1);  // tiles in this run
+    if (L == L0) stamp_k(a, 5);
     // this run's queries: 4 per thread, in spatial order (qperm)
     float2 pxy[Q];
     float pz[Q], lim[Q];
@@ -156,13 +198,22 @@ __global__ void __launch_bounds__(NTS) k_scan(StepArgs a, int64_t units, int64_t
                                     : make_float4(__int_as_float(0x7fc00000), 0.f, 0.f, 0.f);
       pxy[q] = make_float2(me.x, me.y);
       pz[q] = me.z;
-      lim[q] = fminf(r2_in, warm_t0(a, qi, me));  // inclusive limit
+      lim[q] = qi < a.nloc ? __ldg(a.qlim + qi) : r2_in;  // inclusive limit from k_bound
     }
     // Unbounded queries (no warm bound: t0 >= r2, e.g. the agent wrapped to the far
     // side of the world) would append every in-radius pair; the first UBW of each
     // warp keep a running top-7 here instead (limit tightening as it fills) and
     // flush it as a partial list at the end of the run.
+    if (L == L0) stamp_k(a, 6);
+    if (tid == 0)
+      for (int t = 0; t < STAGES && t < nu; ++t) {
+        int64_t tb, te;
+        run_tile(c0, c1, t, tb, te);
+        issue_tile(sm, a, tc + t, tb, te);
+      }
+    if (L == L0) stamp_k(a, 7);
     int ul[Q];
+    bool warp_ul;
     {
       int used = 0;
 #pragma unroll
@@ -173,21 +224,24 @@ __global__ void __launch_bounds__(NTS) k_scan(StepArgs a, int64_t units, int64_t
         ul[q] = (ub && idx < UBW) ? idx : -1;
         used += __popc(bal);
       }
+      warp_ul = used > 0;
       __syncwarp();
       for (int i = lane; i < UBW * 7; i += 32) (&sm.ulist[warp][0][0])[i] = KEY_EMPTY;
       __syncwarp();
     }
     float limc = fmaxf(fmaxf(lim[0], lim[1]), fmaxf(lim[2], lim[3]));
+    if (L == L0) stamp_k(a, 1);
     for (int t = 0; t < nu; ++t, ++tc) {
       const int s = (int)(tc % STAGES);
       mbar_wait(&sm.full[s], (tc / STAGES) & 1u);
       const float4* tile = sm.ring[s];
-      const int jb = (int)((u0 + t) * CT);
-#pragma unroll 2
-      for (int c = 0; c < CT; c += U) {
+      int64_t tb64, te64;
+      run_tile(c0, c1, t, tb64, te64);
+      const int jb = (int)tb64, cnt = (int)(te64 - tb64);
+      auto group = [&](const int c) {
         float4 cc[U];
 #pragma unroll
-        for (int u = 0; u < U; ++u) cc[u] = tile[c + u];
+        for (int u = 0; u < U; ++u) cc[u] = tile[c + u];  // cnt % U == 0
         // d2 = ((dx*dx) + (dy*dy)) + (dz*dz), each op rounded: packed (dx, dy) and
         // squares, scalar dz and sums (see k_fused.cu)
         float d[Q][U];
@@ -216,12 +270,18 @@ __global__ void __launch_bounds__(NTS) k_scan(StepArgs a, int64_t units, int64_t
           for (int q = 0; q < Q; ++q)
 #pragma unroll
             for (int u = 0; u < U; ++u)
-              if (d[q][u] <= lim[q] && jb + c + u != gq[q]) {
-                if (ul[q] >= 0)  // unbounded query with a list: exact running top-7
-                  lim[q] = fminf(lim[q], insert_l7(sm.ulist[warp][ul[q]], make_key(d[q][u], jb + c + u)));
-                else
-                  bits |= 1u << (q * U + u);
+              if (d[q][u] <= lim[q] && jb + c + u != gq[q]) bits |= 1u << (q * U + u);
+          if (warp_ul) {  // warp-uniform and rare: some query of this warp keeps a list
+#pragma unroll
+            for (int q = 0; q < Q; ++q)
+              if (ul[q] >= 0) {
+#pragma unroll
+                for (int u = 0; u < U; ++u)
+                  if (bits & (1u << (q * U + u)))
+                    lim[q] = fminf(lim[q], insert_l7(sm.ulist[warp][ul[q]], make_key(d[q][u], jb + c + u)));
+                bits &= ~(((1u << U) - 1u) << (q * U));
               }
+          }
           const int nrec = __popc(bits);
           int incl = nrec;
 #pragma unroll
@@ -249,10 +309,20 @@ __global__ void __launch_bounds__(NTS) k_scan(StepArgs a, int64_t units, int64_t
           wcount += total;
           limc = fmaxf(fmaxf(lim[0], lim[1]), fmaxf(lim[2], lim[3]));
         }
+            };
+      if (cnt == CT) {  // full tile: constant trip count (the common case)
+#pragma unroll 2
+        for (int c = 0; c < CT; c += U) group(c);
+      } else {  // ragged tile at a run boundary (cnt % U == 0)
+        for (int c = 0; c < cnt; c += U) group(c);
       }
       __syncwarp();
       if (lane == 0) mbar_arrive(&sm.empty[s]);
-      if (tid == 0 && t + STAGES < nu) issue_tile(sm, a, tc + STAGES, u0 + t + STAGES);
+      if (tid == 0 && t + STAGES < nu) {
+        int64_t tb, te;
+        run_tile(c0, c1, t + STAGES, tb, te);
+        issue_tile(sm, a, tc + STAGES, tb, te);
+      }
     }
     // partial lists of the unbounded queries -> global (merged by k_select)
     __syncwarp();
@@ -268,14 +338,29 @@ __global__ void __launch_bounds__(NTS) k_scan(StepArgs a, int64_t units, int64_t
       }
     }
     __syncwarp();
-    L += nu;
+    L += c1 - c0;
   }
+  stamp_k(a, 2);
   __syncwarp();
   flush(a, rec, wcount, lane);
+  stamp_k(a, 3);
   if (a.stats && lane == 0) {
     atomicAdd(a.stats, (unsigned long long)slow_groups);
     atomicAdd(a.stats + 1, (unsigned long long)groups);
   }
+}
+
+// ---------------------------------------------------------------- bound ----
+// qlim[i] = min(prev(r2), t0_i): each agent's inclusive search limit for the warm
+// scan, computed once per step (k_scan reads it instead of re-gathering the 8
+// previous neighbours in every CTA that shares the agent's query block).
+__global__ void __launch_bounds__(256) k_bound(StepArgs a) {
+  const int64_t qi = (int64_t)blockIdx.x * 256 + threadIdx.x;
+  if (qi >= a.nloc) return;
+  const float r2 = __fmul_rn(a.p.search_radius, a.p.search_radius);
+  const float r2_in = __uint_as_float(__float_as_uint(r2) - 1u);
+  const float4 me = __ldg(pos_of(a.full, a.m, a.sdiv, a.lo + qi));
+  a.qlim[qi] = fminf(r2_in, warm_t0(a, qi, me));
 }
 
 // --------------------------------------------------------------- select ----
@@ -373,23 +458,40 @@ __global__ void __launch_bounds__(NSEL) k_select(StepArgs a) {
 
 }  // namespace
 
-cudaError_t launch_warm_scan(const StepArgs& a, cudaStream_t s) {
-  if (a.nloc <= 0) return cudaSuccess;
+template <int NT>
+int scan_grid(int sms) {
   static int grid = 0;
   if (!grid) {
-    int dev = 0, sms = 148, r = 0;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    cudaFuncSetAttribute(k_scan, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&r, k_scan, NTS, 0);
+    int r = 0;
+    cudaFuncSetAttribute(k_scan<NT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(ScanSmem<NT>));
+    cudaFuncSetAttribute(k_scan<NT>, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&r, k_scan<NT>, NT, sizeof(ScanSmem<NT>));
     grid = sms * (r > 0 ? r : 1);
   }
-  const int64_t units = (int64_t)a.world * a.m / CT;
-  const int64_t nqb = (a.nloc + QBS - 1) / QBS;
-  const int64_t items = nqb * units;
-  const int g = (int)std::min<int64_t>(grid, items);
-  k_scan<<<g, NTS, 0, s>>>(a, units, items);
+  return grid;
+}
+
+template <int NT>
+cudaError_t scan_with(const StepArgs& a, int sms, int64_t ncand, cudaStream_t s) {
+  const int64_t nqb = (a.nloc + NT * Q - 1) / (NT * Q);
+  const int64_t items = nqb * ncand;  // (query block, candidate) pairs
+  const int g = (int)std::min<int64_t>(scan_grid<NT>(sms), (items + CT - 1) / CT);
+  k_scan<NT><<<g, NT, sizeof(ScanSmem<NT>), s>>>(a, ncand, items);
   return cudaGetLastError();
+}
+
+cudaError_t launch_warm_scan(const StepArgs& a, cudaStream_t s) {
+  if (a.nloc <= 0) return cudaSuccess;
+  k_bound<<<(unsigned)((a.nloc + 255) / 256), 256, 0, s>>>(a);
+  if (cudaError_t e = cudaGetLastError()) return e;
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const int64_t ncand = (int64_t)a.world * a.m;
+  // one 512-thread CTA per SM when every SM gets >= 4 tiles of (2048 queries x CT)
+  const int64_t tiles512 = (a.nloc + 2047) / 2048 * (ncand / CT);
+  if (tiles512 >= 4LL * sms) return scan_with<512>(a, sms, ncand, s);
+  return scan_with<128>(a, sms, ncand, s);
 }
 
 cudaError_t launch_warm_select(const StepArgs& a, cudaStream_t s) {

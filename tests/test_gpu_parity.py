@@ -249,9 +249,9 @@ def test_launch_count_and_info(pk):
         f.step(DT, 5)
         f.sync()
         info = f.info()
-        # step 1 (cold): the fused cluster kernel; steps 2-5 (warm): scan + select;
+        # step 1 (cold): the fused cluster kernel; steps 2-5 (warm): bound + scan + select;
         # the spatial query order (3 binning kernels) is refreshed on step 1 and every 8th
-        assert info.launches - i0 == 1 + 4 * 2 + 3
+        assert info.launches - i0 == 1 + 4 * 3 + 3
         assert info.cluster == 16 and info.slice == 16384
 
 

@@ -10,7 +10,10 @@ import paper_conf_ipps_breitbart09_b200 as pk  # noqa: E402
 from paper_conf_ipps_breitbart09_b200 import abi  # noqa: E402
 import workloads as W  # noqa: E402
 
-NAMES = ["start", "t0+sync", "scan end", "lists synced", "merged", "epilogue", "exit"]
+import os
+SCAN = os.environ.get("SCAN") == "1"
+NAMES = (["start", "setup done", "scan end", "flushed", "mbar init", "run start", "queries loaded", "tma issued"] if SCAN else
+         ["start", "t0+sync", "scan end", "lists synced", "merged", "epilogue", "exit"])
 cfg = W.CONFIGS[sys.argv[1]]
 clusters = [int(x) for x in sys.argv[2:]] or [0]
 for cl in clusters:
@@ -18,6 +21,9 @@ for cl in clusters:
     abi.boids_set_option(f.h, abi.BOIDS_OPT_PHASES, 8192)
     f.step(float(W.DT), 4)
     f.sync()
+    if SCAN:
+        abi.boids_set_option(f.h, abi.BOIDS_OPT_PHASES, 0)
+        abi.boids_set_option(f.h, abi.BOIDS_OPT_PHASES, 8192)
     f.profile(reset=True)
     f.step(float(W.DT), 1)
     prof = f.profile()
