@@ -42,16 +42,20 @@ __device__ __forceinline__ int cell_of(float4 p, const BinGrid& g) {
 }
 
 // Agents j in [j0, j0 + count) of the segmented buffer `full`.
+// keep_nan: bin agents with a NaN position into cell 0 (query binning: every
+// owned agent must get a query slot); otherwise NaN slots -- the phantoms that
+// pad every slice -- are skipped (candidate binning).
 __global__ void k_bin_count(const float4* __restrict__ full, int64_t m, SliceDiv sd, int64_t j0, int64_t count,
-                            BinGrid g, int2* __restrict__ cellrank, int* __restrict__ cnt) {
+                            BinGrid g, int2* __restrict__ cellrank, int* __restrict__ cnt, int keep_nan) {
   int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (k >= count) return;
   float4 p = __ldg(pos_of(full, m, sd, j0 + k));
-  if (p.x != p.x) {  // phantom (NaN position): not binned
+  const bool nan = p.x != p.x || p.y != p.y || p.z != p.z;
+  if (nan && !keep_nan) {
     cellrank[k] = make_int2(-1, 0);
     return;
   }
-  int c = cell_of(p, g);
+  int c = nan ? 0 : cell_of(p, g);
   int r = atomicAdd(&cnt[c], 1);
   cellrank[k] = make_int2(c, r);
 }
@@ -165,7 +169,7 @@ cudaError_t launch_bin(const float4* full, int64_t m, const SliceDiv& sd, int64_
     k_bin_scan<<<1, SCAN_T, shm0, s>>>(cnt, start, g.cells, item_start, chunk, counter);
     return cudaGetLastError();
   }
-  k_bin_count<<<blocks, 256, 0, s>>>(full, m, sd, j0, count, g, cellrank, cnt);
+  k_bin_count<<<blocks, 256, 0, s>>>(full, m, sd, j0, count, g, cellrank, cnt, spos == nullptr);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return e;
   const size_t shm = (size_t)(g.cells + g.cells / 32 + 1) * sizeof(int);

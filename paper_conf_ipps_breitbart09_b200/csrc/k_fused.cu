@@ -253,6 +253,7 @@ __global__ void __launch_bounds__(NT) k_fused(StepArgs a, int64_t tiles_total) {
     // refill this stage with tile t + STAGES once every warp has released it
     if (tid == 0 && t + STAGES < nt) {
       mbar_wait(&sm.empty[s], (uint32_t)((t / STAGES) & 1));
+      fence_proxy_async_smem();
       mbar_arrive_expect_tx(&sm.full[s], CT * sizeof(float4));
       tma_load_1d(ring[s], tile_src(a, r + (int64_t)(t + STAGES) * K), CT * sizeof(float4), &sm.full[s]);
     }

@@ -57,7 +57,10 @@ __device__ __forceinline__ void next_tile(const GridSmem& sm, int& r, int& off) 
 
 __device__ __forceinline__ void issue(GridSmem& sm, const GridArgs& g, uint32_t tc, int r, int off) {
   const int s = (int)(tc % STAGES);
-  if (tc >= STAGES) mbar_wait(&sm.empty[s], ((tc - STAGES) / STAGES) & 1u);
+  if (tc >= STAGES) {
+    mbar_wait(&sm.empty[s], ((tc - STAGES) / STAGES) & 1u);
+    fence_proxy_async_smem();
+  }
   const int cnt = tile_count(sm, r, off);
   mbar_arrive_expect_tx(&sm.full[s], cnt * (uint32_t)sizeof(float4));
   tma_load_1d(sm.ring[s], g.spos + sm.range[r].x + off, cnt * (uint32_t)sizeof(float4), &sm.full[s]);

@@ -108,7 +108,10 @@ __device__ __forceinline__ void run_tile(int64_t c0, int64_t c1, int k, int64_t&
 template <class SM>
 __device__ __forceinline__ void issue_tile(SM& sm, const StepArgs& a, uint32_t tc, int64_t tb, int64_t te) {
   const int s = (int)(tc % STAGES);
-  if (tc >= STAGES) mbar_wait(&sm.empty[s], ((tc - STAGES) / STAGES) & 1u);
+  if (tc >= STAGES) {
+    mbar_wait(&sm.empty[s], ((tc - STAGES) / STAGES) & 1u);
+    fence_proxy_async_smem();
+  }
   const uint32_t bytes = (uint32_t)(te - tb) * (uint32_t)sizeof(float4);
   mbar_arrive_expect_tx(&sm.full[s], bytes);
   tma_load_1d(sm.ring[s], pos_of(a.full, a.m, a.sdiv, tb), bytes, &sm.full[s]);
