@@ -73,6 +73,9 @@ typedef struct boids_params {
   int32_t max_neighbors; /* must be 7 */
   int32_t search_mode;   /* BOIDS_BRUTE or BOIDS_GRID */
   int32_t init_mode;     /* BOIDS_INIT_OPENSTEER or BOIDS_INIT_WORLD */
+  int32_t think_every;   /* think frequency k >= 1 (skipThink, sec 5.3): agent i runs the
+                            simulation substage at step t iff (i + t) mod k == 0 and otherwise
+                            reuses its stored steering vector; every agent is modified.  1 */
 } boids_params;
 
 typedef struct boids_ctx boids_ctx; /* opaque handle */
@@ -92,6 +95,7 @@ typedef struct boids_info_t {
   int64_t fallbacks;   /* warm path, cumulative: agents re-searched after a hit-buffer overflow */
   int64_t grid_pairs;  /* grid mode, cumulative: (query, candidate) pairs evaluated over the
                           27-cell stencils -- the grid search's algorithmic work */
+  int64_t step_index;  /* steps taken by this handle (the t of the think schedule) */
 } boids_info_t;
 
 #define BOIDS_KERNEL_FUSED 0   /* default: cold steps run the fused cluster kernel (search + merge +
@@ -157,8 +161,8 @@ BOIDS_API int boids_set_state(boids_ctx* ctx, const float* pos3, const float* fw
                     const float* side3, const float* speed);
 
 /* Neighbour lists of the last step for the owned agents: idx7 = count*7 int32,
- * ascending by (d2, index), -1 padded; cnt = count int32.  Synchronises.
- * Before the first step cnt is 0 everywhere. */
+ * ascending by (d2, index), -1 padded; cnt = count int32, or -1 for an agent that
+ * has not been searched yet (before its first step / first think).  Synchronises. */
 BOIDS_API int boids_get_neighbors(boids_ctx* ctx, int32_t* idx7, int32_t* cnt);
 
 /* Steering vectors F (before the max_force clamp) of the last step, count*3 floats.
@@ -167,6 +171,13 @@ BOIDS_API int boids_get_steering(boids_ctx* ctx, float* force3);
 
 /* Wait for all enqueued work; returns the first pending CUDA error. */
 BOIDS_API int boids_sync(boids_ctx* ctx);
+
+/* Think-frequency state (complete snapshot together with boids_get_state and
+ * boids_get_neighbors): the step index t of the next step and every owned agent's
+ * stored steering vector (count*3 floats; zero until the agent first thinks).
+ * set: fstore3 NULL keeps the stored vectors.  Both synchronise. */
+BOIDS_API int boids_get_think_state(boids_ctx* ctx, int64_t* step_index, float* fstore3);
+BOIDS_API int boids_set_think_state(boids_ctx* ctx, int64_t step_index, const float* fstore3);
 
 /* Describe the handle (synchronises: it reads the device-side counters). */
 BOIDS_API int boids_info(boids_ctx* ctx, boids_info_t* out);

@@ -43,6 +43,7 @@ class OracleParams(C.Structure):
         ("max_neighbors", C.c_int32),
         ("search_mode", C.c_int32),
         ("init_mode", C.c_int32),
+        ("think_every", C.c_int32),
     ]
 
 
@@ -75,6 +76,8 @@ def lib():
         L.oracle_step.argtypes = [C.c_int64, P, C.c_float] + [f32p] * 5 + [f32p] * 5 + [i32p, i32p, f32p]
         L.oracle_step_sample.argtypes = ([C.c_int64, P, C.c_float] + [f32p] * 5 + [C.c_int64, i64p]
                                          + [f32p] * 5 + [i32p, i32p, f32p])
+        L.oracle_step_think.argtypes = ([C.c_int64, P, C.c_float, C.c_int64] + [f32p] * 5 + [f32p] * 5
+                                        + [i32p, i32p, f32p, f32p])
         L.oracle_run.argtypes = [C.c_int64, P, C.c_float, C.c_int32] + [f32p] * 5
         L.oracle_run.restype = C.c_int
         _lib = L
@@ -185,6 +188,25 @@ def step_sample(s: State, agents, dt: float, params: OracleParams | None = None)
                              out["pos"], out["fwd"], out["up"], out["side"], out["speed"],
                              idx, cnt, F)
     return out, idx, cnt, F
+
+
+def step_think(s: State, dt: float, t: int, fstore, idx7, cnt, params: OracleParams | None = None):
+    """One step with think frequency params.think_every at step index t.
+
+    idx7 (n,7), cnt (n,), fstore (n,3) are the carried think state (copied, not
+    modified).  Returns (State, idx7, cnt, fstore, F_used)."""
+    p = params or default_params()
+    n = s.n
+    out = State(pos=np.empty((n, 3), np.float32), fwd=np.empty((n, 3), np.float32),
+                up=np.empty((n, 3), np.float32), side=np.empty((n, 3), np.float32),
+                speed=np.empty(n, np.float32))
+    idx = np.array(idx7, np.int32, copy=True).reshape(n, 7)
+    c = np.array(cnt, np.int32, copy=True).reshape(n)
+    fs = np.array(fstore, np.float32, copy=True).reshape(n, 3)
+    F = np.empty((n, 3), np.float32)
+    lib().oracle_step_think(n, C.byref(p), C.c_float(dt), t, *_state_arrays(s), out["pos"], out["fwd"],
+                            out["up"], out["side"], out["speed"], idx, c, fs, F)
+    return out, idx, c, fs, F
 
 
 def run(s: State, dt: float, steps: int, params: OracleParams | None = None) -> State:

@@ -58,6 +58,7 @@ typedef struct oracle_params {
   int32_t max_neighbors;/* 7 */
   int32_t search_mode;  /* ignored by the oracle: every mode has one answer */
   int32_t init_mode;    /* 0 = ball of init_radius, 1 = ball of world_radius */
+  int32_t think_every;  /* think frequency k; 1 = every agent thinks every step */
 } oracle_params;
 
 void oracle_default_params(oracle_params* p) {
@@ -74,6 +75,7 @@ void oracle_default_params(oracle_params* p) {
   p->max_neighbors = ORACLE_K;
   p->search_mode = 0;
   p->init_mode = 0;
+  p->think_every = 1;
 }
 
 /* ---------------- Appendix A vector helpers (each op rounded) ------------ */
@@ -313,6 +315,32 @@ void oracle_step_sample(int64_t n, const oracle_params* p, float dt, const float
   for (int64_t k = 0; k < m; ++k)
     step_agent(n, p, dt, pos3, fwd3, up3, side3, speed, agents[k], pos_o + 3 * k, fwd_o + 3 * k,
                up_o + 3 * k, side_o + 3 * k, speed_o + k, idx7 + 7 * k, cnt + k, force3 + 3 * k);
+}
+
+/* One synchronous step with think frequency k = p->think_every (sec 5.3:
+ * "the simulation substage of a specific agent is executed every ten simulation
+ * time steps.  In one simulation time step only 1/10th of the agents execute the
+ * simulation substage").  Readings (Q15): agent i thinks at step t iff
+ * (i + t) mod k == 0; a thinking agent searches + steers and stores its steering
+ * vector in fstore; a non-thinking agent keeps its neighbour list and uses its
+ * stored vector (zero before its first think); every agent runs the
+ * modification substage.  idx7/cnt/fstore are in/out; force3 = F used. */
+void oracle_step_think(int64_t n, const oracle_params* p, float dt, int64_t t, const float* pos3,
+                       const float* fwd3, const float* up3, const float* side3, const float* speed,
+                       float* pos_o, float* fwd_o, float* up_o, float* side_o, float* speed_o,
+                       int32_t* idx7, int32_t* cnt, float* fstore3, float* force3) {
+  int64_t k = p->think_every < 1 ? 1 : p->think_every;
+  for (int64_t i = 0; i < n; ++i) {
+    if ((i + t) % k == 0) {
+      oracle_search_one(n, pos3, p->search_radius, i, idx7 + 7 * i, cnt + i);
+      oracle_steer_one(pos3, fwd3, i, idx7 + 7 * i, cnt[i], p, fstore3 + 3 * i);
+    }
+    force3[3 * i] = fstore3[3 * i];
+    force3[3 * i + 1] = fstore3[3 * i + 1];
+    force3[3 * i + 2] = fstore3[3 * i + 2];
+    oracle_modify_one(pos3 + 3 * i, fwd3 + 3 * i, up3 + 3 * i, side3 + 3 * i, speed[i], force3 + 3 * i, p,
+                      dt, pos_o + 3 * i, fwd_o + 3 * i, up_o + 3 * i, side_o + 3 * i, speed_o + i);
+  }
 }
 
 /* Many synchronous steps (S_t -> S_{t+steps}); state arrays updated in place. */

@@ -31,6 +31,7 @@ EXPORTS = (
     "boids_set_option", "boids_step", "boids_step_shard", "boids_shard_buffers",
     "boids_get_state", "boids_set_state", "boids_get_neighbors", "boids_get_steering",
     "boids_sync", "boids_info", "boids_get_profile", "boids_get_phases", "boids_destroy", "boids_last_error",
+    "boids_get_think_state", "boids_set_think_state",
 )
 
 
@@ -46,7 +47,7 @@ class boids_params(C.Structure):
         ("w_cohesion", C.c_float), ("max_force", C.c_float), ("max_speed", C.c_float),
         ("mass", C.c_float), ("world_radius", C.c_float), ("init_radius", C.c_float),
         ("init_speed_frac", C.c_float), ("max_neighbors", C.c_int32), ("search_mode", C.c_int32),
-        ("init_mode", C.c_int32),
+        ("init_mode", C.c_int32), ("think_every", C.c_int32),
     ]
 
 
@@ -55,7 +56,7 @@ class boids_info_t(C.Structure):
         ("n", C.c_int64), ("lo", C.c_int64), ("hi", C.c_int64), ("slice", C.c_int64),
         ("rank", C.c_int32), ("world", C.c_int32), ("kernel", C.c_int32), ("cluster", C.c_int32),
         ("launches", C.c_int64), ("slow_groups", C.c_int64), ("vote_groups", C.c_int64),
-        ("fallbacks", C.c_int64), ("grid_pairs", C.c_int64),
+        ("fallbacks", C.c_int64), ("grid_pairs", C.c_int64), ("step_index", C.c_int64),
     ]
 
 
@@ -91,6 +92,8 @@ def load(path: str = LIB_PATH):
         "boids_info": (C.c_int, [vp, C.POINTER(boids_info_t)]),
         "boids_get_profile": (C.c_int, [vp, C.POINTER(C.c_double), C.POINTER(i64), i32]),
         "boids_get_phases": (C.c_int, [vp, C.POINTER(C.c_uint64), i64]),
+        "boids_get_think_state": (C.c_int, [vp, C.POINTER(i64), fp]),
+        "boids_set_think_state": (C.c_int, [vp, i64, fp]),
         "boids_destroy": (None, [vp]),
         "boids_last_error": (C.c_char_p, []),
     }
@@ -230,6 +233,18 @@ def boids_get_phases(h: int, ctas: int):
     out = np.zeros((ctas, 8), np.uint64)
     _check(load().boids_get_phases(h, out.ctypes.data_as(C.POINTER(C.c_uint64)), ctas * 8))
     return out
+
+
+def boids_get_think_state(h: int):
+    t = C.c_int64()
+    F = np.empty((_count(h), 3), np.float32)
+    _check(load().boids_get_think_state(h, C.byref(t), _fptr(F)))
+    return t.value, F
+
+
+def boids_set_think_state(h: int, step_index: int, fstore=None):
+    F = None if fstore is None else _f32(fstore, (_count(h), 3))
+    _check(load().boids_set_think_state(h, step_index, _fptr(F)))
 
 
 def boids_destroy(h: int):

@@ -74,6 +74,11 @@ struct boids_ctx {
   int2* gcellrank = nullptr;
   int32_t *gcnt = nullptr, *gstart = nullptr, *gqstart = nullptr, *item_start = nullptr, *counter = nullptr;
   float4* spos = nullptr;
+  // think frequency
+  float4* fstore = nullptr;         // [m] last steering vector per agent
+  unsigned char* routed = nullptr;  // [m] 1 = searched by k_fused this step (think mode)
+  int32_t *tcold = nullptr, *twarm = nullptr, *tcnt = nullptr;  // thinker lists and their counts
+  int64_t step_index = 0, steps_taken = 0;
   int vote_u = 4;          // fused kernel: candidates per warp vote
   int resort_every = 8;    // refresh the spatial query order every this many steps
   int64_t since_sort = -1; // steps since the last refresh (-1: never sorted)
@@ -113,6 +118,7 @@ int validate(const boids_params* p) {
     return fail(BOIDS_EINVAL, "world_radius must be > 0");
   if (!finite(p->init_radius) || p->init_radius <= 0.f)
     return fail(BOIDS_EINVAL, "init_radius must be > 0");
+  if (p->think_every < 1) return fail(BOIDS_EINVAL, "think_every must be >= 1");
   if (!finite(p->init_speed_frac) || p->init_speed_frac < 0.f)
     return fail(BOIDS_EINVAL, "init_speed_frac must be >= 0");
   if (p->search_mode != BOIDS_BRUTE && p->search_mode != BOIDS_GRID)
@@ -150,6 +156,11 @@ void free_ctx(boids_ctx* c) {
   cudaFree(c->item_start);
   cudaFree(c->counter);
   cudaFree(c->spos);
+  cudaFree(c->fstore);
+  cudaFree(c->routed);
+  cudaFree(c->tcold);
+  cudaFree(c->twarm);
+  cudaFree(c->tcnt);
   cudaFree(c->phase);
   for (auto& r : c->recs) {
     cudaEventDestroy(r.a);
@@ -239,7 +250,12 @@ int create_impl(int64_t n, const boids_params* p, uint64_t seed, int32_t rank, i
       (rc = alloc((void**)&c->qperm, m * sizeof(int32_t))) ||
       (rc = alloc((void**)&c->cand, c->ncand * sizeof(float4))) ||
       (rc = alloc((void**)&c->stats, 4 * sizeof(unsigned long long))) ||
-      (rc = alloc((void**)&c->nbr8, m * sizeof(int32_t)))) {
+      (rc = alloc((void**)&c->nbr8, m * sizeof(int32_t))) ||
+      (rc = alloc((void**)&c->fstore, m * sizeof(float4))) ||
+      (rc = alloc((void**)&c->routed, m)) ||
+      (rc = alloc((void**)&c->tcold, m * sizeof(int32_t))) ||
+      (rc = alloc((void**)&c->twarm, m * sizeof(int32_t))) ||
+      (rc = alloc((void**)&c->tcnt, 2 * sizeof(int32_t)))) {
     free_ctx(c);
     return rc;
   }
@@ -269,7 +285,9 @@ int create_impl(int64_t n, const boids_params* p, uint64_t seed, int32_t rank, i
   // phantoms in every segment of every buffer; then the owned agents
   if (e == cudaSuccess) e = cudaMemsetAsync(c->buf[0], 0, shard ? seg * world : seg, s);
   if (e == cudaSuccess) e = cudaMemsetAsync(c->buf[1], 0, seg, s);
-  if (e == cudaSuccess) e = cudaMemsetAsync(c->cnt, 0, m * sizeof(int32_t), s);
+  if (e == cudaSuccess) e = cudaMemsetAsync(c->cnt, 0xFF, m * sizeof(int32_t), s);  // -1: never searched
+  if (e == cudaSuccess) e = cudaMemsetAsync(c->fstore, 0, m * sizeof(float4), s);
+  if (e == cudaSuccess) e = cudaMemsetAsync(c->routed, 0, m, s);
   if (e == cudaSuccess) e = cudaMemsetAsync(c->nbr, 0xFF, m * 7 * sizeof(int32_t), s);
   if (e == cudaSuccess) e = cudaMemsetAsync(c->up4, 0, m * sizeof(float4), s);
   if (e == cudaSuccess) e = cudaMemsetAsync(c->side4, 0, m * sizeof(float4), s);
@@ -325,21 +343,33 @@ StepArgs make_args(boids_ctx* c, float dt) {
   a.partial = c->partial;
   a.pcnt = c->pcnt;
   a.qlim = c->qlim;
+  a.think_k = c->p.think_every;
+  a.store_only = 0;
+  a.step_t = c->step_index;
+  a.fstore = c->fstore;
+  a.qcount = nullptr;
+  a.nq = c->nloc;
+  a.routed = c->p.think_every > 1 ? c->routed : nullptr;
   return a;
 }
 
 int one_step(boids_ctx* c, float dt) {
   StepArgs a = make_args(c, dt);
   int rc;
-  // Only the warm path keeps the 8th-nearest seed consistent with the lists it
-  // writes; any other step invalidates it (a stale seed could repeat one of the
-  // new 7 neighbours and break the t0 bound).
   const bool grid = c->p.search_mode == BOIDS_GRID;
-  const bool warm_path = !grid && c->kernel == BOIDS_KERNEL_FUSED && c->warm;
-  if (!warm_path) CK(cudaMemsetAsync(c->nbr8, 0xFF, c->m * sizeof(int32_t), c->stream));
+  const bool think = c->p.think_every > 1;
+  if (think && !grid && c->kernel != BOIDS_KERNEL_FUSED)
+    return fail(BOIDS_EINVAL, "think frequency runs on the default kernels (BOIDS_KERNEL_FUSED or BOIDS_GRID)");
+  // Only the warm path keeps the 8th-nearest seed consistent with the lists it
+  // writes; other steps invalidate it (a stale seed could repeat one of the new 7
+  // neighbours and break the t0 bound).  Think mode keeps it per agent (k_select
+  // writes it for warm thinkers, k_think_compact clears it for cold ones).
+  const bool warm_path = !grid && !think && c->kernel == BOIDS_KERNEL_FUSED && c->warm;
+  if (!warm_path && !(think && !grid)) CK(cudaMemsetAsync(c->nbr8, 0xFF, c->m * sizeof(int32_t), c->stream));
   if (grid) {
-    // a2: bin all agents (candidates) and the owned ones (queries) by search cell
-    const bool one = !c->shard || c->world == 1;
+    // a2: bin all agents (candidates) and the owned ones (queries) by search cell;
+    // think mode: only this step's thinkers are queries
+    const bool one = (!c->shard || c->world == 1) && !think;
     const int64_t slots = c->shard ? (int64_t)c->world * c->m : c->m;
     const int chunk = grid_chunk();
     if ((rc = launch(c, 2, [&] {
@@ -348,7 +378,8 @@ int one_step(boids_ctx* c, float dt) {
                                       one ? c->item_start : nullptr, chunk, one ? c->counter : nullptr);
            if (e == cudaSuccess && !one)
              e = launch_bin(a.full, c->m, a.sdiv, c->lo, c->nloc, c->sgrid, c->gcellrank, c->gcnt, c->gqstart,
-                            nullptr, c->qperm, (int)c->lo, c->stream, nullptr, c->item_start, chunk, c->counter);
+                            nullptr, c->qperm, (int)c->lo, c->stream, nullptr, c->item_start, chunk, c->counter,
+                            c->p.think_every, c->step_index);
            return e;
          }, one ? 3 : 6)))
       return rc;
@@ -360,7 +391,10 @@ int one_step(boids_ctx* c, float dt) {
     g.item_start = c->item_start;
     g.counter = c->counter;
     g.grid = c->sgrid;
-    if ((rc = launch(c, 3, [&] { return launch_grid(a, g, c->stream); }))) return rc;
+    StepArgs ag = a;
+    ag.store_only = think ? 1 : 0;
+    if ((rc = launch(c, 3, [&] { return launch_grid(ag, g, c->stream); }))) return rc;
+    if (think && (rc = launch(c, 1, [&] { return launch_apply(a, c->stream); }))) return rc;
   } else if (c->kernel == BOIDS_KERNEL_SIMPLE) {
     if ((rc = launch(c, 0, [&] { return launch_search_simple(a, c->stream); }))) return rc;
     if ((rc = launch(c, 1, [&] { return launch_update(a, c->stream); }))) return rc;
@@ -377,7 +411,28 @@ int one_step(boids_ctx* c, float dt) {
       c->since_sort = 0;
     }
     c->since_sort++;
-    if (warm_path) {
+    if (think) {
+      // this step's thinkers, in spatial order, split into never-searched (cold)
+      // and warm-bounded ones
+      CK(cudaMemsetAsync(c->tcnt, 0, 2 * sizeof(int32_t), c->stream));
+      if ((rc = launch(c, 2, [&] {
+             return launch_think_compact(a, c->qperm, c->tcold, c->tcnt, c->twarm, c->tcnt + 1, c->stream);
+           })))
+        return rc;
+      if (c->steps_taken < c->p.think_every) {  // some agents have never thought
+        StepArgs ac = a;
+        ac.qperm = c->tcold;
+        ac.qcount = c->tcnt;
+        ac.store_only = 1;
+        const int cl = c->cluster_opt;
+        if ((rc = launch(c, 0, [&] { return launch_fused(ac, cl, c->stream); }))) return rc;
+      }
+      StepArgs aw = a;
+      aw.qperm = c->twarm;
+      aw.qcount = c->tcnt + 1;
+      if ((rc = launch(c, 0, [&] { return launch_warm_scan(aw, c->stream); }, 2))) return rc;
+      if ((rc = launch(c, 1, [&] { return launch_warm_select(a, c->stream); }))) return rc;
+    } else if (warm_path) {
       // warm step: all-pairs scan appending passing keys, then select + update
       if ((rc = launch(c, 0, [&] { return launch_warm_scan(a, c->stream); }, 2))) return rc;
       if ((rc = launch(c, 1, [&] { return launch_warm_select(a, c->stream); }))) return rc;
@@ -390,6 +445,8 @@ int one_step(boids_ctx* c, float dt) {
   if (!c->shard) c->cur ^= 1;
   c->warm = true;
   c->steering_valid = c->record_steering;
+  c->step_index++;
+  c->steps_taken++;
   return BOIDS_OK;
 }
 
@@ -429,6 +486,7 @@ BOIDS_API void boids_default_params(boids_params* out) {
   out->max_neighbors = 7;
   out->search_mode = BOIDS_BRUTE;
   out->init_mode = BOIDS_INIT_OPENSTEER;
+  out->think_every = 1;
 }
 
 BOIDS_API int boids_create(int64_t n, const boids_params* p, uint64_t seed, boids_ctx** out) {
@@ -627,6 +685,7 @@ BOIDS_API int boids_info(boids_ctx* c, boids_info_t* o) {
   o->vote_groups = (int64_t)st[1];
   o->fallbacks = (int64_t)st[2];
   o->grid_pairs = (int64_t)st[3];
+  o->step_index = c->step_index;
   return BOIDS_OK;
 }
 
@@ -660,6 +719,34 @@ BOIDS_API int boids_get_phases(boids_ctx* c, uint64_t* out, int64_t count) {
   DeviceGuard g(c->dev);
   CK(cudaMemcpyAsync(out, c->phase, count * sizeof(uint64_t), cudaMemcpyDeviceToHost, c->stream));
   CK(cudaStreamSynchronize(c->stream));
+  return BOIDS_OK;
+}
+
+BOIDS_API int boids_get_think_state(boids_ctx* c, int64_t* step_index, float* fstore3) {
+  if (!c) return fail(BOIDS_EINVAL, "NULL handle");
+  DeviceGuard g(c->dev);
+  if (step_index) *step_index = c->step_index;
+  if (fstore3) {
+    std::vector<float4> h((size_t)c->nloc);
+    CK(cudaMemcpyAsync(h.data(), c->fstore, c->nloc * sizeof(float4), cudaMemcpyDeviceToHost, c->stream));
+    CK(cudaStreamSynchronize(c->stream));
+    to_aos(h, c->nloc, fstore3, false);
+  }
+  return BOIDS_OK;
+}
+
+BOIDS_API int boids_set_think_state(boids_ctx* c, int64_t step_index, const float* fstore3) {
+  if (!c) return fail(BOIDS_EINVAL, "NULL handle");
+  if (step_index < 0) return fail(BOIDS_EINVAL, "step_index must be >= 0");
+  DeviceGuard g(c->dev);
+  c->step_index = step_index;
+  if (fstore3) {
+    std::vector<float4> h((size_t)c->nloc);
+    for (int64_t i = 0; i < c->nloc; ++i)
+      h[i] = make_float4(fstore3[3 * i], fstore3[3 * i + 1], fstore3[3 * i + 2], 0.f);
+    CK(cudaMemcpyAsync(c->fstore, h.data(), c->nloc * sizeof(float4), cudaMemcpyHostToDevice, c->stream));
+    CK(cudaStreamSynchronize(c->stream));
+  }
   return BOIDS_OK;
 }
 

@@ -91,6 +91,14 @@ struct StepArgs {
   unsigned long long* partial;  // warm path: [nloc][PSLOTS][7] partial top-7 lists (unbounded agents)
   int32_t* pcnt;              // warm path: [nloc] partial lists written
   float* qlim;                // warm path: [nloc] inclusive search limit min(prev(r2), t0) (k_bound)
+  // think frequency: agent j thinks at step step_t iff (j + step_t) % think_k == 0
+  int32_t think_k;            // 1 = every agent thinks every step
+  int32_t store_only;         // search epilogues store F in fstore instead of modifying
+  int64_t step_t;
+  float4* fstore;             // [nloc] last steering vector of each agent
+  const int32_t* qcount;      // device-side number of query slots (qperm entries), nullptr = nloc
+  int64_t nq;                 // kernel-local copy of the number of query slots
+  unsigned char* routed;      // [nloc] think mode: 1 = searched by k_fused this step (k_select skips)
   unsigned long long* phase;  // diagnostics: per-CTA %globaltimer stamps [grid][8], nullptr = off
   float dt;
   boids_params p;
@@ -107,6 +115,9 @@ struct GridArgs {
   BinGrid grid;
 };
 
+// Does global agent g think at step t (think frequency k)?
+__host__ __device__ inline bool thinks(int64_t g, int64_t t, int32_t k) { return k <= 1 || (g + t) % k == 0; }
+
 // launchers (return the cudaError_t of the launch)
 cudaError_t launch_init(float4* out, float4* up4, float4* side4, int64_t m, int64_t lo,
                         int64_t nloc, const boids_params& p, uint64_t seed, cudaStream_t s);
@@ -115,10 +126,13 @@ cudaError_t launch_fill_phantoms(float4* seg_base, int64_t m, int64_t nloc, int6
 cudaError_t launch_bin(const float4* full, int64_t m, const SliceDiv& sd, int64_t j0, int64_t count, const BinGrid& g,
                        int2* cellrank, int* cnt, int* start, float4* spos, int* perm, int perm_base,
                        cudaStream_t s, int* launches, int* item_start = nullptr, int chunk = 1,
-                       int* counter = nullptr);
+                       int* counter = nullptr, int think_k = 1, int64_t think_t = 0);
 BinGrid make_locality_grid(int64_t n, const boids_params& p);
 BinGrid make_search_grid(const boids_params& p);
 cudaError_t launch_fill_nan(float4* p, int64_t count, cudaStream_t s);
+cudaError_t launch_apply(const StepArgs& a, cudaStream_t s);
+cudaError_t launch_think_compact(const StepArgs& a, const int32_t* qperm, int32_t* cold, int32_t* ncold,
+                                 int32_t* warm, int32_t* nwarm, cudaStream_t s);
 cudaError_t launch_search_simple(const StepArgs& a, cudaStream_t s);
 cudaError_t launch_update(const StepArgs& a, cudaStream_t s);
 cudaError_t launch_fused(const StepArgs& a, int cluster, cudaStream_t s);

@@ -143,6 +143,73 @@ __global__ void __launch_bounds__(256) k_update(StepArgs a) {
   modify_agent(a, i, v3(p4), f4, F);
 }
 
+// Think mode: the modification substage of every owned agent with its stored
+// steering vector (written this step by the searching kernel for thinkers,
+// kept from an earlier step for the others).  HBM-bound: ~64 B in, 64 B out.
+__global__ void __launch_bounds__(256) k_apply(StepArgs a) {
+  int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= a.nloc) return;
+  const float4 p4 = __ldg(pos_of(a.full, a.m, a.sdiv, a.lo + i));
+  const float4 f4 = __ldg(fwd_of(a.full, a.m, a.sdiv, a.lo + i));
+  const float4 F = a.fstore[i];
+  modify_agent(a, i, v3(p4), f4, v3(F));
+}
+
+cudaError_t launch_apply(const StepArgs& a, cudaStream_t s) {
+  if (a.nloc <= 0) return cudaSuccess;
+  k_apply<<<(unsigned)((a.nloc + 255) / 256), 256, 0, s>>>(a);
+  return cudaGetLastError();
+}
+
+// Think mode: split the thinking agents, in qperm (spatial) order, into those
+// never searched (cnt < 0 -> k_fused) and the rest (-> warm scan).  Block-wide
+// compaction keeps 1024 / k consecutive -- spatially coherent -- agents together.
+__global__ void __launch_bounds__(1024) k_think_compact(StepArgs a, const int32_t* __restrict__ qperm,
+                                                        int32_t* cold, int32_t* ncold, int32_t* warm,
+                                                        int32_t* nwarm) {
+  __shared__ int wsum[2][32];
+  __shared__ int base[2];
+  const int64_t s = (int64_t)blockIdx.x * 1024 + threadIdx.x;
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  int qi = -1;
+  bool th = false, c = false;
+  if (s < a.nloc) {
+    qi = qperm[s];
+    th = thinks(a.lo + qi, a.step_t, a.think_k);
+    c = th && a.cnt[qi] < 0;
+    if (th) a.routed[qi] = c ? 1 : 0;
+    if (c) a.nbr8[qi] = -1;
+  }
+  const unsigned bc = __ballot_sync(0xffffffffu, c), bw = __ballot_sync(0xffffffffu, th && !c);
+  if (lane == 0) {
+    wsum[0][w] = __popc(bc);
+    wsum[1][w] = __popc(bw);
+  }
+  __syncthreads();
+  if (threadIdx.x < 64) {  // warp 0: cold scan, warp 1: warm scan (exclusive over warps)
+    const int k = threadIdx.x >> 5;
+    int v = wsum[k][lane], x = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int y = __shfl_up_sync(0xffffffffu, x, o);
+      if (lane >= o) x += y;
+    }
+    wsum[k][lane] = x - v;
+    if (lane == 31) base[k] = atomicAdd(k ? nwarm : ncold, x);
+  }
+  __syncthreads();
+  const unsigned below = (1u << lane) - 1u;
+  if (c) cold[base[0] + wsum[0][w] + __popc(bc & below)] = qi;
+  if (th && !c) warm[base[1] + wsum[1][w] + __popc(bw & below)] = qi;
+}
+
+cudaError_t launch_think_compact(const StepArgs& a, const int32_t* qperm, int32_t* cold, int32_t* ncold,
+                                 int32_t* warm, int32_t* nwarm, cudaStream_t s) {
+  if (a.nloc <= 0) return cudaSuccess;
+  k_think_compact<<<(unsigned)((a.nloc + 1023) / 1024), 1024, 0, s>>>(a, qperm, cold, ncold, warm, nwarm);
+  return cudaGetLastError();
+}
+
 cudaError_t launch_update(const StepArgs& a, cudaStream_t s) {
   if (a.nloc <= 0) return cudaSuccess;
   k_update<<<(unsigned)((a.nloc + 255) / 256), 256, 0, s>>>(a);

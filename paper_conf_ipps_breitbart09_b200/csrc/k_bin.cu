@@ -46,9 +46,14 @@ __device__ __forceinline__ int cell_of(float4 p, const BinGrid& g) {
 // owned agent must get a query slot); otherwise NaN slots -- the phantoms that
 // pad every slice -- are skipped (candidate binning).
 __global__ void k_bin_count(const float4* __restrict__ full, int64_t m, SliceDiv sd, int64_t j0, int64_t count,
-                            BinGrid g, int2* __restrict__ cellrank, int* __restrict__ cnt, int keep_nan) {
+                            BinGrid g, int2* __restrict__ cellrank, int* __restrict__ cnt, int keep_nan,
+                            int think_k, int64_t think_t) {
   int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (k >= count) return;
+  if (!thinks(j0 + k, think_t, think_k)) {  // think mode: only this step's thinkers are queries
+    cellrank[k] = make_int2(-1, 0);
+    return;
+  }
   float4 p = __ldg(pos_of(full, m, sd, j0 + k));
   const bool nan = p.x != p.x || p.y != p.y || p.z != p.z;
   if (nan && !keep_nan) {
@@ -161,7 +166,8 @@ __global__ void k_bin_scatter(const float4* __restrict__ full, int64_t m, SliceD
 
 cudaError_t launch_bin(const float4* full, int64_t m, const SliceDiv& sd, int64_t j0, int64_t count, const BinGrid& g,
                        int2* cellrank, int* cnt, int* start, float4* spos, int* perm, int perm_base,
-                       cudaStream_t s, int* launches, int* item_start, int chunk, int* counter) {
+                       cudaStream_t s, int* launches, int* item_start, int chunk, int* counter, int think_k,
+                       int64_t think_t) {
   const unsigned blocks = (unsigned)((count + 255) / 256);
   if (count <= 0) {  // still publish an empty binning (starts, items, counter)
     const size_t shm0 = (size_t)(g.cells + g.cells / 32 + 1) * sizeof(int);
@@ -169,7 +175,8 @@ cudaError_t launch_bin(const float4* full, int64_t m, const SliceDiv& sd, int64_
     k_bin_scan<<<1, SCAN_T, shm0, s>>>(cnt, start, g.cells, item_start, chunk, counter);
     return cudaGetLastError();
   }
-  k_bin_count<<<blocks, 256, 0, s>>>(full, m, sd, j0, count, g, cellrank, cnt, spos == nullptr);
+  k_bin_count<<<blocks, 256, 0, s>>>(full, m, sd, j0, count, g, cellrank, cnt, spos == nullptr,
+                                     spos == nullptr ? think_k : 1, think_t);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return e;
   const size_t shm = (size_t)(g.cells + g.cells / 32 + 1) * sizeof(int);

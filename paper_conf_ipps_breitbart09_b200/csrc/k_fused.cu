@@ -90,9 +90,14 @@ __device__ __forceinline__ const float4* tile_src(const StepArgs& a, int64_t til
   return pos_of(a.full, a.m, a.sdiv, tile * CT);  // m % CT == 0: a tile never straddles a slice
 }
 
-// local query index held by block slot qs (>= nloc: inactive slot)
+// number of query slots (think mode: a device-side count)
+__device__ __forceinline__ int64_t num_queries(const StepArgs& a) {
+  return a.qcount ? (int64_t)*a.qcount : a.nloc;
+}
+
+// local query index held by block slot qs (>= nq: inactive slot)
 __device__ __forceinline__ int64_t query_of(const StepArgs& a, int64_t qs) {
-  if (qs >= a.nloc) return a.nloc;
+  if (qs >= a.nq) return a.nloc;
   return a.qperm ? (int64_t)__ldg(a.qperm + qs) : qs;
 }
 
@@ -125,11 +130,14 @@ __device__ __forceinline__ void finish_query(const StepArgs& a, int64_t qi, cons
   float4 p4 = __ldg(pos_of(a.full, a.m, a.sdiv, a.lo + qi));
   float4 f4 = __ldg(fwd_of(a.full, a.m, a.sdiv, a.lo + qi));
   V3 F = steer_agent(a, v3(p4), v3(f4), nb, cnt);
-  modify_agent(a, qi, v3(p4), f4, F);
+  if (a.store_only) a.fstore[qi] = make_float4(F.x, F.y, F.z, 0.f);  // think mode: k_apply modifies
+  else modify_agent(a, qi, v3(p4), f4, F);
 }
 
 template <int NT, int K, int U>
 __global__ void __launch_bounds__(NT) k_fused(StepArgs a, int64_t tiles_total) {
+  a.nq = num_queries(a);
+  if ((int64_t)(blockIdx.x / K) * (NT * Q) >= a.nq) return;  // whole cluster: no queries left
   constexpr int QB = NT * Q;    // queries per CTA (and per cluster)
   constexpr int QPC = QB / K;   // queries owned (merged + finished) by each cluster rank
   constexpr int NW = NT / 32;

@@ -62,7 +62,7 @@ struct __align__(16) ScanSmem {
 
 
 __device__ __forceinline__ int64_t query_of(const StepArgs& a, int64_t qs) {
-  if (qs >= a.nloc) return a.nloc;
+  if (qs >= a.nq) return a.nloc;
   return a.qperm ? (int64_t)__ldg(a.qperm + qs) : qs;
 }
 
@@ -157,6 +157,12 @@ __device__ __forceinline__ void stamp_k(const StepArgs& a, int k) {
 
 template <int NTS>
 __global__ void __launch_bounds__(NTS, NTS == 128 ? 4 : 1) k_scan(StepArgs a, int64_t ncand, int64_t items) {
+  if (a.qcount) {  // think mode: query slots counted on the device
+    a.nq = *a.qcount;
+    items = (a.nq + NTS * Q - 1) / (NTS * Q) * ncand;
+  } else {
+    a.nq = a.nloc;
+  }
   constexpr int QBS = NTS * Q;
   extern __shared__ __align__(16) unsigned char smem_raw[];
   ScanSmem<NTS>& sm = *reinterpret_cast<ScanSmem<NTS>*>(smem_raw);
@@ -405,7 +411,11 @@ __device__ __noinline__ void warp_full_search(const StepArgs& a, int64_t qi, key
 
 __global__ void __launch_bounds__(NSEL) k_select(StepArgs a) {
   const int64_t qi = (int64_t)blockIdx.x * NSEL + threadIdx.x;
-  const bool active = qi < a.nloc;
+  // think mode: only warm thinkers were k_scan queries; the others (non-thinkers,
+  // and thinkers searched by k_fused this step) take their stored vector
+  const bool think = qi < a.nloc && thinks(a.lo + qi, a.step_t, a.think_k);
+  const bool routed = think && a.routed && a.routed[qi];
+  const bool active = think && !routed;
   const int c = active ? a.hitcnt[qi] : 0;
   const int pc = active ? a.pcnt[qi] : 0;
   const bool over = active && (c > HITS || pc > PSLOTS);
@@ -440,7 +450,15 @@ __global__ void __launch_bounds__(NSEL) k_select(StepArgs a) {
       for (int s = 0; s < 7; ++s) A[s] = B[s];
     }
   }
-  if (!active) return;
+  if (qi >= a.nloc) return;
+  const float4 p4 = __ldg(pos_of(a.full, a.m, a.sdiv, a.lo + qi));
+  const float4 f4 = __ldg(fwd_of(a.full, a.m, a.sdiv, a.lo + qi));
+  if (!active) {  // think mode, not searched by k_scan this step
+    if (routed) a.routed[qi] = 0;
+    const float4 F = a.fstore[qi];
+    modify_agent(a, qi, v3(p4), f4, v3(F));
+    return;
+  }
   a.hitcnt[qi] = 0;  // ready for the next step
   a.pcnt[qi] = 0;
   a.nbr8[qi] = eighth == KEY_EMPTY ? -1 : key_idx(eighth);
@@ -453,9 +471,8 @@ __global__ void __launch_bounds__(NSEL) k_select(StepArgs a) {
 #pragma unroll
   for (int s = 0; s < 7; ++s) a.nbr[qi * 7 + s] = nb[s];
   a.cnt[qi] = cnt;
-  const float4 p4 = __ldg(pos_of(a.full, a.m, a.sdiv, a.lo + qi));
-  const float4 f4 = __ldg(fwd_of(a.full, a.m, a.sdiv, a.lo + qi));
   const V3 F = steer_agent(a, v3(p4), v3(f4), nb, cnt);
+  if (a.think_k > 1) a.fstore[qi] = make_float4(F.x, F.y, F.z, 0.f);
   modify_agent(a, qi, v3(p4), f4, F);
 }
 
@@ -477,8 +494,9 @@ int scan_grid(int sms) {
 template <int NT>
 cudaError_t scan_with(const StepArgs& a, int sms, int64_t ncand, cudaStream_t s) {
   const int64_t nqb = (a.nloc + NT * Q - 1) / (NT * Q);
-  const int64_t items = nqb * ncand;  // (query block, candidate) pairs
-  const int g = (int)std::min<int64_t>(scan_grid<NT>(sms), (items + CT - 1) / CT);
+  const int64_t items = nqb * ncand;  // (query block, candidate) pairs; think mode: recomputed on device
+  const int g = a.qcount ? scan_grid<NT>(sms)
+                         : (int)std::min<int64_t>(scan_grid<NT>(sms), (items + CT - 1) / CT);
   k_scan<NT><<<g, NT, sizeof(ScanSmem<NT>), s>>>(a, ncand, items);
   return cudaGetLastError();
 }

@@ -49,14 +49,14 @@ def test_struct_layout_matches_header(tmp_path):
     src = tmp_path / "probe.c"
     src.write_text('#include <stddef.h>\n#include <stdio.h>\n#include "boids.h"\n'
                    'int main(void){printf("%zu %zu %zu %zu %zu\\n", sizeof(boids_params), '
-                   'offsetof(boids_params, init_mode), sizeof(boids_info_t), '
-                   'offsetof(boids_info_t, cluster), offsetof(boids_info_t, grid_pairs));return 0;}\n')
+                   'offsetof(boids_params, think_every), sizeof(boids_info_t), '
+                   'offsetof(boids_info_t, cluster), offsetof(boids_info_t, step_index));return 0;}\n')
     exe = tmp_path / "probe"
     subprocess.check_call(["gcc", "-I", os.path.join(ROOT, "include"), str(src), "-o", str(exe)])
     got = list(map(int, subprocess.check_output([str(exe)], text=True).split()))
-    assert got == [C.sizeof(abi.boids_params), abi.boids_params.init_mode.offset,
+    assert got == [C.sizeof(abi.boids_params), abi.boids_params.think_every.offset,
                    C.sizeof(abi.boids_info_t), abi.boids_info_t.cluster.offset,
-                   abi.boids_info_t.grid_pairs.offset]
+                   abi.boids_info_t.step_index.offset]
 
 
 def test_default_params_match_design_table(boidslib, orc):
@@ -71,7 +71,8 @@ def test_default_params_match_design_table(boidslib, orc):
 
 @pytest.mark.parametrize("field,value", [("max_neighbors", 8), ("search_radius", 0.0),
                                          ("search_radius", float("nan")), ("mass", 0.0),
-                                         ("search_mode", 5), ("init_mode", -1), ("max_speed", -1.0)])
+                                         ("search_mode", 5), ("init_mode", -1), ("max_speed", -1.0),
+                                         ("think_every", 0)])
 def test_create_rejects_bad_params(boidslib, field, value):
     from paper_conf_ipps_breitbart09_b200 import abi
 
