@@ -175,12 +175,16 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true", help="skip the e2e leg (profiling runs)")
     ap.add_argument("--kernel", type=int, default=0, help="0 fused (default), 1 two-kernel simple path")
+    ap.add_argument("--think", type=int, default=1,
+                    help="think frequency k (skipThink, P:424): each agent searches every k-th step")
     ap.add_argument("--force-shard", action="store_true",
                     help="use the multi-GPU code path (NCCL process group + sharded handles) even at N=1")
     args = ap.parse_args()
     cfg = W.CONFIGS[args.workload]
     if args.warmup < 3:
         args.warmup = 3  # timing rule: at least 3 warm-up steps
+    if args.think > 1 and args.warmup < args.think + 1:
+        args.warmup = args.think + 1  # steady state: every agent has thought once
     if args.impl == "reference":
         return run_reference(args, cfg)
 
@@ -203,7 +207,8 @@ def main():
     from paper_conf_ipps_breitbart09_b200 import abi
     from paper_conf_ipps_breitbart09_b200.shard import ShardedFlock
 
-    params = pk.boids_default_params(init_mode=cfg.init_mode, search_mode=cfg.search_mode)
+    params = pk.boids_default_params(init_mode=cfg.init_mode, search_mode=cfg.search_mode,
+                                     think_every=max(1, args.think))
     dt = float(W.DT)
     if dist is not None:
         fl = ShardedFlock(cfg.n, params, seed=1, kernel=args.kernel)
@@ -259,10 +264,11 @@ def main():
     kname = "grid_search" if grid else "fused_or_search"
     k_ms, k_n = prof[kname]
     k_ms_per = k_ms / max(k_n, 1)
+    think = max(1, args.think)
     if grid:  # algorithmic work of the grid search: pairs over the 27-cell stencils (device counter)
         pairs_per_launch = float(info1.grid_pairs - info0.grid_pairs) / max(k_n, 1)
-    else:
-        pairs_per_launch = float(nloc) * float(cfg.n)
+    else:  # every thinking agent against all n (think mode: 1/k of the agents per step)
+        pairs_per_launch = float(nloc) * float(cfg.n) / think
     achieved = OPS_PER_PAIR * pairs_per_launch / (k_ms_per / 1e3) / 1e12  # T lane-op/s
     pk_ = peaks()
     sm_max = float(pk_.get("sm_max_mhz", 1965.0))
@@ -287,6 +293,21 @@ def main():
                 "kernel_ms_per_launch": k_ms_per, "kernel_share_of_step": k_ms / ms if ms else None,
                 "frac_at_measured_clock": (achieved / (148 * LANES_PER_SM * clocks["sm_mhz"] * 1e6 / 1e12))
                 if clocks.get("sm_mhz") else None}
+
+    # ---------------- the update (modification) kernel against HBM ----------------
+    u_ms, u_n = prof["update"]
+    update_roofline = None
+    if u_n:
+        hbm = float(pk_.get("hbm_gbs", 6552.0))
+        if think > 1 and grid:  # k_apply: pos4 fwd4 up4 side4 fstore in (80 B), pos4 fwd4 up4 side4 out (64 B)
+            name, per_agent = "k_apply (modification of every agent, think mode)", 144
+        else:  # k_select: hits in, own state in/out; its neighbour gathers hit L2
+            name, per_agent = "k_select (top-7 + steering + modification)", 128 + 8 * 10
+        ub = per_agent * float(nloc) / (u_ms / u_n / 1e3) / 1e9
+        update_roofline = {"bound": "hbm", "kernel": name, "achieved": ub, "peak": hbm, "unit": "GB/s",
+                           "frac": ub / hbm, "bytes_per_agent": per_agent,
+                           "kernel_ms_per_launch": u_ms / u_n,
+                           "peak_note": "hbm_gbs of MEASURED_PEAKS.json (copy bandwidth, measured)"}
 
     # ---------------- e2e through the C ABI with host buffers ----------------
     e2e = None
@@ -330,7 +351,8 @@ def main():
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-            "config": config_dict(cfg, world), "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
+            "config": dict(config_dict(cfg, world), think_every=think), "roofline": roofline,
+            "update_roofline": update_roofline, "cpu_baseline": cpu, "e2e": e2e,
             "gpu_launches": int(launches), "clocks": clocks,
             "kernel_profile_ms": {k: v[0] for k, v in prof.items() if v[1]},
             "thesis_context": "thesis v5 GPU (GeForce 8800 GTS) vs CPU (Athlon 64 3700+): ~42x at 4096 agents "

@@ -272,7 +272,7 @@ int create_impl(int64_t n, const boids_params* p, uint64_t seed, int32_t rank, i
       free_ctx(c);
       return rc;
     }
-  } else if ((rc = alloc((void**)&c->hits, (size_t)m * HITS * sizeof(unsigned long long))) ||
+  } else if ((rc = alloc((void**)&c->hits, (size_t)m * (p->think_every > 1 ? HITS_THINK : HITS) * sizeof(unsigned long long))) ||
              (rc = alloc((void**)&c->hitcnt, m * sizeof(int32_t))) ||
              (rc = alloc((void**)&c->partial, (size_t)m * PSLOTS * 7 * sizeof(unsigned long long))) ||
              (rc = alloc((void**)&c->pcnt, m * sizeof(int32_t))) ||
@@ -338,6 +338,7 @@ StepArgs make_args(boids_ctx* c, float dt) {
   a.phase = c->phase;
   a.vote_u = c->vote_u;
   a.hits = c->hits;
+  a.hits_cap = c->p.think_every > 1 ? HITS_THINK : HITS;
   a.hitcnt = c->hitcnt;
   a.nbr8 = c->nbr8;
   a.partial = c->partial;

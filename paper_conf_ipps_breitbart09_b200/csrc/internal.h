@@ -9,6 +9,7 @@ namespace boids {
 
 constexpr int TILE = 256;  // slice granularity (agents); every slice m is a multiple
 constexpr int HITS = 48;   // warm path: hit-buffer slots per agent (more -> full re-search)
+constexpr int HITS_THINK = 128;  // ... in think mode (bounds from lists up to k steps old are looser)
 constexpr int PSLOTS = 16; // warm path: partial top-7 lists per unbounded agent
 
 // Device view of the agent state for one step.  Layout:
@@ -85,7 +86,8 @@ struct StepArgs {
   const int32_t* qperm;  // local queries in spatial order (local indices); nullptr = identity
   unsigned long long* stats;  // [0] vote groups that took the insertion path, [1] all vote groups
   int32_t vote_u;             // candidates per warp vote in the fused kernel (4 or 8)
-  unsigned long long* hits;   // warm path: [nloc][HITS] passing (d2, index) keys
+  unsigned long long* hits;   // warm path: [nloc][hits_cap] passing (d2, index) keys
+  int32_t hits_cap;           // HITS, or HITS_THINK in think mode
   int32_t* hitcnt;            // warm path: [nloc] number of passing keys (zero between steps)
   int32_t* nbr8;              // [nloc] 8th nearest agent of the last step, or -1 (warm-bound seed)
   unsigned long long* partial;  // warm path: [nloc][PSLOTS][7] partial top-7 lists (unbounded agents)

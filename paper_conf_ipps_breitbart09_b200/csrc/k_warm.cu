@@ -140,10 +140,10 @@ __device__ __forceinline__ void flush(const StepArgs& a, const Rec* rec, int n, 
       r[k] = i < n ? rec[i] : Rec{-1, 0, 0ull};
     }
 #pragma unroll
-    for (int k = 0; k < 8; ++k) slot[k] = r[k].qi >= 0 ? atomicAdd(a.hitcnt + r[k].qi, 1) : HITS;
+    for (int k = 0; k < 8; ++k) slot[k] = r[k].qi >= 0 ? atomicAdd(a.hitcnt + r[k].qi, 1) : a.hits_cap;
 #pragma unroll
     for (int k = 0; k < 8; ++k)
-      if (slot[k] < HITS) a.hits[(int64_t)r[k].qi * HITS + slot[k]] = r[k].key;
+      if (slot[k] < a.hits_cap) a.hits[(int64_t)r[k].qi * a.hits_cap + slot[k]] = r[k].key;
   }
 }
 
@@ -418,7 +418,7 @@ __global__ void __launch_bounds__(NSEL) k_select(StepArgs a) {
   const bool active = think && !routed;
   const int c = active ? a.hitcnt[qi] : 0;
   const int pc = active ? a.pcnt[qi] : 0;
-  const bool over = active && (c > HITS || pc > PSLOTS);
+  const bool over = active && (c > a.hits_cap || pc > PSLOTS);
   key_t A[7];
 #pragma unroll
   for (int s = 0; s < 7; ++s) A[s] = KEY_EMPTY;
@@ -430,9 +430,9 @@ __global__ void __launch_bounds__(NSEL) k_select(StepArgs a) {
       for (int s = 0; s < 7; ++s) B[s] = a.partial[(qi * PSLOTS + p) * 7 + s];
       merge7(A, B);
     }
-    for (int k = 0; k < c; ++k) insert7(A, a.hits[qi * HITS + k]);
+    for (int k = 0; k < c; ++k) insert7(A, a.hits[qi * a.hits_cap + k]);
     for (int k = 0; k < c; ++k) {
-      const key_t h = a.hits[qi * HITS + k];
+      const key_t h = a.hits[qi * a.hits_cap + k];
       if (h > A[6] && h < eighth) eighth = h;
     }
   }
