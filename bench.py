@@ -315,10 +315,14 @@ def main():
         args_e2e = False
     else:
         args_e2e = True
-    st = abi.boids_get_state(h) if args_e2e else {}
-    host = {k: np.ascontiguousarray(v) for k, v in st.items()}
-    h2d = nloc * 4 * 16  # set_state uploads pos4, fwd4 (+speed), up4, side4
-    d2h = nloc * 4 * 16  # get_state downloads pos4, fwd4, up4, side4
+    host = {}
+    if args_e2e:  # pinned host arrays (the contract: inputs from pinned host memory)
+        for k, shape in (("pos", (nloc, 3)), ("fwd", (nloc, 3)), ("up", (nloc, 3)), ("side", (nloc, 3)),
+                         ("speed", (nloc,))):
+            host[k] = torch.empty(shape, dtype=torch.float32, pin_memory=True).numpy()
+        abi.boids_get_state(h, host)
+    h2d = nloc * 13 * 4  # set_state uploads pos3, fwd3, up3, side3, speed (AoS float32)
+    d2h = nloc * 13 * 4  # get_state downloads the same
     if args_e2e:
         barrier()
         t0 = time.perf_counter()
@@ -334,8 +338,8 @@ def main():
             e2e_s = float(t.item())
         e2e = {"value": cfg.n * args.steps / e2e_s, "unit": UNIT, "h2d_bytes_per_step": h2d * world,
                "d2h_bytes_per_step": d2h * world,
-               "note": "boids_set_state (host AoS -> device) + step + boids_get_state (device -> host AoS), "
-                       "wall clock"}
+               "note": "pinned host AoS arrays: boids_set_state (H2D + device conversion) + step + "
+                       "boids_get_state (device conversion + D2H), wall clock"}
 
     # ---------------- CPU oracle baseline (rank 0, N=1) ----------------
     cpu = None

@@ -74,6 +74,7 @@ struct boids_ctx {
   int2* gcellrank = nullptr;
   int32_t *gcnt = nullptr, *gstart = nullptr, *gqstart = nullptr, *item_start = nullptr, *counter = nullptr;
   float4* spos = nullptr;
+  float* stage = nullptr;  // host-transfer staging [13][m] (lazy)
   // think frequency
   float4* fstore = nullptr;         // [m] last steering vector per agent
   unsigned char* routed = nullptr;  // [m] 1 = searched by k_fused this step (think mode)
@@ -156,6 +157,7 @@ void free_ctx(boids_ctx* c) {
   cudaFree(c->item_start);
   cudaFree(c->counter);
   cudaFree(c->spos);
+  cudaFree(c->stage);
   cudaFree(c->fstore);
   cudaFree(c->routed);
   cudaFree(c->tcold);
@@ -579,33 +581,36 @@ BOIDS_API int boids_shard_buffers(boids_ctx* c, void** send, void** full, int64_
   return BOIDS_OK;
 }
 
+// Host AoS <-> device float4 state goes through a device staging buffer of 13
+// floats per agent ([pos3 | fwd3 | up3 | side3 | speed]) and one conversion
+// kernel: the copies are plain DMA of the caller's arrays (pinned memory: full
+// PCIe/C2C rate), no host-side conversion loops.
+static int ensure_stage(boids_ctx* c) {
+  if (!c->stage) {
+    cudaError_t e = cudaMalloc((void**)&c->stage, (size_t)13 * (c->m > 0 ? c->m : 1) * sizeof(float));
+    if (e != cudaSuccess) {
+      (void)cudaGetLastError();
+      return fail(BOIDS_ENOMEM, std::string("cudaMalloc: ") + cudaGetErrorString(e));
+    }
+  }
+  return BOIDS_OK;
+}
+
 BOIDS_API int boids_get_state(boids_ctx* c, float* pos3, float* fwd3, float* up3, float* side3, float* speed) {
   if (!c) return fail(BOIDS_EINVAL, "NULL handle");
   DeviceGuard g(c->dev);
-  int64_t k = c->nloc, m = c->m;
-  std::vector<float4> h((size_t)k);
-  const float4* L = c->local();
-  if (pos3) {
-    CK(cudaMemcpyAsync(h.data(), L, k * sizeof(float4), cudaMemcpyDeviceToHost, c->stream));
-    CK(cudaStreamSynchronize(c->stream));
-    to_aos(h, k, pos3, false);
-  }
-  if (fwd3 || speed) {
-    CK(cudaMemcpyAsync(h.data(), L + m, k * sizeof(float4), cudaMemcpyDeviceToHost, c->stream));
-    CK(cudaStreamSynchronize(c->stream));
-    if (fwd3) to_aos(h, k, fwd3, false);
-    if (speed) to_aos(h, k, speed, true);
-  }
-  if (up3) {
-    CK(cudaMemcpyAsync(h.data(), c->up4, k * sizeof(float4), cudaMemcpyDeviceToHost, c->stream));
-    CK(cudaStreamSynchronize(c->stream));
-    to_aos(h, k, up3, false);
-  }
-  if (side3) {
-    CK(cudaMemcpyAsync(h.data(), c->side4, k * sizeof(float4), cudaMemcpyDeviceToHost, c->stream));
-    CK(cudaStreamSynchronize(c->stream));
-    to_aos(h, k, side3, false);
-  }
+  int rc = ensure_stage(c);
+  if (rc) return rc;
+  const int64_t k = c->nloc;
+  float* st = c->stage;
+  CK(launch_state_out(c->local(), c->m, c->up4, c->side4, k, st, c->stream));
+  c->launches++;
+  const size_t v = (size_t)k * 3 * sizeof(float);
+  if (pos3) CK(cudaMemcpyAsync(pos3, st, v, cudaMemcpyDeviceToHost, c->stream));
+  if (fwd3) CK(cudaMemcpyAsync(fwd3, st + 3 * k, v, cudaMemcpyDeviceToHost, c->stream));
+  if (up3) CK(cudaMemcpyAsync(up3, st + 6 * k, v, cudaMemcpyDeviceToHost, c->stream));
+  if (side3) CK(cudaMemcpyAsync(side3, st + 9 * k, v, cudaMemcpyDeviceToHost, c->stream));
+  if (speed) CK(cudaMemcpyAsync(speed, st + 12 * k, k * sizeof(float), cudaMemcpyDeviceToHost, c->stream));
   CK(cudaStreamSynchronize(c->stream));
   return BOIDS_OK;
 }
@@ -615,20 +620,18 @@ BOIDS_API int boids_set_state(boids_ctx* c, const float* pos3, const float* fwd3
   if (!c) return fail(BOIDS_EINVAL, "NULL handle");
   if (!pos3 || !fwd3 || !up3 || !speed) return fail(BOIDS_EINVAL, "pos3, fwd3, up3, speed required");
   DeviceGuard g(c->dev);
-  int64_t k = c->nloc, m = c->m;
-  std::vector<float4> hp((size_t)k), hf((size_t)k), hu((size_t)k), hs((size_t)k);
-  for (int64_t i = 0; i < k; ++i) {
-    hp[i] = make_float4(pos3[3 * i], pos3[3 * i + 1], pos3[3 * i + 2], 0.f);
-    hf[i] = make_float4(fwd3[3 * i], fwd3[3 * i + 1], fwd3[3 * i + 2], speed[i]);
-    hu[i] = make_float4(up3[3 * i], up3[3 * i + 1], up3[3 * i + 2], 0.f);
-    hs[i] = side3 ? make_float4(side3[3 * i], side3[3 * i + 1], side3[3 * i + 2], 0.f)
-                  : make_float4(0.f, 0.f, 0.f, 0.f);
-  }
-  float4* L = c->local();
-  CK(cudaMemcpyAsync(L, hp.data(), k * sizeof(float4), cudaMemcpyHostToDevice, c->stream));
-  CK(cudaMemcpyAsync(L + m, hf.data(), k * sizeof(float4), cudaMemcpyHostToDevice, c->stream));
-  CK(cudaMemcpyAsync(c->up4, hu.data(), k * sizeof(float4), cudaMemcpyHostToDevice, c->stream));
-  CK(cudaMemcpyAsync(c->side4, hs.data(), k * sizeof(float4), cudaMemcpyHostToDevice, c->stream));
+  int rc = ensure_stage(c);
+  if (rc) return rc;
+  const int64_t k = c->nloc;
+  float* st = c->stage;
+  const size_t v = (size_t)k * 3 * sizeof(float);
+  CK(cudaMemcpyAsync(st, pos3, v, cudaMemcpyHostToDevice, c->stream));
+  CK(cudaMemcpyAsync(st + 3 * k, fwd3, v, cudaMemcpyHostToDevice, c->stream));
+  CK(cudaMemcpyAsync(st + 6 * k, up3, v, cudaMemcpyHostToDevice, c->stream));
+  if (side3) CK(cudaMemcpyAsync(st + 9 * k, side3, v, cudaMemcpyHostToDevice, c->stream));
+  CK(cudaMemcpyAsync(st + 12 * k, speed, k * sizeof(float), cudaMemcpyHostToDevice, c->stream));
+  CK(launch_state_in(st, side3 != nullptr, k, c->local(), c->m, c->up4, c->side4, c->stream));
+  c->launches++;
   // The previous neighbour lists are KEPT: the warm bound they seed (the 7th
   // smallest current distance to 7-8 distinct existing agents) is an upper bound
   // on the 7th neighbour distance for ANY positions, so the next step stays exact;

@@ -83,6 +83,51 @@ cudaError_t launch_fill_nan(float4* p, int64_t count, cudaStream_t s) {
   return cudaGetLastError();
 }
 
+// Host-transfer staging: [pos3 | fwd3 | up3 | side3 | speed] (k agents each) <-> float4 state.
+__global__ void k_state_in(const float* __restrict__ st, int has_side, int64_t k, float4* local, int64_t m,
+                           float4* up4, float4* side4) {
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= k) return;
+  const float* p = st + 3 * i;
+  const float* f = st + 3 * k + 3 * i;
+  const float* u = st + 6 * k + 3 * i;
+  const float* s = st + 9 * k + 3 * i;
+  local[i] = make_float4(p[0], p[1], p[2], 0.f);
+  local[m + i] = make_float4(f[0], f[1], f[2], st[12 * k + i]);
+  up4[i] = make_float4(u[0], u[1], u[2], 0.f);
+  side4[i] = has_side ? make_float4(s[0], s[1], s[2], 0.f) : make_float4(0.f, 0.f, 0.f, 0.f);
+}
+
+__global__ void k_state_out(const float4* __restrict__ local, int64_t m, const float4* __restrict__ up4,
+                            const float4* __restrict__ side4, int64_t k, float* st) {
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= k) return;
+  const float4 p = local[i], f = local[m + i], u = up4[i], s = side4[i];
+  float* P = st + 3 * i;
+  float* F = st + 3 * k + 3 * i;
+  float* Uu = st + 6 * k + 3 * i;
+  float* S = st + 9 * k + 3 * i;
+  P[0] = p.x, P[1] = p.y, P[2] = p.z;
+  F[0] = f.x, F[1] = f.y, F[2] = f.z;
+  Uu[0] = u.x, Uu[1] = u.y, Uu[2] = u.z;
+  S[0] = s.x, S[1] = s.y, S[2] = s.z;
+  st[12 * k + i] = f.w;
+}
+
+cudaError_t launch_state_in(const float* stage, bool has_side, int64_t k, float4* local, int64_t m, float4* up4,
+                            float4* side4, cudaStream_t s) {
+  if (k <= 0) return cudaSuccess;
+  k_state_in<<<(unsigned)((k + 255) / 256), 256, 0, s>>>(stage, has_side ? 1 : 0, k, local, m, up4, side4);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_state_out(const float4* local, int64_t m, const float4* up4, const float4* side4, int64_t k,
+                             float* stage, cudaStream_t s) {
+  if (k <= 0) return cudaSuccess;
+  k_state_out<<<(unsigned)((k + 255) / 256), 256, 0, s>>>(local, m, up4, side4, k, stage);
+  return cudaGetLastError();
+}
+
 // ------------------------------------------------------- simple search ----
 // One thread per owned agent; candidate positions staged through shared memory
 // one TILE at a time (the thesis's version-2 structure, Listing 6.2), register
