@@ -341,6 +341,28 @@ def main():
                "note": "pinned host AoS arrays: boids_set_state (H2D + device conversion) + step + "
                        "boids_get_state (device conversion + D2H), wall clock"}
 
+    # ---------------- the thesis's draw loop: step + double-buffered readback ----------------
+    # (the host consumes step n's 4x4 draw matrices while step n+1 runs)
+    e2e_draw = None
+    if args_e2e:
+        bufs = [torch.empty((nloc, 4, 4), dtype=torch.float32, pin_memory=True).numpy() for _ in range(2)]
+        barrier()
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        for k in range(args.steps):
+            step()
+            abi.boids_readback_begin(h, bufs[k % 2])
+        abi.boids_readback_wait(h)
+        e2e_draw_s = time.perf_counter() - t0
+        if dist is not None:
+            t = torch.tensor([e2e_draw_s], device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            e2e_draw_s = float(t.item())
+        e2e_draw = {"value": cfg.n * args.steps / e2e_draw_s, "unit": UNIT, "h2d_bytes_per_step": 0,
+                    "d2h_bytes_per_step": nloc * 64 * world,
+                    "note": "steps with the 4x4 draw matrices (64 B/agent) read back every step on a copy "
+                            "stream into alternating pinned buffers (double buffering, P:535-539), wall clock"}
+
     # ---------------- CPU oracle baseline (rank 0, N=1) ----------------
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
@@ -356,7 +378,7 @@ def main():
             "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
             "config": dict(config_dict(cfg, world), think_every=think), "roofline": roofline,
-            "update_roofline": update_roofline, "cpu_baseline": cpu, "e2e": e2e,
+            "update_roofline": update_roofline, "cpu_baseline": cpu, "e2e": e2e, "e2e_draw": e2e_draw,
             "gpu_launches": int(launches), "clocks": clocks,
             "kernel_profile_ms": {k: v[0] for k, v in prof.items() if v[1]},
             "thesis_context": "thesis v5 GPU (GeForce 8800 GTS) vs CPU (Athlon 64 3700+): ~42x at 4096 agents "

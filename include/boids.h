@@ -172,6 +172,20 @@ BOIDS_API int boids_get_steering(boids_ctx* ctx, float* force3);
 /* Wait for all enqueued work; returns the first pending CUDA error. */
 BOIDS_API int boids_sync(boids_ctx* ctx);
 
+/* Double-buffered asynchronous readback of the draw data (the thesis's double
+ * buffering; "only the required information to draw the agents -- a
+ * 4x4 matrix containing 16 float values -- is moved from the device").
+ * begin: enqueue, on the handle's stream, a kernel packing each owned agent's
+ * 4x4 local-space matrix of the CURRENT state (rows side, up, fwd, pos as
+ * (x,y,z,0|0|0|1), count*16 floats, row-major) into a device buffer, then a copy
+ * to host16 on a separate copy stream; returns at once, so later boids_step
+ * calls overlap the copy.  At most one readback in flight per handle (begin
+ * waits for the previous one).  host16 should be pinned (page-locked) memory and
+ * must stay valid until boids_readback_wait; alternate two host buffers to draw
+ * step n while step n+1 runs.  wait: block until the readback landed in host16. */
+BOIDS_API int boids_readback_begin(boids_ctx* ctx, float* host16);
+BOIDS_API int boids_readback_wait(boids_ctx* ctx);
+
 /* Think-frequency state (complete snapshot together with boids_get_state and
  * boids_get_neighbors): the step index t of the next step and every owned agent's
  * stored steering vector (count*3 floats; zero until the agent first thinks).

@@ -31,7 +31,7 @@ EXPORTS = (
     "boids_set_option", "boids_step", "boids_step_shard", "boids_shard_buffers",
     "boids_get_state", "boids_set_state", "boids_get_neighbors", "boids_get_steering",
     "boids_sync", "boids_info", "boids_get_profile", "boids_get_phases", "boids_destroy", "boids_last_error",
-    "boids_get_think_state", "boids_set_think_state",
+    "boids_get_think_state", "boids_set_think_state", "boids_readback_begin", "boids_readback_wait",
 )
 
 
@@ -92,6 +92,8 @@ def load(path: str = LIB_PATH):
         "boids_info": (C.c_int, [vp, C.POINTER(boids_info_t)]),
         "boids_get_profile": (C.c_int, [vp, C.POINTER(C.c_double), C.POINTER(i64), i32]),
         "boids_get_phases": (C.c_int, [vp, C.POINTER(C.c_uint64), i64]),
+        "boids_readback_begin": (C.c_int, [vp, fp]),
+        "boids_readback_wait": (C.c_int, [vp]),
         "boids_get_think_state": (C.c_int, [vp, C.POINTER(i64), fp]),
         "boids_set_think_state": (C.c_int, [vp, i64, fp]),
         "boids_destroy": (None, [vp]),
@@ -233,6 +235,17 @@ def boids_get_phases(h: int, ctas: int):
     out = np.zeros((ctas, 8), np.uint64)
     _check(load().boids_get_phases(h, out.ctypes.data_as(C.POINTER(C.c_uint64)), ctas * 8))
     return out
+
+
+def boids_readback_begin(h: int, host16) -> None:
+    """host16: float32 (count, 4, 4), C-contiguous, ideally pinned; must outlive the readback."""
+    if host16.dtype != np.float32 or not host16.flags["C_CONTIGUOUS"] or host16.size != _count(h) * 16:
+        raise ValueError("host16 must be a C-contiguous float32 array of count*16 elements")
+    _check(load().boids_readback_begin(h, _fptr(host16)))
+
+
+def boids_readback_wait(h: int) -> None:
+    _check(load().boids_readback_wait(h))
 
 
 def boids_get_think_state(h: int):

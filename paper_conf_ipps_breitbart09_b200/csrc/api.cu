@@ -75,6 +75,11 @@ struct boids_ctx {
   int32_t *gcnt = nullptr, *gstart = nullptr, *gqstart = nullptr, *item_start = nullptr, *counter = nullptr;
   float4* spos = nullptr;
   float* stage = nullptr;  // host-transfer staging [13][m] (lazy)
+  // double-buffered readback (lazy): packed draw matrices, copy stream, events
+  float4* draw = nullptr;  // [m][4] rows
+  cudaStream_t copy_stream = nullptr;
+  cudaEvent_t packed = nullptr, landed = nullptr;
+  bool rb_pending = false;
   // think frequency
   float4* fstore = nullptr;         // [m] last steering vector per agent
   unsigned char* routed = nullptr;  // [m] 1 = searched by k_fused this step (think mode)
@@ -158,6 +163,11 @@ void free_ctx(boids_ctx* c) {
   cudaFree(c->counter);
   cudaFree(c->spos);
   cudaFree(c->stage);
+  if (c->rb_pending) cudaEventSynchronize(c->landed);
+  cudaFree(c->draw);
+  if (c->packed) cudaEventDestroy(c->packed);
+  if (c->landed) cudaEventDestroy(c->landed);
+  if (c->copy_stream) cudaStreamDestroy(c->copy_stream);
   cudaFree(c->fstore);
   cudaFree(c->routed);
   cudaFree(c->tcold);
@@ -723,6 +733,36 @@ BOIDS_API int boids_get_phases(boids_ctx* c, uint64_t* out, int64_t count) {
   DeviceGuard g(c->dev);
   CK(cudaMemcpyAsync(out, c->phase, count * sizeof(uint64_t), cudaMemcpyDeviceToHost, c->stream));
   CK(cudaStreamSynchronize(c->stream));
+  return BOIDS_OK;
+}
+
+BOIDS_API int boids_readback_begin(boids_ctx* c, float* host16) {
+  if (!c || !host16) return fail(BOIDS_EINVAL, "NULL argument");
+  DeviceGuard g(c->dev);
+  if (!c->draw) {
+    CK(cudaMalloc((void**)&c->draw, (size_t)(c->m > 0 ? c->m : 1) * 4 * sizeof(float4)));
+    CK(cudaStreamCreateWithFlags(&c->copy_stream, cudaStreamNonBlocking));
+    CK(cudaEventCreateWithFlags(&c->packed, cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&c->landed, cudaEventDisableTiming));
+  }
+  if (c->rb_pending) CK(cudaEventSynchronize(c->landed));  // one in flight (the draw buffer is reused)
+  // pack on the compute stream (ordered after the last step), copy on the copy stream
+  CK(launch_pack_draw(c->local(), c->m, c->up4, c->side4, c->nloc, c->draw, c->stream));
+  c->launches++;
+  CK(cudaEventRecord(c->packed, c->stream));
+  CK(cudaStreamWaitEvent(c->copy_stream, c->packed, 0));
+  CK(cudaMemcpyAsync(host16, c->draw, c->nloc * 4 * sizeof(float4), cudaMemcpyDeviceToHost, c->copy_stream));
+  CK(cudaEventRecord(c->landed, c->copy_stream));
+  c->rb_pending = true;
+  return BOIDS_OK;
+}
+
+BOIDS_API int boids_readback_wait(boids_ctx* c) {
+  if (!c) return fail(BOIDS_EINVAL, "NULL handle");
+  if (!c->rb_pending) return BOIDS_OK;
+  DeviceGuard g(c->dev);
+  CK(cudaEventSynchronize(c->landed));
+  c->rb_pending = false;
   return BOIDS_OK;
 }
 

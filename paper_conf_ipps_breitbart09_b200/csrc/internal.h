@@ -133,6 +133,8 @@ BinGrid make_locality_grid(int64_t n, const boids_params& p);
 BinGrid make_search_grid(const boids_params& p);
 cudaError_t launch_fill_nan(float4* p, int64_t count, cudaStream_t s);
 cudaError_t launch_apply(const StepArgs& a, cudaStream_t s);
+cudaError_t launch_pack_draw(const float4* local, int64_t m, const float4* up4, const float4* side4, int64_t k,
+                             float4* draw, cudaStream_t s);
 cudaError_t launch_state_in(const float* stage, bool has_side, int64_t k, float4* local, int64_t m, float4* up4,
                             float4* side4, cudaStream_t s);
 cudaError_t launch_state_out(const float4* local, int64_t m, const float4* up4, const float4* side4, int64_t k,

@@ -128,6 +128,26 @@ cudaError_t launch_state_out(const float4* local, int64_t m, const float4* up4, 
   return cudaGetLastError();
 }
 
+// Draw data of the double-buffered readback: the 4x4 local-space matrix per agent
+// (rows side, up, forward, position), 64 B, packed contiguously.
+__global__ void k_pack_draw(const float4* __restrict__ local, int64_t m, const float4* __restrict__ up4,
+                            const float4* __restrict__ side4, int64_t k, float4* __restrict__ draw) {
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= k) return;
+  const float4 s = side4[i], u = up4[i], f = local[m + i], p = local[i];
+  draw[4 * i + 0] = make_float4(s.x, s.y, s.z, 0.f);
+  draw[4 * i + 1] = make_float4(u.x, u.y, u.z, 0.f);
+  draw[4 * i + 2] = make_float4(f.x, f.y, f.z, 0.f);
+  draw[4 * i + 3] = make_float4(p.x, p.y, p.z, 1.f);
+}
+
+cudaError_t launch_pack_draw(const float4* local, int64_t m, const float4* up4, const float4* side4, int64_t k,
+                             float4* draw, cudaStream_t s) {
+  if (k <= 0) return cudaSuccess;
+  k_pack_draw<<<(unsigned)((k + 255) / 256), 256, 0, s>>>(local, m, up4, side4, k, draw);
+  return cudaGetLastError();
+}
+
 // ------------------------------------------------------- simple search ----
 // One thread per owned agent; candidate positions staged through shared memory
 // one TILE at a time (the thesis's version-2 structure, Listing 6.2), register

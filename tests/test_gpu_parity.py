@@ -320,3 +320,29 @@ def test_config_c5_sampled(pk, orc):
         np.testing.assert_allclose(f.steering()[ag], o_F, rtol=RTOL, atol=ATOL)
         for k in KEYS:
             np.testing.assert_array_equal(g[k][ag], o[k])
+
+
+# ----------------------------------------- double-buffered readback
+def test_readback_draw_matrix_double_buffered(pk):
+    """boids_readback_begin packs the 4x4 draw matrices (side, up, fwd, pos) of the
+    current state and copies them on a second stream while later steps run."""
+    import torch
+
+    from paper_conf_ipps_breitbart09_b200 import abi
+
+    n = 5000
+    p = pk.boids_default_params(init_mode=1)
+    bufs = [torch.empty((n, 4, 4), dtype=torch.float32, pin_memory=True).numpy() for _ in range(2)]
+    with pk.Flock(n, p, seed=4) as f, pk.Flock(n, p, seed=4) as ref:
+        states = []
+        for t in range(4):
+            f.step(DT, 1)
+            abi.boids_readback_begin(f.h, bufs[t % 2])  # waits for the previous copy only
+            ref.step(DT, 1)
+            states.append(ref.state())
+        abi.boids_readback_wait(f.h)
+        for t in (2, 3):  # the two buffers hold the last two steps
+            m, s = bufs[t % 2], states[t]
+            assert np.array_equal(m[:, 0, :3], s["side"]) and np.array_equal(m[:, 1, :3], s["up"])
+            assert np.array_equal(m[:, 2, :3], s["fwd"]) and np.array_equal(m[:, 3, :3], s["pos"])
+            assert (m[:, :3, 3] == 0).all() and (m[:, 3, 3] == 1).all()
