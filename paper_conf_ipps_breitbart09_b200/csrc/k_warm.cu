@@ -501,6 +501,13 @@ cudaError_t scan_with(const StepArgs& a, int sms, int64_t ncand, cudaStream_t s)
   return cudaGetLastError();
 }
 
+#ifndef BOIDS_SCAN_BIG
+#define BOIDS_SCAN_BIG 512  // 640 (20 warps) caps registers at 96 and spills: measured 15% slower
+#endif
+cudaError_t scan_big(const StepArgs& a, int sms, int64_t ncand, cudaStream_t s) {
+  return scan_with<BOIDS_SCAN_BIG>(a, sms, ncand, s);
+}
+
 cudaError_t launch_warm_scan(const StepArgs& a, cudaStream_t s) {
   if (a.nloc <= 0) return cudaSuccess;
   k_bound<<<(unsigned)((a.nloc + 255) / 256), 256, 0, s>>>(a);
@@ -511,7 +518,7 @@ cudaError_t launch_warm_scan(const StepArgs& a, cudaStream_t s) {
   const int64_t ncand = (int64_t)a.world * a.m;
   // one 512-thread CTA per SM when every SM gets >= 4 tiles of (2048 queries x CT)
   const int64_t tiles512 = (a.nloc + 2047) / 2048 * (ncand / CT);
-  if (tiles512 >= 4LL * sms) return scan_with<512>(a, sms, ncand, s);
+  if (tiles512 >= 4LL * sms) return scan_big(a, sms, ncand, s);
   return scan_with<128>(a, sms, ncand, s);
 }
 
