@@ -177,6 +177,9 @@ def main():
     ap.add_argument("--kernel", type=int, default=0, help="0 fused (default), 1 two-kernel simple path")
     ap.add_argument("--think", type=int, default=1,
                     help="think frequency k (skipThink, P:424): each agent searches every k-th step")
+    ap.add_argument("--no-sym", action="store_true",
+                    help="single-GPU brute force: evaluate every ordered pair (k_scan) instead of each "
+                         "unordered pair once (k_sym, default)")
     ap.add_argument("--force-shard", action="store_true",
                     help="use the multi-GPU code path (NCCL process group + sharded handles) even at N=1")
     args = ap.parse_args()
@@ -216,7 +219,7 @@ def main():
         step = lambda: fl.step(dt, 1)  # noqa: E731
         nloc = fl.hi - fl.lo
     else:
-        fl = pk.Flock(cfg.n, params, seed=1, kernel=args.kernel)
+        fl = pk.Flock(cfg.n, params, seed=1, kernel=args.kernel, symmetric=not args.no_sym)
         h = fl.h
         step = lambda: fl.step(dt, 1)  # noqa: E731
         nloc = cfg.n
@@ -265,10 +268,16 @@ def main():
     k_ms, k_n = prof[kname]
     k_ms_per = k_ms / max(k_n, 1)
     think = max(1, args.think)
+    sym = dist is None and not grid and think == 1 and not args.no_sym and args.kernel == 0
     if grid:  # algorithmic work of the grid search: pairs over the 27-cell stencils (device counter)
         pairs_per_launch = float(info1.grid_pairs - info0.grid_pairs) / max(k_n, 1)
+        pairs_note = " (27-cell stencil candidates, device counter)"
+    elif sym:  # k_sym: every unordered pair once, tested against both agents' limits
+        pairs_per_launch = float(cfg.n) * float(cfg.n - 1) / 2
+        pairs_note = " (n(n-1)/2 unordered pairs: d2 is symmetric, each evaluated once for both agents)"
     else:  # every thinking agent against all n (think mode: 1/k of the agents per step)
         pairs_per_launch = float(nloc) * float(cfg.n) / think
+        pairs_note = " (n_local x n ordered pairs)"
     achieved = OPS_PER_PAIR * pairs_per_launch / (k_ms_per / 1e3) / 1e12  # T lane-op/s
     pk_ = peaks()
     sm_max = float(pk_.get("sm_max_mhz", 1965.0))
@@ -283,16 +292,22 @@ def main():
             traffic = None
     roofline = {"bound": "alu",
                 "kernel": ("k_grid (binned search + steer + modify)" if grid else
-                           "k_scan (warm-step all-pairs search; k_fused on cold steps)"),
+                           "k_sym_prep + k_sym (warm-step unordered-pair search)" if sym else
+                           "k_bound + k_scan (warm-step all-pairs search; k_fused on cold steps)"),
                 "achieved": achieved, "peak": peak, "unit": "TFLOP/s", "frac": achieved / peak,
                 "traffic": traffic,
                 "peak_note": f"FP32 SIMT lane-ops: 148 SM x 128 lanes x {sm_max:.0f} MHz "
                              f"(sm_max_mhz of MEASURED_PEAKS.json; each add/sub/mul counted once, no FMA)",
-                "work_per_launch": f"{OPS_PER_PAIR} lane-ops x {pairs_per_launch:.4g} pairs"
-                                   + (" (27-cell stencil candidates, device counter)" if grid else " (n_local x n)"),
+                "work_per_launch": f"{OPS_PER_PAIR} lane-ops x {pairs_per_launch:.4g} pairs" + pairs_note,
                 "kernel_ms_per_launch": k_ms_per, "kernel_share_of_step": k_ms / ms if ms else None,
                 "frac_at_measured_clock": (achieved / (148 * LANES_PER_SM * clocks["sm_mhz"] * 1e6 / 1e12))
                 if clocks.get("sm_mhz") else None}
+    if sym:  # the thesis's per-agent formulation evaluates n x n ordered pairs
+        roofline["ordered_pair_equivalent"] = {
+            "achieved": 2 * achieved * cfg.n / (cfg.n - 1) if cfg.n > 1 else 0.0,
+            "frac_of_peak": (2 * achieved * cfg.n / (cfg.n - 1) if cfg.n > 1 else 0.0) / peak,
+            "note": "n x n pairs of the thesis's formulation / the same kernel time: the rate an "
+                    "ordered-pair kernel would need to match; not a hardware utilisation"}
 
     # ---------------- the update (modification) kernel against HBM ----------------
     u_ms, u_n = prof["update"]

@@ -112,6 +112,10 @@ typedef struct boids_info_t {
 #define BOIDS_OPT_RESORT 6          /* refresh the spatial order of the fused kernel's query blocks every
                                        `value` steps (default 8; results never depend on it) */
 #define BOIDS_OPT_VOTE_U 7          /* fused kernel: candidates per warp vote, 4 (default) or 8 */
+#define BOIDS_OPT_SYMMETRIC 8       /* warm brute-force steps of a single-GPU handle with n >= 8192:
+                                       1 (default) = evaluate every unordered pair once and test it
+                                       against both agents' limits (k_sym; d2 is bitwise symmetric),
+                                       0 = every ordered pair (k_scan).  Results are identical. */
 #define BOIDS_OPT_PHASES 5          /* diagnostics: value = max CTAs; the fused kernel records per-CTA
                                        %globaltimer stamps (read with boids_get_phases); 0 = off */
 

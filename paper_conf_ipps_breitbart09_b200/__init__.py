@@ -32,7 +32,8 @@ class Flock:
     """One single-rank handle: ``Flock(n, params, seed).step(dt, steps)``."""
 
     def __init__(self, n: int, params=None, seed: int = 1, *, stream=None, kernel: int | None = None,
-                 record_steering: bool = False, cluster: int = 0, profile: bool = False):
+                 record_steering: bool = False, cluster: int = 0, profile: bool = False,
+                 symmetric: bool | None = None):
         self.params = params or boids_default_params()
         self.h = abi.boids_create(n, self.params, seed)
         abi.boids_set_stream(self.h, stream if stream is not None else _torch_stream())
@@ -44,6 +45,8 @@ class Flock:
             abi.boids_set_option(self.h, abi.BOIDS_OPT_CLUSTER, cluster)
         if profile:
             abi.boids_set_option(self.h, abi.BOIDS_OPT_PROFILE, 1)
+        if symmetric is not None:
+            abi.boids_set_option(self.h, abi.BOIDS_OPT_SYMMETRIC, int(symmetric))
         self.n = n
 
     def step(self, dt: float, steps: int = 1):

@@ -67,6 +67,11 @@ struct boids_ctx {
   int32_t* nbr8 = nullptr;              // 8th nearest of the last step or -1 [m]
   unsigned long long* partial = nullptr;  // warm path partial lists [m][PSLOTS][7]
   float* qlim = nullptr;                  // warm path search limits [m]
+  float4* sym_sp = nullptr;               // k_sym: agents in spatial order (x, y, z, limit) [sym_capacity]
+  int32_t* sym_idx = nullptr;             // k_sym: their local indices [sym_capacity]
+  int32_t* sym_rlist = nullptr;           // k_sym: agents routed to k_route this step [m]
+  int32_t* sym_rcount = nullptr;          // ... and their number
+  bool symmetric = true;                  // BOIDS_OPT_SYMMETRIC
   int32_t* pcnt = nullptr;
   unsigned long long* phase = nullptr;  // diagnostics (BOIDS_OPT_PHASES): per-CTA timestamps
   // grid mode (BOIDS_GRID): search grid and its binning buffers
@@ -174,6 +179,10 @@ void free_ctx(boids_ctx* c) {
   cudaFree(c->twarm);
   cudaFree(c->tcnt);
   cudaFree(c->phase);
+  cudaFree(c->sym_sp);
+  cudaFree(c->sym_idx);
+  cudaFree(c->sym_rlist);
+  cudaFree(c->sym_rcount);
   for (auto& r : c->recs) {
     cudaEventDestroy(r.a);
     cudaEventDestroy(r.b);
@@ -288,7 +297,11 @@ int create_impl(int64_t n, const boids_params* p, uint64_t seed, int32_t rank, i
              (rc = alloc((void**)&c->hitcnt, m * sizeof(int32_t))) ||
              (rc = alloc((void**)&c->partial, (size_t)m * PSLOTS * 7 * sizeof(unsigned long long))) ||
              (rc = alloc((void**)&c->pcnt, m * sizeof(int32_t))) ||
-             (rc = alloc((void**)&c->qlim, m * sizeof(float)))) {
+             (rc = alloc((void**)&c->qlim, m * sizeof(float))) ||
+             (!shard && ((rc = alloc((void**)&c->sym_sp, sym_capacity(c->nloc) * sizeof(float4))) ||
+                         (rc = alloc((void**)&c->sym_idx, sym_capacity(c->nloc) * sizeof(int32_t))) ||
+                         (rc = alloc((void**)&c->sym_rlist, m * sizeof(int32_t))) ||
+                         (rc = alloc((void**)&c->sym_rcount, sizeof(int32_t)))))) {
     free_ctx(c);
     return rc;
   }
@@ -446,9 +459,22 @@ int one_step(boids_ctx* c, float dt) {
       if ((rc = launch(c, 0, [&] { return launch_warm_scan(aw, c->stream); }, 2))) return rc;
       if ((rc = launch(c, 1, [&] { return launch_warm_select(a, c->stream); }))) return rc;
     } else if (warm_path) {
-      // warm step: all-pairs scan appending passing keys, then select + update
-      if ((rc = launch(c, 0, [&] { return launch_warm_scan(a, c->stream); }, 2))) return rc;
-      if ((rc = launch(c, 1, [&] { return launch_warm_select(a, c->stream); }))) return rc;
+      // warm step: all-pairs scan appending passing keys, then select + update;
+      // a single-GPU handle evaluates each unordered pair once (k_sym)
+      // (below 8192 agents the step is latency-bound and the ordered-pair path,
+      // with one launch less, is faster: measured C1/C2 55 vs 68 us)
+      if (c->symmetric && c->sym_sp && c->nloc >= 8192) {
+        StepArgs as = a;
+        as.routed = c->routed;  // agents searched whole by k_route (k_select skips them)
+        if ((rc = launch(c, 0, [&] {
+               return launch_sym_scan(as, c->sym_sp, c->sym_idx, c->sym_rlist, c->sym_rcount, c->stream);
+             }, 3)))
+          return rc;
+        if ((rc = launch(c, 1, [&] { return launch_warm_select(as, c->stream); }))) return rc;
+      } else {
+        if ((rc = launch(c, 0, [&] { return launch_warm_scan(a, c->stream); }, 2))) return rc;
+        if ((rc = launch(c, 1, [&] { return launch_warm_select(a, c->stream); }))) return rc;
+      }
     } else {
       // cold step (no previous lists) or forced: the cluster kernel
       int cl = c->cluster_opt;
@@ -532,6 +558,9 @@ BOIDS_API int boids_set_option(boids_ctx* c, int32_t opt, int64_t v) {
       return BOIDS_OK;
     case BOIDS_OPT_PROFILE:
       c->profile = v != 0;
+      return BOIDS_OK;
+    case BOIDS_OPT_SYMMETRIC:
+      c->symmetric = v != 0;
       return BOIDS_OK;
     case BOIDS_OPT_VOTE_U:
       if (v != 4 && v != 8) return fail(BOIDS_EINVAL, "vote width must be 4 or 8");

@@ -148,6 +148,8 @@ cudaError_t launch_warm_scan(const StepArgs& a, cudaStream_t s);
 cudaError_t launch_grid(const StepArgs& a, const GridArgs& g, cudaStream_t s);
 int grid_chunk();
 cudaError_t launch_warm_select(const StepArgs& a, cudaStream_t s);
+int64_t sym_capacity(int64_t nloc);
+cudaError_t launch_sym_scan(const StepArgs& a, float4* sp, int* sidx, int* rlist, int* rcount, cudaStream_t s);
 int fused_auto_cluster(int64_t n_pad_total, int64_t nloc, int sm_count);
 
 }  // namespace boids

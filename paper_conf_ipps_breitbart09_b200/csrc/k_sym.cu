@@ -1,0 +1,510 @@
+// k_sym.cu -- the warm-step all-pairs hit scan evaluating every UNORDERED pair once
+// (single-GPU handles; DESIGN.md sec 5 "k_sym").
+//
+// The distance is symmetric bit for bit: fl(a - b) = -fl(b - a) under round to
+// nearest even, so d2(i, j) = ((dx*dx) + (dy*dy)) + (dz*dz) is the same float
+// whichever agent is the query (the oracle pins this invariant).  A pair (i, j)
+// evaluated once can therefore be tested against BOTH agents' warm limits: it
+// is appended to i's hit buffer if d2 <= lim_i and to j's if d2 <= lim_j.  The
+// hit set of every agent is exactly the one k_scan builds ({j != i : d2(i, j) <=
+// lim_i}), so k_select (unchanged) returns the identical lists; the search
+// evaluates n(n-1)/2 distances instead of n(n-1) and is still brute force in the
+// thesis's sense (every pair is tested, Listing 5.2).
+//
+// Layout.  k_sym_prep writes the agents in spatial (Morton) order: sp[p] = (x, y,
+// z, lim) of agent sidx[p], with lim = min(prev(r2), t0) the inclusive warm limit
+// (the thread's own limit for its queries and the candidate's limit for the
+// reverse test both come from the same array; phantoms p >= n have NaN positions
+// and lim = -1).  Query block b holds sorted positions [b*QB, (b+1)*QB); its item
+// space is the candidates [b*QB, npad):
+//   * diagonal tiles [b*QB, (b+1)*QB): every ordered pair inside the block is
+//     evaluated from the query side only (self excluded by sorted position), as
+//     in k_scan -- the block's pairs are not split by a triangle mask;
+//   * off-diagonal tiles [(b+1)*QB, npad): both sides are tested.
+// Stream-K: the triangular item space sum_b (npad - b*QB) is cut into equal
+// contiguous ranges per CTA, as in k_scan.  Candidates and their original
+// indices stream through a TMA ring (cp.async.bulk + mbarrier).
+#include "step_common.cuh"
+#include "tma.cuh"
+
+#include <cstdlib>
+
+namespace boids {
+namespace {
+
+constexpr int Q = 4;        // queries per thread
+constexpr int CT = 128;     // candidates per tile
+#ifndef BOIDS_SYM_STAGES
+#define BOIDS_SYM_STAGES 24
+#endif
+// TMA ring depth.  Deep on purpose: with queries AND candidates in spatial order,
+// the slow path (passing pairs) of a tile concentrates in the 1-2 warps whose
+// queries lie next to it -- on the diagonal, tile k is hot for warp k -- and a
+// shallow ring couples every warp to the slowest one tile by tile (measured:
+// 27% of stall samples spinning on the full barrier with 4 stages).  With a deep
+// ring a warp can run STAGES-1 tiles ahead, so each warp's hot tiles only cost
+// that warp.
+constexpr int STAGES = BOIDS_SYM_STAGES;
+constexpr int U = 4;        // candidates per warp vote
+constexpr int WB = Q * U * 32;  // records per warp buffer: one vote group's maximum per side
+
+struct __align__(8) Rec {
+  int qi;  // local agent whose buffer receives the key
+  int pad;
+  key_t key;
+};
+
+template <int NT>
+struct __align__(16) SymSmem {
+  float4 ring[STAGES][CT];
+  int ridx[STAGES][CT];
+  Rec rec[NT / 32][WB];
+  uint64_t full[STAGES];
+  int rel[STAGES];  // warps done with the tile in the stage (the last one refills it)
+};
+
+// 8 records per lane per round: the atomics' round trips overlap.
+__device__ __forceinline__ void flush(const StepArgs& a, const Rec* rec, int n, int lane) {
+  for (int i0 = 0; i0 < n; i0 += 32 * 8) {
+    Rec r[8];
+    int slot[8];
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      const int i = i0 + k * 32 + lane;
+      r[k] = i < n ? rec[i] : Rec{-1, 0, 0ull};
+    }
+#pragma unroll
+    for (int k = 0; k < 8; ++k) slot[k] = r[k].qi >= 0 ? atomicAdd(a.hitcnt + r[k].qi, 1) : a.hits_cap;
+#pragma unroll
+    for (int k = 0; k < 8; ++k)
+      if (slot[k] < a.hits_cap) a.hits[(int64_t)r[k].qi * a.hits_cap + slot[k]] = r[k].key;
+  }
+}
+
+// Items before query block b: S(b) = sum_{b' < b} (npad - b'*QB).
+__device__ __forceinline__ int64_t sym_prefix(int64_t b, int64_t npad, int64_t qb) {
+  return b * npad - qb * (b * (b - 1) / 2);
+}
+
+// Append the passing keys of one vote group (bits over q*U+u) to the warp buffer.
+// `side` 0: query side (buffer of the query, key index = candidate), 1: candidate side.
+template <int SIDE>
+__device__ __forceinline__ void emit(const StepArgs& a, Rec* rec, int& wcount, int lane, unsigned bits,
+                                     const float (&d)[Q][U], const int (&gq)[Q], const int* cidx) {
+  const int nrec = __popc(bits);
+  int incl = nrec;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const int y = __shfl_up_sync(0xffffffffu, incl, o);
+    if (lane >= o) incl += y;
+  }
+  const int total = __shfl_sync(0xffffffffu, incl, 31);
+  if (total == 0) return;
+  if (wcount + total > WB) {  // warp-uniform; total <= WB always
+    __syncwarp();
+    flush(a, rec, wcount, lane);
+    __syncwarp();
+    wcount = 0;
+  }
+  int off = wcount + incl - nrec;
+#pragma unroll
+  for (int q = 0; q < Q; ++q)
+#pragma unroll
+    for (int u = 0; u < U; ++u)
+      if (bits & (1u << (q * U + u))) {
+        if (SIDE == 0) {
+          rec[off].qi = gq[q];
+          rec[off].key = make_key(d[q][u], cidx[u]);
+        } else {
+          rec[off].qi = cidx[u];
+          rec[off].key = make_key(d[q][u], gq[q]);
+        }
+        ++off;
+      }
+  wcount += total;
+}
+
+// Tile k of a CTA whose item range is [L0, L1): items [max(L0, A + k*CT), min(L1,
+// A + (k+1)*CT)) with A = L0 rounded down to CT.  Rows (npad - b*QB items) and
+// their starts S(b) are multiples of CT, so a tile never straddles two rows.
+struct TileDesc {
+  int64_t b;   // query block (row)
+  int64_t jb;  // first candidate (sorted position)
+  int cnt;     // candidates (multiple of U)
+};
+__device__ __forceinline__ TileDesc tile_desc(int k, int64_t L0, int64_t L1, int64_t npad, int64_t qb) {
+  const int64_t A = L0 / CT * CT;
+  const int64_t Ls = max(L0, A + (int64_t)k * CT), Le = min(L1, A + (int64_t)(k + 1) * CT);
+  // row: largest b with S(b) <= Ls; S is increasing and concave -> solve, then fix up
+  const double nb2 = (double)npad / (double)qb + 0.5;
+  int64_t b = (int64_t)(nb2 - sqrt(fmax(0.0, nb2 * nb2 - 2.0 * (double)Ls / (double)qb)));
+  b = b < 0 ? 0 : b;
+  while (b > 0 && sym_prefix(b, npad, qb) > Ls) --b;
+  while (sym_prefix(b + 1, npad, qb) <= Ls) ++b;
+  return TileDesc{b, b * qb + (Ls - sym_prefix(b, npad, qb)), (int)(Le - Ls)};
+}
+
+template <int NTS>
+__global__ void __launch_bounds__(NTS, NTS == 128 ? 4 : 1)
+    k_sym(StepArgs a, const float4* __restrict__ sp, const int* __restrict__ sidx, int64_t npad, int64_t items) {
+  constexpr int QBS = NTS * Q, NW = NTS / 32;
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  SymSmem<NTS>& sm = *reinterpret_cast<SymSmem<NTS>*>(smem_raw);
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const int64_t L0 = items * blockIdx.x / gridDim.x / U * U, L1 = items * (blockIdx.x + 1) / gridDim.x / U * U;
+  const int ntiles = L1 > L0 ? (int)((L1 + CT - 1) / CT - L0 / CT) : 0;
+  // Ring protocol: stage s = k % STAGES holds tile k.  full[s] completes when the
+  // tile's bytes land (TMA complete_tx).  Each warp, when done with tile k,
+  // increments rel[s]; the LAST of the NW warps refills the stage with tile
+  // k + STAGES.  So the refill waits only for the slowest warp on that tile and
+  // no warp is the dedicated producer: warps drift up to STAGES - 1 tiles apart.
+  auto issue = [&](int k) {
+    const TileDesc d = tile_desc(k, L0, L1, npad, QBS);
+    const int s = k % STAGES;
+    const uint32_t n = (uint32_t)d.cnt;
+    mbar_arrive_expect_tx(&sm.full[s], n * 20u);
+    tma_load_1d(sm.ring[s], sp + d.jb, n * 16u, &sm.full[s]);
+    tma_load_1d(sm.ridx[s], sidx + d.jb, n * 4u, &sm.full[s]);
+  };
+  if (tid == 0) {
+    if (a.phase) {  // diagnostics: [0] start, [1] end (%globaltimer), [2] L0, [3] L1, [4] slow groups
+      unsigned long long t;
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+      a.phase[blockIdx.x * 8 + 0] = t;
+      a.phase[blockIdx.x * 8 + 2] = (unsigned long long)L0;
+      a.phase[blockIdx.x * 8 + 3] = (unsigned long long)L1;
+      a.phase[blockIdx.x * 8 + 4] = 0;
+      a.phase[blockIdx.x * 8 + 5] = 0;
+      a.phase[blockIdx.x * 8 + 6] = 0;
+    }
+#pragma unroll
+    for (int s = 0; s < STAGES; ++s) {
+      mbar_init(&sm.full[s], 1);
+      sm.rel[s] = 0;
+    }
+    mbar_fence_init();
+    for (int k = 0; k < STAGES && k < ntiles; ++k) issue(k);
+  }
+  __syncthreads();
+  Rec* rec = sm.rec[warp];
+  int wcount = 0;
+  unsigned slow_groups = 0, groups = 0;
+  long long t_wait = 0, t_slow = 0;  // diagnostics (a.phase): cycles in full-barrier waits / emits
+  int64_t cur_b = -1;
+  float2 pxy[Q];
+  float pz[Q], lim[Q], limq = 0.f;
+  int gq[Q], qpos[Q];
+  for (int k = 0; k < ntiles; ++k) {
+    const TileDesc td = tile_desc(k, L0, L1, npad, QBS);
+    if (td.b != cur_b) {  // this warp's 4 x 32 queries of row b (spatially compact)
+      cur_b = td.b;
+#pragma unroll
+      for (int q = 0; q < Q; ++q) {
+        const int p = (int)(cur_b * QBS + warp * 32 * Q + q * 32 + lane);
+        const float4 me = __ldg(sp + p);
+        qpos[q] = p;
+        gq[q] = __ldg(sidx + p);
+        pxy[q] = make_float2(me.x, me.y);
+        pz[q] = me.z;
+        lim[q] = me.w;
+      }
+      limq = fmaxf(fmaxf(lim[0], lim[1]), fmaxf(lim[2], lim[3]));
+    }
+    const int s = k % STAGES;
+    long long tw0 = 0;
+    if (a.phase) tw0 = clock64();
+    mbar_wait(&sm.full[s], (uint32_t)(k / STAGES) & 1u);
+    if (a.phase) t_wait += clock64() - tw0;
+    {
+      const float4* tile = sm.ring[s];
+      const int* tidx = sm.ridx[s];
+      const int jb = (int)td.jb, cnt = td.cnt;
+      const bool diag = td.jb < (cur_b + 1) * QBS;  // candidates of the query block itself
+      auto group = [&](const int c, auto diag_c) {
+        constexpr bool DIAG = decltype(diag_c)::value;
+        float4 cc[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) cc[u] = tile[c + u];
+        float d[Q][U];
+#pragma unroll
+        for (int u = 0; u < U; ++u)
+#pragma unroll
+          for (int q = 0; q < Q; ++q) {
+            const float2 dxy = __fadd2_rn(pxy[q], make_float2(-cc[u].x, -cc[u].y));
+            const float2 sq = __fmul2_rn(dxy, dxy);
+            const float dz = __fsub_rn(pz[q], cc[u].z);
+            d[q][u] = __fadd_rn(__fadd_rn(sq.x, sq.y), __fmul_rn(dz, dz));
+          }
+        float mq[Q];
+#pragma unroll
+        for (int q = 0; q < Q; ++q) {
+          mq[q] = d[q][0];
+#pragma unroll
+          for (int u = 1; u < U; ++u) mq[q] = fminf(mq[q], d[q][u]);
+        }
+        const float m = fminf(fminf(mq[0], mq[1]), fminf(mq[2], mq[3]));  // NaN (phantoms) ignored
+        const float thr = DIAG ? limq : fmaxf(fmaxf(limq, fmaxf(cc[0].w, cc[1].w)), fmaxf(cc[2].w, cc[3].w));
+        ++groups;
+        if (__any_sync(0xffffffffu, m <= thr)) {  // rare, warp-uniform
+          ++slow_groups;
+          int cidx[U];
+#pragma unroll
+          for (int u = 0; u < U; ++u) cidx[u] = tidx[c + u];
+          unsigned qb = 0, cb = 0;
+#pragma unroll
+          for (int q = 0; q < Q; ++q)
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+              if (d[q][u] <= lim[q] && (!DIAG || jb + c + u != qpos[q])) qb |= 1u << (q * U + u);
+              if (!DIAG && d[q][u] <= cc[u].w) cb |= 1u << (q * U + u);
+            }
+          long long ts0 = 0;
+          if (a.phase) ts0 = clock64();
+          emit<0>(a, rec, wcount, lane, qb, d, gq, cidx);
+          if (!DIAG) emit<1>(a, rec, wcount, lane, cb, d, gq, cidx);
+          if (a.phase) t_slow += clock64() - ts0;
+        }
+      };
+      if (!diag && cnt == CT) {  // full off-diagonal tile: constant trip count (the common case)
+#pragma unroll 2
+        for (int c = 0; c < CT; c += U) group(c, std::false_type{});
+      } else if (!diag) {
+        for (int c = 0; c < cnt; c += U) group(c, std::false_type{});
+      } else {
+        for (int c = 0; c < cnt; c += U) group(c, std::true_type{});
+      }
+    }
+    __syncwarp();
+    if (lane == 0) {  // release stage s; the last warp refills it with tile k + STAGES
+      __threadfence_block();
+      const int old = atomicAdd(&sm.rel[s], 1);
+      if (old == NW - 1) {
+        sm.rel[s] = 0;
+        __threadfence_block();
+        if (k + STAGES < ntiles) {
+          fence_proxy_async_smem();
+          issue(k + STAGES);
+        }
+      }
+    }
+  }
+  __syncwarp();
+  flush(a, rec, wcount, lane);
+  if (a.stats && lane == 0) {
+    atomicAdd(a.stats, (unsigned long long)slow_groups);
+    atomicAdd(a.stats + 1, (unsigned long long)groups);
+  }
+  if (a.phase) {
+    if (lane == 0) {
+      atomicAdd(a.phase + blockIdx.x * 8 + 4, (unsigned long long)slow_groups);
+      atomicMax(a.phase + blockIdx.x * 8 + 5, (unsigned long long)t_wait);  // [5] max wait cycles of a warp
+      atomicMax(a.phase + blockIdx.x * 8 + 6, (unsigned long long)t_slow);  // [6] max emit cycles of a warp
+      if (warp == 0) a.phase[blockIdx.x * 8 + 7] = (unsigned long long)t_wait;  // [7] warp 0 wait
+    }
+    __syncthreads();
+    if (tid == 0) {
+      unsigned long long t;
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+      a.phase[blockIdx.x * 8 + 1] = t;
+    }
+  }
+}
+
+// t0 of local agent qi (see k_warm.cu warm_t0): 7th smallest current d2 to the
+// previous 7 neighbours and the previous 8th nearest; +inf without 7.
+__device__ __forceinline__ float sym_t0(const StepArgs& a, int64_t qi, float4 me, int& c) {
+  int nb[8];
+#pragma unroll
+  for (int k = 0; k < 7; ++k) nb[k] = __ldg(a.nbr + qi * 7 + k);
+  nb[7] = __ldg(a.nbr8 + qi);
+  c = __ldg(a.cnt + qi);
+  float4 p[8];
+#pragma unroll
+  for (int k = 0; k < 8; ++k) p[k] = __ldg(pos_of(a.full, a.m, a.sdiv, nb[k] < 0 ? 0 : nb[k]));
+  float m1 = 0.f, m2 = 0.f;
+#pragma unroll
+  for (int k = 0; k < 8; ++k) {
+    const float d = (k < 7 || nb[7] >= 0) ? dist2(me.x, me.y, me.z, p[k]) : 0.f;
+    m2 = fmaxf(m2, fminf(m1, d));
+    m1 = fmaxf(m1, d);
+  }
+  if (c < 7) return __int_as_float(0x7f800000);
+  return nb[7] >= 0 ? m2 : m1;
+}
+
+// sp[p] = (x, y, z, min(prev(r2), t0)) of agent sidx[p] = qperm[p]; phantoms beyond nloc.
+// An agent whose previous 7 neighbours are all out of range now (t0 >= r2 with a
+// full previous list: it wrapped to the far side of the world) would append
+// every in-radius pair -- hundreds -- to its hit buffer.  It is ROUTED instead:
+// limit -1 (no hits on either side in k_sym) and searched whole by k_route.
+__global__ void __launch_bounds__(256) k_sym_prep(StepArgs a, float4* __restrict__ sp, int* __restrict__ sidx,
+                                                   int64_t npad, int* __restrict__ rlist, int* __restrict__ rcount) {
+  const int64_t p = (int64_t)blockIdx.x * 256 + threadIdx.x;
+  if (p >= npad) return;
+  if (p >= a.nloc) {
+    sp[p] = make_float4(__int_as_float(0x7fc00000), __int_as_float(0x7fc00000), __int_as_float(0x7fc00000), -1.f);
+    sidx[p] = -1;
+    return;
+  }
+  const int qi = a.qperm ? __ldg(a.qperm + p) : (int)p;
+  const float r2 = __fmul_rn(a.p.search_radius, a.p.search_radius);
+  const float r2_in = __uint_as_float(__float_as_uint(r2) - 1u);  // d2 < r2  <=>  d2 <= r2_in
+  const float4 me = __ldg(pos_of(a.full, a.m, a.sdiv, a.lo + qi));
+  int c = 0;
+  const float t0 = sym_t0(a, qi, me, c);
+  float lim = fminf(r2_in, t0);
+  if (c == 7 && t0 > r2_in && rlist) {
+    rlist[atomicAdd(rcount, 1)] = qi;
+    a.routed[qi] = 1;
+    lim = -1.f;
+  }
+  sp[p] = make_float4(me.x, me.y, me.z, lim);
+  sidx[p] = qi;
+}
+
+// A := the 8 smallest keys of A u B, ascending (half-cleaner + 8-wide bitonic merge).
+__device__ __forceinline__ void merge8(key_t (&A)[8], const key_t (&B)[8]) {
+  key_t S[8];
+#pragma unroll
+  for (int s = 0; s < 8; ++s) S[s] = A[s] < B[7 - s] ? A[s] : B[7 - s];
+#pragma unroll
+  for (int i = 0; i < 4; ++i) cex(S[i], S[i + 4]);
+  cex(S[0], S[2]); cex(S[1], S[3]); cex(S[4], S[6]); cex(S[5], S[7]);
+  cex(S[0], S[1]); cex(S[2], S[3]); cex(S[4], S[5]); cex(S[6], S[7]);
+#pragma unroll
+  for (int s = 0; s < 8; ++s) A[s] = S[s];
+}
+__device__ __forceinline__ void insert8(key_t (&L)[8], key_t k) {
+#pragma unroll
+  for (int s = 7; s >= 1; --s) {
+    const key_t x = L[s - 1];
+    const key_t y = L[s] < k ? L[s] : k;
+    L[s] = k < x ? x : y;
+  }
+  L[0] = L[0] < k ? L[0] : k;
+}
+
+// Routed agents (k_sym_prep): one CTA per agent searches all candidates (Listing
+// 5.2: every agent, index order irrelevant under the (d2, index) key), keeping the
+// 8 smallest keys per thread; a shuffle butterfly and a shared-memory pass merge
+// them.  The CTA then finishes the agent -- list, 8th nearest (the next step's
+// warm-bound seed), steering, modification -- and k_select skips it.
+constexpr int RT = 512;
+__global__ void __launch_bounds__(RT) k_route(StepArgs a, const int* __restrict__ rlist,
+                                              const int* __restrict__ rcount) {
+  __shared__ key_t wl[RT / 32][8];
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int nr = *rcount;
+  const float r2 = __fmul_rn(a.p.search_radius, a.p.search_radius);
+  const int64_t total = (int64_t)a.world * a.m;  // candidate slots (phantoms are NaN)
+  for (int r = blockIdx.x; r < nr; r += gridDim.x) {
+    const int qi = __ldg(rlist + r);
+    const float4 me = __ldg(pos_of(a.full, a.m, a.sdiv, a.lo + qi));
+    const int g = (int)(a.lo + qi);
+    key_t A[8];
+#pragma unroll
+    for (int s = 0; s < 8; ++s) A[s] = KEY_EMPTY;
+    for (int64_t j0 = tid; j0 < total; j0 += RT * 4) {
+      float4 c[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const int64_t j = j0 + (int64_t)RT * u;
+        c[u] = j < total ? __ldg(pos_of(a.full, a.m, a.sdiv, j)) : make_float4(__int_as_float(0x7fc00000), 0.f, 0.f, 0.f);
+      }
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const float d2 = dist2(me.x, me.y, me.z, c[u]);
+        const int j = (int)(j0 + (int64_t)RT * u);
+        if (d2 < r2 && j != g) {
+          const key_t k = make_key(d2, j);
+          if (k < A[7]) insert8(A, k);
+        }
+      }
+    }
+#pragma unroll
+    for (int w = 1; w < 32; w <<= 1) {
+      key_t B[8];
+#pragma unroll
+      for (int s = 0; s < 8; ++s) B[s] = __shfl_xor_sync(0xffffffffu, A[s], w);
+      merge8(A, B);
+    }
+    if (lane == 0)
+#pragma unroll
+      for (int s = 0; s < 8; ++s) wl[warp][s] = A[s];
+    __syncthreads();
+    if (tid == 0) {
+      for (int w = 1; w < RT / 32; ++w) {
+        key_t B[8];
+#pragma unroll
+        for (int s = 0; s < 8; ++s) B[s] = wl[w][s];
+        merge8(A, B);
+      }
+      key_t L7[7];
+#pragma unroll
+      for (int s = 0; s < 7; ++s) L7[s] = A[s];
+      a.nbr8[qi] = A[7] == KEY_EMPTY ? -1 : key_idx(A[7]);
+      finish_agent(a, qi, L7);
+    }
+    __syncthreads();
+  }
+}
+
+template <int NT>
+int sym_grid(int sms) {
+  static int grid = 0;
+  if (!grid) {
+    int r = 0;
+    cudaFuncSetAttribute(k_sym<NT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(SymSmem<NT>));
+    cudaFuncSetAttribute(k_sym<NT>, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&r, k_sym<NT>, NT, sizeof(SymSmem<NT>));
+    grid = sms * (r > 0 ? r : 1);
+  }
+  return grid;
+}
+
+template <int NT>
+cudaError_t sym_with(const StepArgs& a, float4* sp, int* sidx, int* rlist, int* rcount, int sms, cudaStream_t s) {
+  constexpr int64_t QBS = NT * Q;
+  const int64_t npad = (a.nloc + QBS - 1) / QBS * QBS;
+  if (rlist) {
+    if (cudaError_t e = cudaMemsetAsync(rcount, 0, sizeof(int), s)) return e;
+  }
+  k_sym_prep<<<(unsigned)((npad + 255) / 256), 256, 0, s>>>(a, sp, sidx, npad, rlist, rcount);
+  if (cudaError_t e = cudaGetLastError()) return e;
+  const int64_t nb = npad / QBS;
+  const int64_t items = nb * npad - QBS * (nb * (nb - 1) / 2);
+  const int g = (int)std::min<int64_t>(sym_grid<NT>(sms), (items + CT - 1) / CT);
+  k_sym<NT><<<g, NT, sizeof(SymSmem<NT>), s>>>(a, sp, sidx, npad, items);
+  if (cudaError_t e = cudaGetLastError()) return e;
+  if (rlist) {
+    k_route<<<(unsigned)std::min<int64_t>(a.nloc, 2LL * sms), RT, 0, s>>>(a, rlist, rcount);
+    return cudaGetLastError();
+  }
+  return cudaSuccess;
+}
+
+}  // namespace
+
+int64_t sym_capacity(int64_t nloc) { return (nloc + 2047) / 2048 * 2048; }
+
+// Launches: (memset of the routed count) k_sym_prep (spatial order + limits,
+// routing), k_sym, and k_route when rlist is given (a.routed must then be set).  Requires the
+// handle's previous lists (warm step), qperm = the spatial order of the owned
+// agents, world == 1, and think_every == 1.
+cudaError_t launch_sym_scan(const StepArgs& a, float4* sp, int* sidx, int* rlist, int* rcount, cudaStream_t s) {
+  if (a.nloc <= 0) return cudaSuccess;
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  // one 512-thread CTA per SM when every SM gets >= 2 tiles of (2048 queries x CT)
+  const int64_t nb = (a.nloc + 2047) / 2048, np = nb * 2048;
+  const int64_t tiles512 = (nb * np - 2048 * (nb * (nb - 1) / 2)) / CT;
+  static const int force = [] {
+    const char* e = getenv("BOIDS_SYM_NT");  // diagnostics: force a CTA shape (128 or 512)
+    return e ? atoi(e) : 0;
+  }();
+  if (force == 512 || (force != 128 && tiles512 >= 2LL * sms)) return sym_with<512>(a, sp, sidx, rlist, rcount, sms, s);
+  return sym_with<128>(a, sp, sidx, rlist, rcount, sms, s);
+}
+
+}  // namespace boids

@@ -455,6 +455,7 @@ __global__ void __launch_bounds__(NSEL) k_select(StepArgs a) {
   const float4 f4 = __ldg(fwd_of(a.full, a.m, a.sdiv, a.lo + qi));
   if (!active) {  // think mode, not searched by k_scan this step
     if (routed) a.routed[qi] = 0;
+    if (routed && a.think_k <= 1) return;  // k_sym step: k_route finished this agent
     const float4 F = a.fstore[qi];
     modify_agent(a, qi, v3(p4), f4, v3(F));
     return;

@@ -37,7 +37,7 @@ __device__ __forceinline__ float warm_bound(const StepArgs& a, int64_t qi, float
 // Insert key k into a sorted 7-list in shared memory (stride between entries);
 // returns the new worst d2 (+inf while fewer than 7 are held).  Out of line: it
 // runs rarely and one copy keeps the hot loops small in the instruction cache.
-__device__ __noinline__ float insert_smem7(key_t* L7, int stride, key_t k) {
+static __device__ __noinline__ float insert_smem7(key_t* L7, int stride, key_t k) {
   key_t L[7];
 #pragma unroll
   for (int s = 0; s < 7; ++s) L[s] = L7[s * stride];

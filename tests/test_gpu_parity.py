@@ -120,12 +120,18 @@ def test_wrap_agents_outside(pk, orc):
 
 
 # -------------------------------------------------- trajectories (warm path)
-@pytest.mark.parametrize("kernel,n,steps", [(0, 1024, 30), (0, 4096, 10), (1, 1024, 10), (2, 1024, 12),
-                                            (0, 20000, 3)])
-def test_trajectory_from_init(pk, orc, kernel, n, steps):
+@pytest.mark.parametrize("kernel,n,steps,sym", [(0, 1024, 30, 1), (0, 4096, 10, 1), (1, 1024, 10, 1),
+                                                (2, 1024, 12, 1), (0, 20000, 3, 1), (0, 1024, 12, 0),
+                                                (0, 4096, 5, 0), (0, 20000, 3, 0), (0, 1, 3, 1), (0, 2, 3, 1),
+                                                (0, 8192, 4, 1), (0, 8193, 4, 1), (0, 10239, 4, 1),
+                                                (0, 12289, 3, 1), (0, 9000, 3, 1), (0, 40000, 2, 1)])
+def test_trajectory_from_init(pk, orc, kernel, n, steps, sym):
     """GPU steps continuously (warm thresholds active after step 1); the oracle
-    runs the same steps from its own init.  Bit-exact sides stay identical."""
-    with pk.Flock(n, seed=1, kernel=kernel) as f:
+    runs the same steps from its own init.  Bit-exact sides stay identical.
+    sym=1: warm steps evaluate each unordered pair once (k_sym, the default for
+    n >= 8192); sym=0: every ordered pair (k_scan).  Sizes straddle the 2048-agent
+    query blocks of k_sym (ragged diagonal and off-diagonal tiles, phantoms)."""
+    with pk.Flock(n, seed=1, kernel=kernel, symmetric=bool(sym)) as f:
         o = orc.init(n, seed=1)
         for t in range(steps):
             o, o_idx, o_cnt, _ = orc.step(o, DT)
@@ -155,14 +161,15 @@ def test_set_state_keeps_exact_with_stale_lists(pk, orc, new):
         assert bitexact(f.state(), o_state) and np.array_equal(f.steering(), o_F)
 
 
-def test_trajectory_wraps_and_overflow(pk, orc):
+@pytest.mark.parametrize("sym", [1, 0])
+def test_trajectory_wraps_and_overflow(pk, orc, sym):
     """Small world, long dt: many agents wrap to the diametric opposite point each
     step, so their old neighbours end far away -> t0 >= r2 -> the warm
     scan's hit buffers overflow and k_select's warp re-search runs.  Bit-exact."""
     p = pk.boids_default_params(init_mode=1, world_radius=12.0, max_speed=30.0)
     op = _oparams(orc, p)
     n, dt = 3000, 0.05
-    with pk.Flock(n, p, seed=5) as f:
+    with pk.Flock(n, p, seed=5, symmetric=bool(sym)) as f:
         o = orc.init(n, op, seed=5)
         wrapped = 0
         for t in range(8):
@@ -219,6 +226,33 @@ def test_config_c4_sampled(pk, orc):
         assert (cnt2 <= 7).all() and (idx2[np.arange(c.n), 0] != np.arange(c.n)).all()
 
 
+@pytest.mark.parametrize("sym", [1, 0])
+def test_config_c4_warm_sampled(pk, orc, sym):
+    """C4 at full size on the WARM path (the bench's steady state): a cold step on
+    the oracle's initial state leaves neighbour lists; the input is then replaced
+    by a jittered copy (workloads.jitter, numpy only), so the next step runs the
+    warm scan (k_sym / k_scan) with stale-but-close lists as bound seeds.  A
+    seeded sample of 1024 agents is checked one by one against the oracle."""
+    c = W.CONFIGS["c4"]
+    p = pk.boids_default_params(init_mode=c.init_mode)
+    op = _oparams(orc, p)
+    ag = W.sample_agents(c.n, 1024, seed=3)
+    s0 = orc.init(c.n, op, seed=1)
+    s1 = W.jitter({k: s0[k] for k in KEYS}, 0.05, seed=4)
+    with pk.Flock(c.n, p, seed=1, record_steering=True, symmetric=bool(sym)) as f:
+        f.set_state({k: s0[k] for k in KEYS})
+        f.step(DT, 1)
+        f.set_state(s1)
+        f.step(DT, 1)
+        g = f.state()
+        g_idx, _ = f.neighbors()
+        o, o_idx, _, o_F = orc.step_sample(orc.State(s1), ag, DT, op)
+        np.testing.assert_array_equal(g_idx[ag], o_idx)
+        np.testing.assert_array_equal(f.steering()[ag], o_F)
+        for k in KEYS:
+            np.testing.assert_array_equal(g[k][ag], o[k])
+
+
 # --------------------------------------------------------------- edges
 def test_steps_zero_is_noop(pk):
     with pk.Flock(300, seed=2) as f:
@@ -249,9 +283,16 @@ def test_launch_count_and_info(pk):
         f.step(DT, 5)
         f.sync()
         info = f.info()
-        # step 1 (cold): the fused cluster kernel; steps 2-5 (warm): bound + scan + select;
-        # the spatial query order (3 binning kernels) is refreshed on step 1 and every 8th
-        assert info.launches - i0 == 1 + 4 * 3 + 3
+        # step 1 (cold): the fused cluster kernel; steps 2-5 (warm, single GPU):
+        # k_sym_prep + k_sym + k_route + k_select; the spatial query order (3
+        # binning kernels) is refreshed on step 1 and every 8th
+        assert info.launches - i0 == 1 + 4 * 4 + 3
+    with pk.Flock(16384, seed=1, symmetric=False) as f:
+        i0 = f.info().launches
+        f.step(DT, 5)
+        f.sync()
+        # warm steps on the ordered-pair path: k_bound + k_scan + k_select
+        assert f.info().launches - i0 == 1 + 4 * 3 + 3
         assert info.cluster == 16 and info.slice == 16384
 
 

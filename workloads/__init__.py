@@ -99,6 +99,17 @@ def radius_shell_flock(radius: float = 9.0, seed: int = 1) -> dict:
                 speed=(rng.random(n) * 9.0).astype(np.float32))
 
 
+def jitter(state: dict, scale: float, seed: int = 11) -> dict:
+    """Copy of a state dict with every position moved by a seeded normal offset
+    (std `scale` per axis): a new input that keeps the spatial structure, so a
+    handle stepped on the old state has neighbour lists that are stale but close
+    (the warm path's realistic case)."""
+    rng = np.random.default_rng(seed)
+    out = {k: np.array(v, dtype=np.float32, copy=True) for k, v in state.items()}
+    out["pos"] = (out["pos"] + scale * rng.standard_normal(out["pos"].shape)).astype(np.float32)
+    return out
+
+
 def sample_agents(n: int, m: int, seed: int = 7) -> np.ndarray:
     """Seeded sample of m distinct agent indices (always includes 0 and n-1)."""
     rng = np.random.default_rng(seed)
