@@ -298,10 +298,10 @@ int create_impl(int64_t n, const boids_params* p, uint64_t seed, int32_t rank, i
              (rc = alloc((void**)&c->partial, (size_t)m * PSLOTS * 7 * sizeof(unsigned long long))) ||
              (rc = alloc((void**)&c->pcnt, m * sizeof(int32_t))) ||
              (rc = alloc((void**)&c->qlim, m * sizeof(float))) ||
+             (rc = alloc((void**)&c->sym_rlist, m * sizeof(int32_t))) ||
+             (rc = alloc((void**)&c->sym_rcount, sizeof(int32_t))) ||
              (!shard && ((rc = alloc((void**)&c->sym_sp, sym_capacity(c->nloc) * sizeof(float4))) ||
-                         (rc = alloc((void**)&c->sym_idx, sym_capacity(c->nloc) * sizeof(int32_t))) ||
-                         (rc = alloc((void**)&c->sym_rlist, m * sizeof(int32_t))) ||
-                         (rc = alloc((void**)&c->sym_rcount, sizeof(int32_t)))))) {
+                         (rc = alloc((void**)&c->sym_idx, sym_capacity(c->nloc) * sizeof(int32_t)))))) {
     free_ctx(c);
     return rc;
   }
@@ -376,6 +376,8 @@ StepArgs make_args(boids_ctx* c, float dt) {
   a.qcount = nullptr;
   a.nq = c->nloc;
   a.routed = c->p.think_every > 1 ? c->routed : nullptr;
+  a.rlist = c->sym_rlist;  // warm steps route overflowed agents to k_route (nullptr in grid mode)
+  a.rcount = c->sym_rcount;
   return a;
 }
 
@@ -456,8 +458,10 @@ int one_step(boids_ctx* c, float dt) {
       StepArgs aw = a;
       aw.qperm = c->twarm;
       aw.qcount = c->tcnt + 1;
+      CK(cudaMemsetAsync(c->sym_rcount, 0, sizeof(int32_t), c->stream));
       if ((rc = launch(c, 0, [&] { return launch_warm_scan(aw, c->stream); }, 2))) return rc;
       if ((rc = launch(c, 1, [&] { return launch_warm_select(a, c->stream); }))) return rc;
+      if ((rc = launch(c, 0, [&] { return launch_route(a, c->stream); }))) return rc;
     } else if (warm_path) {
       // warm step: all-pairs scan appending passing keys, then select + update;
       // a single-GPU handle evaluates each unordered pair once (k_sym)
@@ -465,15 +469,17 @@ int one_step(boids_ctx* c, float dt) {
       // with one launch less, is faster: measured C1/C2 55 vs 68 us)
       if (c->symmetric && c->sym_sp && c->nloc >= 8192) {
         StepArgs as = a;
-        as.routed = c->routed;  // agents searched whole by k_route (k_select skips them)
-        if ((rc = launch(c, 0, [&] {
-               return launch_sym_scan(as, c->sym_sp, c->sym_idx, c->sym_rlist, c->sym_rcount, c->stream);
-             }, 3)))
+        as.routed = c->routed;  // agents routed to k_route by k_sym_prep (k_select skips them)
+        CK(cudaMemsetAsync(c->sym_rcount, 0, sizeof(int32_t), c->stream));
+        if ((rc = launch(c, 0, [&] { return launch_sym_scan(as, c->sym_sp, c->sym_idx, c->stream); }, 2)))
           return rc;
         if ((rc = launch(c, 1, [&] { return launch_warm_select(as, c->stream); }))) return rc;
+        if ((rc = launch(c, 0, [&] { return launch_route(as, c->stream); }))) return rc;
       } else {
+        CK(cudaMemsetAsync(c->sym_rcount, 0, sizeof(int32_t), c->stream));
         if ((rc = launch(c, 0, [&] { return launch_warm_scan(a, c->stream); }, 2))) return rc;
         if ((rc = launch(c, 1, [&] { return launch_warm_select(a, c->stream); }))) return rc;
+        if ((rc = launch(c, 0, [&] { return launch_route(a, c->stream); }))) return rc;
       }
     } else {
       // cold step (no previous lists) or forced: the cluster kernel

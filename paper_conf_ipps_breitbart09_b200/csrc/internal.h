@@ -100,7 +100,10 @@ struct StepArgs {
   float4* fstore;             // [nloc] last steering vector of each agent
   const int32_t* qcount;      // device-side number of query slots (qperm entries), nullptr = nloc
   int64_t nq;                 // kernel-local copy of the number of query slots
-  unsigned char* routed;      // [nloc] think mode: 1 = searched by k_fused this step (k_select skips)
+  unsigned char* routed;      // [nloc] think mode: 1 = searched by k_fused this step (k_select skips);
+                              // k_sym steps: 1 = routed to k_route by k_sym_prep
+  int32_t* rlist;             // warm steps: agents finished by k_route (hit-buffer overflow, routed);
+  int32_t* rcount;            // their number (zeroed before the step).  nullptr = warp re-search in k_select
   unsigned long long* phase;  // diagnostics: per-CTA %globaltimer stamps [grid][8], nullptr = off
   float dt;
   boids_params p;
@@ -149,7 +152,8 @@ cudaError_t launch_grid(const StepArgs& a, const GridArgs& g, cudaStream_t s);
 int grid_chunk();
 cudaError_t launch_warm_select(const StepArgs& a, cudaStream_t s);
 int64_t sym_capacity(int64_t nloc);
-cudaError_t launch_sym_scan(const StepArgs& a, float4* sp, int* sidx, int* rlist, int* rcount, cudaStream_t s);
+cudaError_t launch_sym_scan(const StepArgs& a, float4* sp, int* sidx, cudaStream_t s);
+cudaError_t launch_route(const StepArgs& a, cudaStream_t s);
 int fused_auto_cluster(int64_t n_pad_total, int64_t nloc, int sm_count);
 
 }  // namespace boids

@@ -91,14 +91,17 @@ __device__ __forceinline__ int64_t sym_prefix(int64_t b, int64_t npad, int64_t q
 template <int SIDE>
 __device__ __forceinline__ void emit(const StepArgs& a, Rec* rec, int& wcount, int lane, unsigned bits,
                                      const float (&d)[Q][U], const int (&gq)[Q], const int* cidx) {
+  // exclusive prefix of the per-lane record counts (0..16) from 5 independent
+  // ballots on their bits: no dependent shuffle chain on this path
   const int nrec = __popc(bits);
-  int incl = nrec;
+  const unsigned lt = (1u << lane) - 1u;
+  int excl = 0, total = 0;
 #pragma unroll
-  for (int o = 1; o < 32; o <<= 1) {
-    const int y = __shfl_up_sync(0xffffffffu, incl, o);
-    if (lane >= o) incl += y;
+  for (int k = 0; k < 5; ++k) {
+    const unsigned bk = __ballot_sync(0xffffffffu, (nrec >> k) & 1);
+    excl += __popc(bk & lt) << k;
+    total += __popc(bk) << k;
   }
-  const int total = __shfl_sync(0xffffffffu, incl, 31);
   if (total == 0) return;
   if (wcount + total > WB) {  // warp-uniform; total <= WB always
     __syncwarp();
@@ -106,7 +109,7 @@ __device__ __forceinline__ void emit(const StepArgs& a, Rec* rec, int& wcount, i
     __syncwarp();
     wcount = 0;
   }
-  int off = wcount + incl - nrec;
+  int off = wcount + excl;
 #pragma unroll
   for (int q = 0; q < Q; ++q)
 #pragma unroll
@@ -122,6 +125,27 @@ __device__ __forceinline__ void emit(const StepArgs& a, Rec* rec, int& wcount, i
         ++off;
       }
   wcount += total;
+}
+
+// Stream-K split with weights: a diagonal item (query side only, but where most
+// passing pairs -- the slow path -- are, since a query block is spatially
+// compact) costs wd4/4 of an off-diagonal one.  Row b has weighted length
+// 4*(npad - b*QB) + (wd4 - 4)*QB; CTA i gets the items of the weighted range
+// [i*W/grid, (i+1)*W/grid), rounded to multiples of U.
+__device__ __forceinline__ int64_t sym_split(int64_t i, int64_t grid, int64_t npad, int64_t qb, int wd4) {
+  const int64_t nb = npad / qb;
+  auto sw = [&](int64_t b) { return 4 * sym_prefix(b, npad, qb) + (int64_t)(wd4 - 4) * qb * b; };
+  const int64_t W = sw(nb);
+  if (i >= grid) return sym_prefix(nb, npad, qb);
+  const int64_t x = (int64_t)((__int128)W * i / grid);
+  int64_t lo = 0, hi = nb - 1;  // largest b with sw(b) <= x
+  while (lo < hi) {
+    const int64_t mid = (lo + hi + 1) / 2;
+    if (sw(mid) <= x) lo = mid; else hi = mid - 1;
+  }
+  const int64_t o = x - sw(lo), dw = (int64_t)wd4 * qb;
+  const int64_t off = o < dw ? o / wd4 : qb + (o - dw) / 4;
+  return (sym_prefix(lo, npad, qb) + off) / U * U;
 }
 
 // Tile k of a CTA whose item range is [L0, L1): items [max(L0, A + k*CT), min(L1,
@@ -146,12 +170,12 @@ __device__ __forceinline__ TileDesc tile_desc(int k, int64_t L0, int64_t L1, int
 
 template <int NTS>
 __global__ void __launch_bounds__(NTS, NTS == 128 ? 4 : 1)
-    k_sym(StepArgs a, const float4* __restrict__ sp, const int* __restrict__ sidx, int64_t npad, int64_t items) {
+    k_sym(StepArgs a, const float4* __restrict__ sp, const int* __restrict__ sidx, int64_t npad, int wd4) {
   constexpr int QBS = NTS * Q, NW = NTS / 32;
   extern __shared__ __align__(16) unsigned char smem_raw[];
   SymSmem<NTS>& sm = *reinterpret_cast<SymSmem<NTS>*>(smem_raw);
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-  const int64_t L0 = items * blockIdx.x / gridDim.x / U * U, L1 = items * (blockIdx.x + 1) / gridDim.x / U * U;
+  const int64_t L0 = sym_split(blockIdx.x, gridDim.x, npad, QBS, wd4), L1 = sym_split(blockIdx.x + 1, gridDim.x, npad, QBS, wd4);
   const int ntiles = L1 > L0 ? (int)((L1 + CT - 1) / CT - L0 / CT) : 0;
   // Ring protocol: stage s = k % STAGES holds tile k.  full[s] completes when the
   // tile's bytes land (TMA complete_tx).  Each warp, when done with tile k,
@@ -338,7 +362,7 @@ __device__ __forceinline__ float sym_t0(const StepArgs& a, int64_t qi, float4 me
 // every in-radius pair -- hundreds -- to its hit buffer.  It is ROUTED instead:
 // limit -1 (no hits on either side in k_sym) and searched whole by k_route.
 __global__ void __launch_bounds__(256) k_sym_prep(StepArgs a, float4* __restrict__ sp, int* __restrict__ sidx,
-                                                   int64_t npad, int* __restrict__ rlist, int* __restrict__ rcount) {
+                                                   int64_t npad) {
   const int64_t p = (int64_t)blockIdx.x * 256 + threadIdx.x;
   if (p >= npad) return;
   if (p >= a.nloc) {
@@ -353,8 +377,8 @@ __global__ void __launch_bounds__(256) k_sym_prep(StepArgs a, float4* __restrict
   int c = 0;
   const float t0 = sym_t0(a, qi, me, c);
   float lim = fminf(r2_in, t0);
-  if (c == 7 && t0 > r2_in && rlist) {
-    rlist[atomicAdd(rcount, 1)] = qi;
+  if (c == 7 && t0 > r2_in && a.rlist) {
+    a.rlist[atomicAdd(a.rcount, 1)] = qi;
     a.routed[qi] = 1;
     lim = -1.f;
   }
@@ -390,15 +414,14 @@ __device__ __forceinline__ void insert8(key_t (&L)[8], key_t k) {
 // them.  The CTA then finishes the agent -- list, 8th nearest (the next step's
 // warm-bound seed), steering, modification -- and k_select skips it.
 constexpr int RT = 512;
-__global__ void __launch_bounds__(RT) k_route(StepArgs a, const int* __restrict__ rlist,
-                                              const int* __restrict__ rcount) {
+__global__ void __launch_bounds__(RT) k_route(StepArgs a) {
   __shared__ key_t wl[RT / 32][8];
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  const int nr = *rcount;
+  const int nr = *a.rcount;
   const float r2 = __fmul_rn(a.p.search_radius, a.p.search_radius);
   const int64_t total = (int64_t)a.world * a.m;  // candidate slots (phantoms are NaN)
   for (int r = blockIdx.x; r < nr; r += gridDim.x) {
-    const int qi = __ldg(rlist + r);
+    const int qi = a.rlist[r];
     const float4 me = __ldg(pos_of(a.full, a.m, a.sdiv, a.lo + qi));
     const int g = (int)(a.lo + qi);
     key_t A[8];
@@ -439,11 +462,20 @@ __global__ void __launch_bounds__(RT) k_route(StepArgs a, const int* __restrict_
         for (int s = 0; s < 8; ++s) B[s] = wl[w][s];
         merge8(A, B);
       }
-      key_t L7[7];
-#pragma unroll
-      for (int s = 0; s < 7; ++s) L7[s] = A[s];
       a.nbr8[qi] = A[7] == KEY_EMPTY ? -1 : key_idx(A[7]);
-      finish_agent(a, qi, L7);
+      int nb[7], cnt = 0;
+#pragma unroll
+      for (int s = 0; s < 7; ++s) {
+        nb[s] = A[s] == KEY_EMPTY ? -1 : key_idx(A[s]);
+        cnt += A[s] == KEY_EMPTY ? 0 : 1;
+      }
+#pragma unroll
+      for (int s = 0; s < 7; ++s) a.nbr[qi * 7 + s] = nb[s];
+      a.cnt[qi] = cnt;
+      const float4 f4 = __ldg(fwd_of(a.full, a.m, a.sdiv, a.lo + qi));
+      const V3 F = steer_agent(a, v3(me), v3(f4), nb, cnt);
+      if (a.think_k > 1) a.fstore[qi] = make_float4(F.x, F.y, F.z, 0.f);  // think mode: a warm thinker
+      modify_agent(a, qi, v3(me), f4, F);
     }
     __syncthreads();
   }
@@ -463,35 +495,42 @@ int sym_grid(int sms) {
 }
 
 template <int NT>
-cudaError_t sym_with(const StepArgs& a, float4* sp, int* sidx, int* rlist, int* rcount, int sms, cudaStream_t s) {
+cudaError_t sym_with(const StepArgs& a, float4* sp, int* sidx, int sms, cudaStream_t s) {
   constexpr int64_t QBS = NT * Q;
   const int64_t npad = (a.nloc + QBS - 1) / QBS * QBS;
-  if (rlist) {
-    if (cudaError_t e = cudaMemsetAsync(rcount, 0, sizeof(int), s)) return e;
-  }
-  k_sym_prep<<<(unsigned)((npad + 255) / 256), 256, 0, s>>>(a, sp, sidx, npad, rlist, rcount);
+  k_sym_prep<<<(unsigned)((npad + 255) / 256), 256, 0, s>>>(a, sp, sidx, npad);
   if (cudaError_t e = cudaGetLastError()) return e;
   const int64_t nb = npad / QBS;
   const int64_t items = nb * npad - QBS * (nb * (nb - 1) / 2);
   const int g = (int)std::min<int64_t>(sym_grid<NT>(sms), (items + CT - 1) / CT);
-  k_sym<NT><<<g, NT, sizeof(SymSmem<NT>), s>>>(a, sp, sidx, npad, items);
-  if (cudaError_t e = cudaGetLastError()) return e;
-  if (rlist) {
-    k_route<<<(unsigned)std::min<int64_t>(a.nloc, 2LL * sms), RT, 0, s>>>(a, rlist, rcount);
-    return cudaGetLastError();
-  }
-  return cudaSuccess;
+  static const int wd4 = [] {
+    const char* e = getenv("BOIDS_SYM_WD4");  // diagnostics: diagonal item weight x4
+    return e ? atoi(e) : 6;  // measured best of 4..16 at C3 and C4
+  }();
+  k_sym<NT><<<g, NT, sizeof(SymSmem<NT>), s>>>(a, sp, sidx, npad, wd4);
+  return cudaGetLastError();
 }
 
 }  // namespace
 
 int64_t sym_capacity(int64_t nloc) { return (nloc + 2047) / 2048 * 2048; }
 
-// Launches: (memset of the routed count) k_sym_prep (spatial order + limits,
-// routing), k_sym, and k_route when rlist is given (a.routed must then be set).  Requires the
+// Launches k_sym_prep (spatial order + limits; routing into a.rlist, flagged in
+// a.routed) and k_sym.  a.rcount must be zero.  Requires the
 // handle's previous lists (warm step), qperm = the spatial order of the owned
 // agents, world == 1, and think_every == 1.
-cudaError_t launch_sym_scan(const StepArgs& a, float4* sp, int* sidx, int* rlist, int* rcount, cudaStream_t s) {
+// After k_select: agents in a.rlist (routed by k_sym_prep, or hit-buffer overflow)
+// are searched whole and finished, one CTA each (grid-stride over the device count).
+cudaError_t launch_route(const StepArgs& a, cudaStream_t s) {
+  if (a.nloc <= 0 || !a.rlist) return cudaSuccess;
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  k_route<<<(unsigned)std::min<int64_t>(a.nloc, 2LL * sms), RT, 0, s>>>(a);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_sym_scan(const StepArgs& a, float4* sp, int* sidx, cudaStream_t s) {
   if (a.nloc <= 0) return cudaSuccess;
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
@@ -503,8 +542,8 @@ cudaError_t launch_sym_scan(const StepArgs& a, float4* sp, int* sidx, int* rlist
     const char* e = getenv("BOIDS_SYM_NT");  // diagnostics: force a CTA shape (128 or 512)
     return e ? atoi(e) : 0;
   }();
-  if (force == 512 || (force != 128 && tiles512 >= 2LL * sms)) return sym_with<512>(a, sp, sidx, rlist, rcount, sms, s);
-  return sym_with<128>(a, sp, sidx, rlist, rcount, sms, s);
+  if (force == 512 || (force != 128 && tiles512 >= 2LL * sms)) return sym_with<512>(a, sp, sidx, sms, s);
+  return sym_with<128>(a, sp, sidx, sms, s);
 }
 
 }  // namespace boids

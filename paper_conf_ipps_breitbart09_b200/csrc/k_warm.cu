@@ -436,9 +436,19 @@ __global__ void __launch_bounds__(NSEL) k_select(StepArgs a) {
       if (h > A[6] && h < eighth) eighth = h;
     }
   }
-  // overflowed buffers: the warp searches those agents again, one at a time
+  // overflowed buffers: routed to k_route (one CTA per agent, after this kernel),
+  // or else the warp searches those agents again, one at a time
   unsigned om = __ballot_sync(0xffffffffu, over);
   if (a.stats && (threadIdx.x & 31) == 0 && om) atomicAdd(a.stats + 2, (unsigned long long)__popc(om));
+  if (a.rlist) {
+    if (over) {
+      a.rlist[atomicAdd(a.rcount, 1)] = (int)qi;
+      a.hitcnt[qi] = 0;
+      a.pcnt[qi] = 0;
+      return;
+    }
+    om = 0;
+  }
   while (om) {
     const int src = __ffs(om) - 1;
     om &= om - 1;

@@ -284,15 +284,15 @@ def test_launch_count_and_info(pk):
         f.sync()
         info = f.info()
         # step 1 (cold): the fused cluster kernel; steps 2-5 (warm, single GPU):
-        # k_sym_prep + k_sym + k_route + k_select; the spatial query order (3
+        # k_sym_prep + k_sym + k_select + k_route; the spatial query order (3
         # binning kernels) is refreshed on step 1 and every 8th
         assert info.launches - i0 == 1 + 4 * 4 + 3
     with pk.Flock(16384, seed=1, symmetric=False) as f:
         i0 = f.info().launches
         f.step(DT, 5)
         f.sync()
-        # warm steps on the ordered-pair path: k_bound + k_scan + k_select
-        assert f.info().launches - i0 == 1 + 4 * 3 + 3
+        # warm steps on the ordered-pair path: k_bound + k_scan + k_select + k_route
+        assert f.info().launches - i0 == 1 + 4 * 4 + 3
         assert info.cluster == 16 and info.slice == 16384
 
 
