@@ -151,7 +151,7 @@ def run_reference(args, cfg):
         "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
         "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
-    print(json.dumps(line), flush=True)
+    emit(line)
     return 0
 
 
@@ -164,7 +164,20 @@ def config_dict(cfg: W.Config, gpus: int):
             "dt": float(W.DT), "seed": 1, "l2": "flushed (256 MiB write) before every timed step"}
 
 
+_OUT = None
+
+
+def emit(line: dict):
+    """Print the one JSON line on the real stdout (fd 1 is redirected to stderr
+    during the run so library banners, e.g. NCCL's version line, cannot mix in)."""
+    os.write(_OUT, (json.dumps(line) + "\n").encode())
+
+
 def main():
+    global _OUT
+    sys.stdout.flush()
+    _OUT = os.dup(1)
+    os.dup2(2, 1)
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=10)
@@ -399,7 +412,7 @@ def main():
             "thesis_context": "thesis v5 GPU (GeForce 8800 GTS) vs CPU (Athlon 64 3700+): ~42x at 4096 agents "
                               "(PAPER.md P:499, P:465); different hardware and baseline, not comparable",
         }
-        print(json.dumps(line), flush=True)
+        emit(line)
     fl.close()
     if dist is not None:
         dist.destroy_process_group()

@@ -92,7 +92,9 @@ typedef struct boids_info_t {
   int64_t slow_groups; /* fused kernel, cumulative: vote groups (U candidates x Q queries x 32
                           lanes) that took the insertion path ... */
   int64_t vote_groups; /* ... out of this many (diagnostics; boids_info synchronises) */
-  int64_t fallbacks;   /* warm path, cumulative: agents re-searched after a hit-buffer overflow */
+  int64_t fallbacks;   /* warm path, cumulative: agents searched whole (k_route) after a hit-buffer
+                          overflow or, on k_sym steps, because their previous neighbours all
+                          left the radius (a wrap) */
   int64_t grid_pairs;  /* grid mode, cumulative: (query, candidate) pairs evaluated over the
                           27-cell stencils -- the grid search's algorithmic work */
   int64_t step_index;  /* steps taken by this handle (the t of the think schedule) */
@@ -202,8 +204,9 @@ BOIDS_API int boids_info(boids_ctx* ctx, boids_info_t* out);
 
 /* Accumulated kernel time (ms) and launch count per kernel class since the last
  * reset, measured with CUDA events on the handle's stream (BOIDS_OPT_PROFILE).
- * Classes: 0 fused/search, 1 update, 2 binning, 3 grid search.  Synchronises. */
-#define BOIDS_PROF_CLASSES 4
+ * Classes: 0 fused/search, 1 update, 2 binning, 3 grid search, 4 k_route (agents searched
+ * whole after a hit-buffer overflow or a wrap).  Synchronises. */
+#define BOIDS_PROF_CLASSES 5
 BOIDS_API int boids_get_profile(boids_ctx* ctx, double* ms, int64_t* launches, int32_t reset);
 
 /* Diagnostics: copy `count` u64 phase stamps (8 per CTA) of the last fused step to host. */

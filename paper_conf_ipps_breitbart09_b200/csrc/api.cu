@@ -77,7 +77,9 @@ struct boids_ctx {
   // grid mode (BOIDS_GRID): search grid and its binning buffers
   BinGrid sgrid{};
   int2* gcellrank = nullptr;
-  int32_t *gcnt = nullptr, *gstart = nullptr, *gqstart = nullptr, *item_start = nullptr, *counter = nullptr;
+  int32_t *gcnt = nullptr, *gstart = nullptr, *gqstart = nullptr, *counter = nullptr;
+  int4* gitems = nullptr;      // grid search work items (k_bin_scan)
+  int32_t* gnitems = nullptr;  // their number
   float4* spos = nullptr;
   float* stage = nullptr;  // host-transfer staging [13][m] (lazy)
   // double-buffered readback (lazy): packed draw matrices, copy stream, events
@@ -105,8 +107,8 @@ struct boids_ctx {
   };
   std::vector<Rec> recs;
   std::vector<cudaEvent_t> pool;
-  double prof_ms[BOIDS_PROF_CLASSES] = {0, 0, 0, 0};
-  int64_t prof_n[BOIDS_PROF_CLASSES] = {0, 0, 0, 0};
+  double prof_ms[BOIDS_PROF_CLASSES] = {0, 0, 0, 0, 0};
+  int64_t prof_n[BOIDS_PROF_CLASSES] = {0, 0, 0, 0, 0};
 
   float4* local() const { return shard ? buf[1] : buf[cur]; }
 };
@@ -164,7 +166,8 @@ void free_ctx(boids_ctx* c) {
   cudaFree(c->gcnt);
   cudaFree(c->gstart);
   cudaFree(c->gqstart);
-  cudaFree(c->item_start);
+  cudaFree(c->gitems);
+  cudaFree(c->gnitems);
   cudaFree(c->counter);
   cudaFree(c->spos);
   cudaFree(c->stage);
@@ -287,8 +290,11 @@ int create_impl(int64_t n, const boids_params* p, uint64_t seed, int32_t rank, i
         (rc = alloc((void**)&c->gcnt, C * sizeof(int32_t))) ||
         (rc = alloc((void**)&c->gstart, (C + 1) * sizeof(int32_t))) ||
         (rc = alloc((void**)&c->gqstart, (C + 1) * sizeof(int32_t))) ||
-        (rc = alloc((void**)&c->item_start, (C + 1) * sizeof(int32_t))) ||
+        (rc = alloc((void**)&c->gitems, (size_t)(C + m / grid_chunk() + 2) * sizeof(int4))) ||
+        (rc = alloc((void**)&c->gnitems, sizeof(int32_t))) ||
         (rc = alloc((void**)&c->counter, sizeof(int32_t))) ||
+        (rc = alloc((void**)&c->sym_rlist, m * sizeof(int32_t))) ||
+        (rc = alloc((void**)&c->sym_rcount, sizeof(int32_t))) ||
         (rc = alloc((void**)&c->spos, (size_t)n * sizeof(float4)))) {
       free_ctx(c);
       return rc;
@@ -376,7 +382,7 @@ StepArgs make_args(boids_ctx* c, float dt) {
   a.qcount = nullptr;
   a.nq = c->nloc;
   a.routed = c->p.think_every > 1 ? c->routed : nullptr;
-  a.rlist = c->sym_rlist;  // warm steps route overflowed agents to k_route (nullptr in grid mode)
+  a.rlist = c->sym_rlist;  // warm brute-force steps route overflowed agents to k_route
   a.rcount = c->sym_rcount;
   return a;
 }
@@ -403,10 +409,12 @@ int one_step(boids_ctx* c, float dt) {
     if ((rc = launch(c, 2, [&] {
            cudaError_t e = launch_bin(a.full, c->m, a.sdiv, 0, slots, c->sgrid, c->gcellrank, c->gcnt, c->gstart,
                                       c->spos, one ? c->qperm : nullptr, 0, c->stream, nullptr,
-                                      one ? c->item_start : nullptr, chunk, one ? c->counter : nullptr);
+                                      one ? c->gitems : nullptr, one ? c->gnitems : nullptr, chunk,
+                                      one ? c->counter : nullptr);
            if (e == cudaSuccess && !one)
              e = launch_bin(a.full, c->m, a.sdiv, c->lo, c->nloc, c->sgrid, c->gcellrank, c->gcnt, c->gqstart,
-                            nullptr, c->qperm, (int)c->lo, c->stream, nullptr, c->item_start, chunk, c->counter,
+                            nullptr, c->qperm, (int)c->lo, c->stream, nullptr, c->gitems, c->gnitems, chunk,
+                            c->counter,
                             c->p.think_every, c->step_index);
            return e;
          }, one ? 3 : 6)))
@@ -416,12 +424,17 @@ int one_step(boids_ctx* c, float dt) {
     g.cstart = c->gstart;
     g.qstart = one ? c->gstart : c->gqstart;
     g.qperm = c->qperm;
-    g.item_start = c->item_start;
+    g.items = c->gitems;
+    g.nitems = c->gnitems;
+    g.flist = c->sym_rlist;  // (the brute-force routing list; unused in grid mode otherwise)
+    g.fcount = c->sym_rcount;
     g.counter = c->counter;
     g.grid = c->sgrid;
     StepArgs ag = a;
     ag.store_only = think ? 1 : 0;
+    CK(cudaMemsetAsync(c->sym_rcount, 0, sizeof(int32_t), c->stream));
     if ((rc = launch(c, 3, [&] { return launch_grid(ag, g, c->stream); }))) return rc;
+    if ((rc = launch(c, 4, [&] { return launch_grid_far(ag, g, c->stream); }))) return rc;
     if (think && (rc = launch(c, 1, [&] { return launch_apply(a, c->stream); }))) return rc;
   } else if (c->kernel == BOIDS_KERNEL_SIMPLE) {
     if ((rc = launch(c, 0, [&] { return launch_search_simple(a, c->stream); }))) return rc;
@@ -461,7 +474,7 @@ int one_step(boids_ctx* c, float dt) {
       CK(cudaMemsetAsync(c->sym_rcount, 0, sizeof(int32_t), c->stream));
       if ((rc = launch(c, 0, [&] { return launch_warm_scan(aw, c->stream); }, 2))) return rc;
       if ((rc = launch(c, 1, [&] { return launch_warm_select(a, c->stream); }))) return rc;
-      if ((rc = launch(c, 0, [&] { return launch_route(a, c->stream); }))) return rc;
+      if ((rc = launch(c, 4, [&] { return launch_route(a, c->stream); }))) return rc;
     } else if (warm_path) {
       // warm step: all-pairs scan appending passing keys, then select + update;
       // a single-GPU handle evaluates each unordered pair once (k_sym)
@@ -474,12 +487,12 @@ int one_step(boids_ctx* c, float dt) {
         if ((rc = launch(c, 0, [&] { return launch_sym_scan(as, c->sym_sp, c->sym_idx, c->stream); }, 2)))
           return rc;
         if ((rc = launch(c, 1, [&] { return launch_warm_select(as, c->stream); }))) return rc;
-        if ((rc = launch(c, 0, [&] { return launch_route(as, c->stream); }))) return rc;
+        if ((rc = launch(c, 4, [&] { return launch_route(as, c->stream); }))) return rc;
       } else {
         CK(cudaMemsetAsync(c->sym_rcount, 0, sizeof(int32_t), c->stream));
         if ((rc = launch(c, 0, [&] { return launch_warm_scan(a, c->stream); }, 2))) return rc;
         if ((rc = launch(c, 1, [&] { return launch_warm_select(a, c->stream); }))) return rc;
-        if ((rc = launch(c, 0, [&] { return launch_route(a, c->stream); }))) return rc;
+        if ((rc = launch(c, 4, [&] { return launch_route(a, c->stream); }))) return rc;
       }
     } else {
       // cold step (no previous lists) or forced: the cluster kernel

@@ -62,6 +62,7 @@ struct BinGrid {
   int dim[3];
   int cells;
   int morton;  // 1: cell id = Morton code (dim must be a power of two), 0: row-major
+  int reach;   // search grid: cells per axis an agent closer than r can be away (h * reach >= r)
 };
 
 struct StepArgs {
@@ -95,7 +96,7 @@ struct StepArgs {
   float* qlim;                // warm path: [nloc] inclusive search limit min(prev(r2), t0) (k_bound)
   // think frequency: agent j thinks at step step_t iff (j + step_t) % think_k == 0
   int32_t think_k;            // 1 = every agent thinks every step
-  int32_t store_only;         // search epilogues store F in fstore instead of modifying
+  int32_t store_only;         // search epilogues: 1 store F in fstore instead of modifying, 2 both
   int64_t step_t;
   float4* fstore;             // [nloc] last steering vector of each agent
   const int32_t* qcount;      // device-side number of query slots (qperm entries), nullptr = nloc
@@ -115,8 +116,11 @@ struct GridArgs {
   const int* cstart;      // [cells + 1] start of each cell in spos
   const int* qstart;      // [cells + 1] start of each cell in qperm (owned agents)
   const int* qperm;       // owned agents (local indices) sorted by cell
-  const int* item_start;  // [cells + 1] first work item (cell, chunk of 512 owned agents) per cell
+  const int4* items;      // work items (first query slot, count, first cell, x span) (k_bin_scan)
+  const int* nitems;      // their number
   int* counter;           // work-queue counter (reset by the binning scan)
+  int* flist;             // queries routed to k_grid_far (limit beyond the adjacent cells)
+  int* fcount;            // their number (zeroed before k_grid)
   BinGrid grid;
 };
 
@@ -130,7 +134,7 @@ cudaError_t launch_fill_phantoms(float4* seg_base, int64_t m, int64_t nloc, int6
                                  cudaStream_t s);
 cudaError_t launch_bin(const float4* full, int64_t m, const SliceDiv& sd, int64_t j0, int64_t count, const BinGrid& g,
                        int2* cellrank, int* cnt, int* start, float4* spos, int* perm, int perm_base,
-                       cudaStream_t s, int* launches, int* item_start = nullptr, int chunk = 1,
+                       cudaStream_t s, int* launches, int4* items = nullptr, int* nitems = nullptr, int chunk = 1,
                        int* counter = nullptr, int think_k = 1, int64_t think_t = 0);
 BinGrid make_locality_grid(int64_t n, const boids_params& p);
 BinGrid make_search_grid(const boids_params& p);
@@ -149,6 +153,7 @@ cudaError_t launch_update(const StepArgs& a, cudaStream_t s);
 cudaError_t launch_fused(const StepArgs& a, int cluster, cudaStream_t s);
 cudaError_t launch_warm_scan(const StepArgs& a, cudaStream_t s);
 cudaError_t launch_grid(const StepArgs& a, const GridArgs& g, cudaStream_t s);
+cudaError_t launch_grid_far(const StepArgs& a, const GridArgs& g, cudaStream_t s);
 int grid_chunk();
 cudaError_t launch_warm_select(const StepArgs& a, cudaStream_t s);
 int64_t sym_capacity(int64_t nloc);

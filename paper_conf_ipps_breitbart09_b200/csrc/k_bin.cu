@@ -108,15 +108,59 @@ __device__ __forceinline__ int block_scan_runs(int* sh, int C, int* warp_sums) {
   return total;
 }
 
+// Work items of the grid search from the (query) cell starts in sh (padded
+// layout): runs of consecutive non-empty cells along x in one row holding at most
+// `chunk` agents together; a cell with more than `chunk` agents is split into
+// chunk-sized items of its own; a run spans at most MAX_SPAN cells.  Item = (first query slot, count, first cell,
+// last x - first x).  One thread per row; pass 0 counts, pass 1 writes.
+constexpr int MAX_SPAN = 8;  // cells per item: wider runs scan more candidates per query (think mode)
+__device__ __forceinline__ int row_items(const int* sh, int C, int total, int row, int D, int chunk, int4* out) {
+  int n = 0, acc = 0, xs = -1, q0 = 0;
+  auto cnt_of = [&](int c, int& s0) {
+    s0 = sh[c + (c >> 5)];
+    const int s1 = c + 1 < C ? sh[(c + 1) + ((c + 1) >> 5)] : total;
+    return s1 - s0;
+  };
+  auto close = [&](int xe) {
+    if (xs >= 0) {
+      if (out) out[n] = make_int4(q0, acc, row * D + xs, xe - xs);
+      ++n;
+    }
+    xs = -1;
+    acc = 0;
+  };
+  for (int x = 0; x < D; ++x) {
+    int s0;
+    const int k = cnt_of(row * D + x, s0);
+    if (k == 0) {
+      close(x - 1);
+    } else if (k > chunk) {
+      close(x - 1);
+      for (int i = 0; i < k; i += chunk) {
+        if (out) out[n] = make_int4(s0 + i, min(chunk, k - i), row * D + x, 0);
+        ++n;
+      }
+    } else {
+      if (acc + k > chunk || (xs >= 0 && x - xs >= MAX_SPAN)) close(x - 1);
+      if (xs < 0) {
+        xs = x;
+        q0 = s0;
+      }
+      acc += k;
+    }
+  }
+  close(D - 1);
+  return n;
+}
+
 // Exclusive scan of cnt[0..C) into start[0..C], start[C] = total; zeroes cnt.
 // One CTA; counts are staged through shared memory with coalesced accesses.
-// With item_start: also the work items of the grid search -- ceil(count / chunk)
-// per cell -- scanned into item_start[0..C] (item_start[C] = number of items),
-// and the grid kernel's work counter is reset.
+// With items: also the work items of the grid search (row_items) into
+// items[0..*nitems), and the grid kernel's work counter is reset.
 __global__ void __launch_bounds__(SCAN_T) k_bin_scan(int* __restrict__ cnt, int* __restrict__ start, int C,
-                                                    int* __restrict__ item_start, int chunk,
-                                                    int* __restrict__ counter) {
-  extern __shared__ int sh[];  // C + C / 32 words
+                                                    int4* __restrict__ items, int* __restrict__ nitems, int chunk,
+                                                    int* __restrict__ counter, int D) {
+  extern __shared__ int sh[];  // C + C / 32 words, then (items) rows + rows / 32 + 1 words
   __shared__ int warp_sums[SCAN_T / 32];
   const int tid = threadIdx.x;
   for (int i = tid; i < C; i += SCAN_T) {
@@ -127,23 +171,15 @@ __global__ void __launch_bounds__(SCAN_T) k_bin_scan(int* __restrict__ cnt, int*
   const int total = block_scan_runs(sh, C, warp_sums);
   for (int i = tid; i < C; i += SCAN_T) start[i] = sh[i + (i >> 5)];
   if (tid == 0) start[C] = total;
-  if (!item_start) return;
+  if (!items) return;
+  const int rows = C / D;
+  int* rc = sh + C + (C >> 5) + 1;
+  for (int r = tid; r < rows; r += SCAN_T) rc[r + (r >> 5)] = row_items(sh, C, total, r, D, chunk, nullptr);
   __syncthreads();
-  for (int i = tid; i < C; i += SCAN_T) {  // chunks per cell from the starts
-    const int s0 = sh[i + (i >> 5)];
-    const int s1 = i + 1 < C ? sh[(i + 1) + ((i + 1) >> 5)] : total;
-    cnt[i] = (s1 - s0 + chunk - 1) / chunk;  // cnt is scratch here (re-zeroed below)
-  }
-  __syncthreads();
-  for (int i = tid; i < C; i += SCAN_T) sh[i + (i >> 5)] = cnt[i];
-  __syncthreads();
-  const int items = block_scan_runs(sh, C, warp_sums);
-  for (int i = tid; i < C; i += SCAN_T) {
-    item_start[i] = sh[i + (i >> 5)];
-    cnt[i] = 0;
-  }
+  const int n = block_scan_runs(rc, rows, warp_sums);
+  for (int r = tid; r < rows; r += SCAN_T) row_items(sh, C, total, r, D, chunk, items + rc[r + (r >> 5)]);
   if (tid == 0) {
-    item_start[C] = items;
+    *nitems = n;
     *counter = 0;
   }
 }
@@ -166,54 +202,67 @@ __global__ void k_bin_scatter(const float4* __restrict__ full, int64_t m, SliceD
 
 cudaError_t launch_bin(const float4* full, int64_t m, const SliceDiv& sd, int64_t j0, int64_t count, const BinGrid& g,
                        int2* cellrank, int* cnt, int* start, float4* spos, int* perm, int perm_base,
-                       cudaStream_t s, int* launches, int* item_start, int chunk, int* counter, int think_k,
-                       int64_t think_t) {
+                       cudaStream_t s, int* launches, int4* items, int* nitems, int chunk, int* counter,
+                       int think_k, int64_t think_t) {
   const unsigned blocks = (unsigned)((count + 255) / 256);
+  const int rows = g.cells / g.dim[0];
+  const size_t shm = (size_t)(g.cells + g.cells / 32 + 1 + (items ? rows + rows / 32 + 1 : 0)) * sizeof(int);
+  if (shm > 48 * 1024) {
+    cudaError_t e = cudaFuncSetAttribute(k_bin_scan, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)shm);
+    if (e != cudaSuccess) return e;
+  }
   if (count <= 0) {  // still publish an empty binning (starts, items, counter)
-    const size_t shm0 = (size_t)(g.cells + g.cells / 32 + 1) * sizeof(int);
-    if (shm0 > 48 * 1024) cudaFuncSetAttribute(k_bin_scan, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)shm0);
-    k_bin_scan<<<1, SCAN_T, shm0, s>>>(cnt, start, g.cells, item_start, chunk, counter);
+    k_bin_scan<<<1, SCAN_T, shm, s>>>(cnt, start, g.cells, items, nitems, chunk, counter, g.dim[0]);
     return cudaGetLastError();
   }
   k_bin_count<<<blocks, 256, 0, s>>>(full, m, sd, j0, count, g, cellrank, cnt, spos == nullptr,
                                      spos == nullptr ? think_k : 1, think_t);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return e;
-  const size_t shm = (size_t)(g.cells + g.cells / 32 + 1) * sizeof(int);
-  if (shm > 48 * 1024) {
-    e = cudaFuncSetAttribute(k_bin_scan, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)shm);
-    if (e != cudaSuccess) return e;
-  }
-  k_bin_scan<<<1, SCAN_T, shm, s>>>(cnt, start, g.cells, item_start, chunk, counter);
+  k_bin_scan<<<1, SCAN_T, shm, s>>>(cnt, start, g.cells, items, nitems, chunk, counter, g.dim[0]);
   if ((e = cudaGetLastError()) != cudaSuccess) return e;
   k_bin_scatter<<<blocks, 256, 0, s>>>(full, m, sd, j0, count, cellrank, start, spos, perm, perm_base);
   if (launches) *launches += 3;
   return cudaGetLastError();
 }
 
-// Search grid of BOIDS_GRID: cells of size h = r (1 + 2^-10) (a margin far above
-// the fp32 rounding of the cell coordinate and of d2 < r2), row-major over the
-// world box [-B, B]^3, B = max(world, init radius) * 1.02; agents outside are
-// clamped into boundary cells, which keeps every pair closer than r in the same
-// or adjacent cells (clamping is monotone and 1-Lipschitz on cell coordinates).
-// The 27-cell stencil of a cell is then 9 contiguous x-runs of the sorted array.
+// Search grid of BOIDS_GRID: row-major over the world box [-B, B]^3, B = max(world,
+// init radius) * 1.02; agents outside are clamped into boundary cells (clamping
+// is monotone and 1-Lipschitz on cell coordinates, so it never separates a pair
+// by more cells than the distance allows).  Cells are SMALLER than r: h =
+// r (1 + 2^-10) / 3, so an agent closer than r lies within `reach` = 3 cells per
+// axis (the 2^-10 margin is far above the fp32 rounding of the cell coordinate
+// and of d2), and the warm bound of k_grid prunes the stencil to the cells its
+// queries can reach (usually 1 per axis: 27 small cells instead of 27 cells of
+// size r).  The table is capped at MAXD cells per axis (single-CTA scan in
+// shared memory): larger worlds get larger cells and a smaller reach (>= 1).
+constexpr int MAXD = 34;
 BinGrid make_search_grid(const boids_params& p) {
   BinGrid g{};
   const float B = fmaxf(p.world_radius, p.init_radius) * 1.02f;
-  g.h = p.search_radius * (1.0f + 1.0f / 1024.0f);
-  int dim = (int)ceilf(2.f * B / g.h);
-  if (dim < 1) dim = 1;
-  if (dim > 1024) {  // huge world vs radius: cap the table (cells grow, still >= r)
-    dim = 1024;
-    g.h = 2.f * B / dim;
+  const float hr = p.search_radius * (1.0f + 1.0f / 1024.0f);  // >= r with margin
+  int reach = 3;
+  float h = hr / 3.f;
+  int dim = (int)ceilf(2.f * B / h);
+  while (dim > MAXD && reach > 1) {  // coarser cells: reach 2, then 1 (cells >= r)
+    --reach;
+    h = hr / (float)reach;
+    dim = (int)ceilf(2.f * B / h);
   }
+  if (dim > MAXD) {  // cells larger than r (reach 1 still covers r)
+    dim = MAXD;
+    h = fmaxf(hr, 2.f * B / dim * (1.0f + 1.0f / 1024.0f));
+  }
+  if (dim < 1) dim = 1;
   for (int d = 0; d < 3; ++d) {
     g.lo[d] = -B;
     g.dim[d] = dim;
   }
+  g.h = h;
   g.inv_h = 1.f / g.h;
   g.cells = dim * dim * dim;
   g.morton = 0;
+  g.reach = reach;
   return g;
 }
 

@@ -3,17 +3,26 @@
 //
 // The thesis names spatial data structures as the way to speed up the neighbour
 // search (future work); north_star asks for a uniform-grid variant that
-// returns the IDENTICAL neighbour sets.  Cells have size h >= r (make_search_grid),
-// so every agent closer than r lies in the same or one of the 26 adjacent cells;
-// within those the search is exactly the brute-force definition (d2 < fl(r*r),
-// top-7 by the (d2, index) key, Listing 5.2 / 6.3 with readings Q2-Q4), so the
-// result is bit-identical to BOIDS_BRUTE.
+// returns the IDENTICAL neighbour sets.  Cells have size h >= r / reach
+// (make_search_grid, reach = 3 by default), so every agent closer than r lies
+// within `reach` cells per axis; within those the search is exactly the
+// brute-force definition (d2 < fl(r*r), top-7 by the (d2, index) key, Listing
+// 5.2 / 6.3 with readings Q2-Q4), so the result is bit-identical to BOIDS_BRUTE.
 //
-// Work item = (cell, chunk of <= 512 of the cell's owned agents).  A persistent
-// grid of CTAs pulls items from an atomic queue (cells hold very different
-// numbers of agents -- the flock is a ball inside a box -- so static splits
-// would be unbalanced).  Row-major cell order makes the 3 cells along x of each
-// of the 9 stencil rows one contiguous range of the sorted candidate array; the
+// Stencil pruning by the warm bound: only agents with d2 <= lim_i can enter query
+// i's list (lim_i = min(prev(r2), t0_i), the bound of k_warm.cu), and such an
+// agent is at most floor(sqrt(lim_i) / h) + 1 cells away per axis.  Each item
+// takes R = that reach for the largest limit among its queries (capped at
+// `reach`; a cold step or a wrapped agent gives the full reach), so a warm step
+// typically scans 3 x 3 x 3 cells of r/3 -- 1/27 of the volume of the
+// unpruned 27-cell stencil of cells >= r.
+//
+// Work item = a run of consecutive cells along x in one row holding <= 512
+// owned agents (a larger cell is split into chunks of its own; k_bin_scan).  A
+// persistent grid of CTAs pulls items from an atomic queue (cells hold very
+// different numbers of agents -- the flock is a ball inside a box).  Row-major
+// cell order makes each of the (2R+1)^2 stencil rows one contiguous range of the
+// sorted candidate array (x from the run's first cell - R to its last + R); the
 // ranges stream through a TMA ring (cp.async.bulk of any 16-byte multiple, so
 // partial tiles need no padding).  A query's whole stencil is scanned by one CTA,
 // so its top-7 list (shared memory, limit tightened by the warm bound and by the
@@ -32,14 +41,18 @@ constexpr int QBG = NTG * Q;    // queries per item (512)
 constexpr int CT = 256;         // candidates per tile (<= 4 KB bulk copy)
 constexpr int STAGES = 3;
 constexpr int U = 4;
+constexpr int FAR_MAX = 16;  // queries per item routed to k_grid_far
 
 struct __align__(16) GridSmem {
   float4 ring[STAGES][CT];
   key_t lists[7 * QBG];  // [7][QBG]
   uint64_t full[STAGES];
   uint64_t empty[STAGES];
-  int2 range[9];         // stencil row ranges [lo, hi) in the sorted candidate array
-  int nrange, item, cell, qs0, qn;
+  int2 range[49];        // stencil row ranges [lo, hi) in the sorted candidate array ((2R+1)^2 <= 49)
+  int nrange, item, cell, span, qs0, qn;
+  int maxlim;            // largest query limit of the item (float bits; limits are >= 0)
+  int maxnear;           // ... over the queries that need only the adjacent cells
+  int nfar;              // queries that need more (routed to k_grid_far when few)
 };
 
 __device__ __forceinline__ int tile_count(const GridSmem& sm, int r, int off) {
@@ -80,7 +93,7 @@ __global__ void __launch_bounds__(NTG) k_grid(StepArgs a, GridArgs g) {
   const float r2 = __fmul_rn(a.p.search_radius, a.p.search_radius);
   const float r2_in = __uint_as_float(__float_as_uint(r2) - 1u);  // d2 < r2  <=>  d2 <= r2_in
   const int D = g.grid.dim[0];
-  const int n_items = g.item_start[g.grid.cells];
+  const int n_items = *g.nitems;
   uint32_t tc = 0;  // tiles issued / consumed by this CTA
   unsigned slow_groups = 0, groups = 0;
   for (;;) {
@@ -89,45 +102,21 @@ __global__ void __launch_bounds__(NTG) k_grid(StepArgs a, GridArgs g) {
       const int it = atomicAdd(g.counter, 1);
       sm.item = it;
       if (it < n_items) {
-        // cell = last c with item_start[c] <= it (binary search)
-        int lo = 0, hi = g.grid.cells;
-        while (hi - lo > 1) {
-          const int mid = (lo + hi) >> 1;
-          if (g.item_start[mid] <= it) lo = mid;
-          else hi = mid;
-        }
-        const int cell = lo;
-        sm.cell = cell;
-        sm.qs0 = g.qstart[cell] + (it - g.item_start[cell]) * QBG;
-        sm.qn = min(QBG, g.qstart[cell + 1] - sm.qs0);
-        const int cx = cell % D, cy = (cell / D) % D, cz = cell / (D * D);
-        const int x0 = max(cx - 1, 0), x1 = min(cx + 1, D - 1);
-        int nr = 0;
-        for (int z = max(cz - 1, 0); z <= min(cz + 1, D - 1); ++z)
-          for (int y = max(cy - 1, 0); y <= min(cy + 1, D - 1); ++y) {
-            const int row = (z * D + y) * D;
-            const int lo_r = g.cstart[row + x0], hi_r = g.cstart[row + x1 + 1];
-            if (hi_r > lo_r) sm.range[nr++] = make_int2(lo_r, hi_r);
-          }
-        sm.nrange = nr;
-        if (a.stats) {
-          long long cand = 0;
-          for (int r = 0; r < nr; ++r) cand += sm.range[r].y - sm.range[r].x;
-          atomicAdd(a.stats + 3, (unsigned long long)(cand * sm.qn));
-        }
-        // producer: first tiles of the item
-        int r = 0, off = 0;
-        for (int t = 0; t < STAGES && r < nr; ++t) {
-          issue(sm, g, tc + t, r, off);
-          next_tile(sm, r, off);
-        }
+        const int4 w = g.items[it];
+        sm.qs0 = w.x;
+        sm.qn = w.y;
+        sm.cell = w.z;
+        sm.span = w.w;
       }
+      sm.maxlim = 0;
+      sm.maxnear = 0;
+      sm.nfar = 0;
     }
     __syncthreads();
     if (sm.item >= n_items) break;
-    const int nr = sm.nrange, qs0 = sm.qs0, qn = sm.qn;
+    const int qs0 = sm.qs0, qn = sm.qn;
 
-    // queries: 4 per thread
+    // queries: 4 per thread, with their limits (the warm bound)
     float2 pxy[Q];
     float pz[Q], lim[Q];
     int gq[Q];
@@ -146,6 +135,80 @@ __global__ void __launch_bounds__(NTG) k_grid(StepArgs a, GridArgs g) {
 #pragma unroll
       for (int s = 0; s < 7; ++s) sm.lists[s * QBG + slot] = KEY_EMPTY;
     }
+    {
+      // A query whose limit reaches past the adjacent cells (a wrapped agent, a
+      // neighbour that left) would widen the whole item's stencil: up to FAR_MAX
+      // of them per item are routed to k_grid_far (one CTA each, own stencil)
+      // and skipped here.  More than that (a cold step) -> the item takes the
+      // full reach itself.
+      float ml = 0.f, mn = 0.f;  // max limit over all / over the near queries
+      bool far[Q];
+      int nf = 0;
+#pragma unroll
+      for (int q = 0; q < Q; ++q) {
+        const bool valid = qloc[q] < a.nloc;
+        far[q] = valid && g.flist && sqrtf(lim[q]) * g.grid.inv_h * (1.0f + 1.0f / 1024.0f) >= 1.0f;
+        if (valid) ml = fmaxf(ml, lim[q]);
+        if (valid && !far[q]) mn = fmaxf(mn, lim[q]);
+        nf += far[q] ? 1 : 0;
+      }
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) {
+        ml = fmaxf(ml, __shfl_xor_sync(0xffffffffu, ml, o));
+        mn = fmaxf(mn, __shfl_xor_sync(0xffffffffu, mn, o));
+        nf += __shfl_xor_sync(0xffffffffu, nf, o);
+      }
+      if (lane == 0) {
+        atomicMax(&sm.maxlim, __float_as_int(ml));
+        atomicMax(&sm.maxnear, __float_as_int(mn));
+        atomicAdd(&sm.nfar, nf);
+      }
+      __syncthreads();
+      if (sm.nfar > 0 && sm.nfar <= FAR_MAX) {
+#pragma unroll
+        for (int q = 0; q < Q; ++q)
+          if (far[q]) {
+            g.flist[atomicAdd(g.fcount, 1)] = (int)qloc[q];
+            qloc[q] = a.nloc;  // not finished here
+            pxy[q] = make_float2(__int_as_float(0x7fc00000), 0.f);
+            lim[q] = -1.f;
+          }
+        if (tid == 0) sm.maxlim = sm.maxnear;
+      }
+    }
+    __syncthreads();
+    if (tid == 0) {
+      // stencil reach of this item: agents within sqrt(maxlim) are at most
+      // floor(sqrt(maxlim) / h) + 1 cells away per axis (margin 2^-10 >> fp32 rounding)
+      const float ml = __int_as_float(sm.maxlim);
+      const int Rg = g.grid.reach;
+      const float cells = sqrtf(ml) * g.grid.inv_h * (1.0f + 1.0f / 1024.0f);
+      const int R = cells >= (float)Rg ? Rg : min(Rg, 1 + (int)cells);
+      const int cell = sm.cell;
+      const int cx = cell % D, cy = (cell / D) % D, cz = cell / (D * D);
+      const int x0 = max(cx - R, 0), x1 = min(cx + sm.span + R, D - 1);
+      int nr = 0;
+      for (int z = max(cz - R, 0); z <= min(cz + R, D - 1); ++z)
+        for (int y = max(cy - R, 0); y <= min(cy + R, D - 1); ++y) {
+          const int row = (z * D + y) * D;
+          const int lo_r = g.cstart[row + x0], hi_r = g.cstart[row + x1 + 1];
+          if (hi_r > lo_r) sm.range[nr++] = make_int2(lo_r, hi_r);
+        }
+      sm.nrange = nr;
+      if (a.stats) {
+        long long cand = 0;
+        for (int r = 0; r < nr; ++r) cand += sm.range[r].y - sm.range[r].x;
+        atomicAdd(a.stats + 3, (unsigned long long)(cand * sm.qn));
+      }
+      // producer: first tiles of the item
+      int r = 0, off = 0;
+      for (int t = 0; t < STAGES && r < nr; ++t) {
+        issue(sm, g, tc + t, r, off);
+        next_tile(sm, r, off);
+      }
+    }
+    __syncthreads();
+    const int nr = sm.nrange;
     float limc = fmaxf(fmaxf(lim[0], lim[1]), fmaxf(lim[2], lim[3]));
     __syncwarp();
 
@@ -159,7 +222,8 @@ __global__ void __launch_bounds__(NTG) k_grid(StepArgs a, GridArgs g) {
       mbar_wait(&sm.full[s], (tc / STAGES) & 1u);
       const float4* tile = sm.ring[s];
       const int cnt = tile_count(sm, r, off);
-      for (int c = 0; c < cnt; c += U) {
+      // warps without queries in this item only keep the ring protocol
+      for (int c = 0; c < (warp * 32 * Q < qn ? cnt : 0); c += U) {
         float4 cc[U];
         if (c + U <= cnt) {
 #pragma unroll
@@ -217,7 +281,7 @@ __global__ void __launch_bounds__(NTG) k_grid(StepArgs a, GridArgs g) {
 #pragma unroll
     for (int q = 0; q < Q; ++q) {
       const int slot = warp * 32 * Q + q * 32 + lane;
-      if (slot < qn) {
+      if (slot < qn && qloc[q] < a.nloc) {
         key_t A[7];
 #pragma unroll
         for (int s = 0; s < 7; ++s) A[s] = sm.lists[s * QBG + slot];
@@ -231,7 +295,93 @@ __global__ void __launch_bounds__(NTG) k_grid(StepArgs a, GridArgs g) {
   }
 }
 
+// Queries routed by k_grid (limit beyond the adjacent cells): one CTA per agent
+// scans its own stencil -- the reach of its own limit -- with the exact
+// brute-force test, per-thread top-7 lists merged by a shuffle butterfly and a
+// shared-memory pass, then finishes the agent.
+constexpr int FT = 128;
+__global__ void __launch_bounds__(FT) k_grid_far(StepArgs a, GridArgs g) {
+  __shared__ key_t wl[FT / 32][7];
+  __shared__ int2 rng[49];
+  __shared__ int nrng;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int nf = *g.fcount;
+  const float r2 = __fmul_rn(a.p.search_radius, a.p.search_radius);
+  const float r2_in = __uint_as_float(__float_as_uint(r2) - 1u);
+  const int D = g.grid.dim[0];
+  for (int f = blockIdx.x; f < nf; f += gridDim.x) {
+    const int qi = g.flist[f];
+    const float4 me = __ldg(pos_of(a.full, a.m, a.sdiv, a.lo + qi));
+    const int gi = (int)(a.lo + qi);
+    const float lim = fminf(r2_in, a.warm ? warm_bound(a, qi, me) : __int_as_float(0x7f800000));
+    if (tid == 0) {
+      const int Rg = g.grid.reach;
+      const float cells = sqrtf(lim) * g.grid.inv_h * (1.0f + 1.0f / 1024.0f);
+      const int R = cells >= (float)Rg ? Rg : min(Rg, 1 + (int)cells);
+      const float4 c4 = me;
+      auto coord = [&](float v, int d) {
+        const int c = (int)floorf((v - g.grid.lo[d]) * g.grid.inv_h);
+        return c < 0 ? 0 : (c >= g.grid.dim[d] ? g.grid.dim[d] - 1 : c);
+      };
+      const int cx = coord(c4.x, 0), cy = coord(c4.y, 1), cz = coord(c4.z, 2);
+      const int x0 = max(cx - R, 0), x1 = min(cx + R, D - 1);
+      int nr = 0;
+      for (int z = max(cz - R, 0); z <= min(cz + R, D - 1); ++z)
+        for (int y = max(cy - R, 0); y <= min(cy + R, D - 1); ++y) {
+          const int row = (z * D + y) * D;
+          const int lo_r = g.cstart[row + x0], hi_r = g.cstart[row + x1 + 1];
+          if (hi_r > lo_r) rng[nr++] = make_int2(lo_r, hi_r);
+        }
+      nrng = nr;
+    }
+    __syncthreads();
+    key_t A[7];
+#pragma unroll
+    for (int s = 0; s < 7; ++s) A[s] = KEY_EMPTY;
+    for (int r = 0; r < nrng; ++r)
+      for (int k = rng[r].x + tid; k < rng[r].y; k += FT) {
+        const float4 c = __ldg(g.spos + k);
+        const float d2 = dist2(me.x, me.y, me.z, c);
+        const int j = __float_as_int(c.w);
+        if (d2 <= lim && j != gi) {
+          const key_t key = make_key(d2, j);
+          if (key < A[6]) insert7(A, key);
+        }
+      }
+#pragma unroll
+    for (int w = 1; w < 32; w <<= 1) {
+      key_t B[7];
+#pragma unroll
+      for (int s = 0; s < 7; ++s) B[s] = __shfl_xor_sync(0xffffffffu, A[s], w);
+      merge7(A, B);
+    }
+    if (lane == 0)
+#pragma unroll
+      for (int s = 0; s < 7; ++s) wl[warp][s] = A[s];
+    __syncthreads();
+    if (tid == 0) {
+      for (int w = 1; w < FT / 32; ++w) {
+        key_t B[7];
+#pragma unroll
+        for (int s = 0; s < 7; ++s) B[s] = wl[w][s];
+        merge7(A, B);
+      }
+      finish_agent(a, qi, A);
+    }
+    __syncthreads();
+  }
+}
+
 }  // namespace
+
+cudaError_t launch_grid_far(const StepArgs& a, const GridArgs& g, cudaStream_t s) {
+  if (!g.flist) return cudaSuccess;
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  k_grid_far<<<(unsigned)(4 * sms), FT, 0, s>>>(a, g);
+  return cudaGetLastError();
+}
 
 cudaError_t launch_grid(const StepArgs& a, const GridArgs& g, cudaStream_t s) {
   static int grid = 0;

@@ -380,6 +380,7 @@ __global__ void __launch_bounds__(256) k_sym_prep(StepArgs a, float4* __restrict
   if (c == 7 && t0 > r2_in && a.rlist) {
     a.rlist[atomicAdd(a.rcount, 1)] = qi;
     a.routed[qi] = 1;
+    if (a.stats) atomicAdd(a.stats + 2, 1ull);
     lim = -1.f;
   }
   sp[p] = make_float4(me.x, me.y, me.z, lim);
@@ -413,13 +414,12 @@ __device__ __forceinline__ void insert8(key_t (&L)[8], key_t k) {
 // 8 smallest keys per thread; a shuffle butterfly and a shared-memory pass merge
 // them.  The CTA then finishes the agent -- list, 8th nearest (the next step's
 // warm-bound seed), steering, modification -- and k_select skips it.
-constexpr int RT = 512;
+constexpr int RT = 512, RU = 16;
 __global__ void __launch_bounds__(RT) k_route(StepArgs a) {
   __shared__ key_t wl[RT / 32][8];
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int nr = *a.rcount;
   const float r2 = __fmul_rn(a.p.search_radius, a.p.search_radius);
-  const int64_t total = (int64_t)a.world * a.m;  // candidate slots (phantoms are NaN)
   for (int r = blockIdx.x; r < nr; r += gridDim.x) {
     const int qi = a.rlist[r];
     const float4 me = __ldg(pos_of(a.full, a.m, a.sdiv, a.lo + qi));
@@ -427,20 +427,28 @@ __global__ void __launch_bounds__(RT) k_route(StepArgs a) {
     key_t A[8];
 #pragma unroll
     for (int s = 0; s < 8; ++s) A[s] = KEY_EMPTY;
-    for (int64_t j0 = tid; j0 < total; j0 += RT * 4) {
-      float4 c[4];
+    // slice by slice (no per-candidate slice division); 16 independent loads in
+    // flight per thread: the candidates are L2-resident and this loop is
+    // latency-bound.  (Measured: k_fused on the compacted list instead costs
+    // 2.5-4 ms per step at C4 -- its grid is sized for all n.)
+    for (int sl = 0; sl < a.world; ++sl) {
+      const float4* base = a.full + (int64_t)sl * 2 * a.m;
+      const int jg0 = (int)((int64_t)sl * a.m);
+      for (int j0 = tid; j0 < (int)a.m; j0 += RT * RU) {
+        float4 c[RU];
 #pragma unroll
-      for (int u = 0; u < 4; ++u) {
-        const int64_t j = j0 + (int64_t)RT * u;
-        c[u] = j < total ? __ldg(pos_of(a.full, a.m, a.sdiv, j)) : make_float4(__int_as_float(0x7fc00000), 0.f, 0.f, 0.f);
-      }
+        for (int u = 0; u < RU; ++u) {
+          const int j = j0 + RT * u;
+          c[u] = j < (int)a.m ? __ldg(base + j) : make_float4(__int_as_float(0x7fc00000), 0.f, 0.f, 0.f);
+        }
 #pragma unroll
-      for (int u = 0; u < 4; ++u) {
-        const float d2 = dist2(me.x, me.y, me.z, c[u]);
-        const int j = (int)(j0 + (int64_t)RT * u);
-        if (d2 < r2 && j != g) {
-          const key_t k = make_key(d2, j);
-          if (k < A[7]) insert8(A, k);
+        for (int u = 0; u < RU; ++u) {
+          const float d2 = dist2(me.x, me.y, me.z, c[u]);
+          if (d2 < r2) {  // rare: in radius
+            const int j = jg0 + j0 + RT * u;
+            const key_t k = make_key(d2, j);
+            if (j != g && k < A[7]) insert8(A, k);
+          }
         }
       }
     }

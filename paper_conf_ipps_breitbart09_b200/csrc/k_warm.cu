@@ -445,6 +445,7 @@ __global__ void __launch_bounds__(NSEL) k_select(StepArgs a) {
       a.rlist[atomicAdd(a.rcount, 1)] = (int)qi;
       a.hitcnt[qi] = 0;
       a.pcnt[qi] = 0;
+      a.nbr8[qi] = -1;  // the router writes no 8th nearest: a stale one could repeat a new neighbour
       return;
     }
     om = 0;
@@ -465,7 +466,10 @@ __global__ void __launch_bounds__(NSEL) k_select(StepArgs a) {
   const float4 f4 = __ldg(fwd_of(a.full, a.m, a.sdiv, a.lo + qi));
   if (!active) {  // think mode, not searched by k_scan this step
     if (routed) a.routed[qi] = 0;
-    if (routed && a.think_k <= 1) return;  // k_sym step: k_route finished this agent
+    if (routed && a.think_k <= 1) {  // k_sym step: routed, finished by launch_route after this kernel
+      a.nbr8[qi] = -1;
+      return;
+    }
     const float4 F = a.fstore[qi];
     modify_agent(a, qi, v3(p4), f4, v3(F));
     return;

@@ -62,8 +62,9 @@ __device__ __forceinline__ void finish_agent(const StepArgs& a, int64_t qi, cons
   const float4 p4 = __ldg(pos_of(a.full, a.m, a.sdiv, a.lo + qi));
   const float4 f4 = __ldg(fwd_of(a.full, a.m, a.sdiv, a.lo + qi));
   const V3 F = steer_agent(a, v3(p4), v3(f4), nb, cnt);
-  if (a.store_only) a.fstore[qi] = make_float4(F.x, F.y, F.z, 0.f);  // think mode: k_apply modifies
-  else modify_agent(a, qi, v3(p4), f4, F);
+  // store_only 1: think mode, k_apply/k_select modifies later; 2: store and modify
+  if (a.store_only) a.fstore[qi] = make_float4(F.x, F.y, F.z, 0.f);
+  if (a.store_only != 1) modify_agent(a, qi, v3(p4), f4, F);
 }
 
 }  // namespace boids
