@@ -118,6 +118,11 @@ typedef struct boids_info_t {
                                        1 (default) = evaluate every unordered pair once and test it
                                        against both agents' limits (k_sym; d2 is bitwise symmetric),
                                        0 = every ordered pair (k_scan).  Results are identical. */
+#define BOIDS_OPT_BALANCE 9         /* k_sym work split: 1 (default) = cut the unordered-pair item space
+                                       so that every CTA gets an equal share of the SM time the previous
+                                       k_sym launch measured per item range (feedback; the first launch
+                                       uses a static weighted split), 0 = static split always.  Only the
+                                       partition of the work changes; results are identical. */
 #define BOIDS_OPT_PHASES 5          /* diagnostics: value = max CTAs; the fused kernel records per-CTA
                                        %globaltimer stamps (read with boids_get_phases); 0 = off */
 

@@ -21,7 +21,7 @@ BOIDS_BRUTE, BOIDS_GRID = 0, 1
 BOIDS_INIT_OPENSTEER, BOIDS_INIT_WORLD = 0, 1
 BOIDS_KERNEL_FUSED, BOIDS_KERNEL_SIMPLE, BOIDS_KERNEL_CLUSTER = 0, 1, 2
 BOIDS_OPT_RECORD_STEERING, BOIDS_OPT_KERNEL, BOIDS_OPT_PROFILE, BOIDS_OPT_CLUSTER, BOIDS_OPT_PHASES = 1, 2, 3, 4, 5
-BOIDS_OPT_RESORT, BOIDS_OPT_VOTE_U, BOIDS_OPT_SYMMETRIC = 6, 7, 8
+BOIDS_OPT_RESORT, BOIDS_OPT_VOTE_U, BOIDS_OPT_SYMMETRIC, BOIDS_OPT_BALANCE = 6, 7, 8, 9
 BOIDS_PROF_CLASSES = 5
 PROF_NAMES = ("fused_or_search", "update", "binning", "grid_search", "route")
 

@@ -8,14 +8,47 @@
 
 namespace boids {
 
-// Steering vector of agent g from its <=7 neighbours (in key order, Q8).
+// Diagnostics (BOIDS_OPT_PHASES): the span of a whole launch in slot `slot` of
+// the phase buffer -- [0] = ~(earliest CTA start), [1] = latest CTA end
+// (%globaltimer, ns), both by atomicMax so the buffer's zero fill is neutral.
+constexpr int SPAN_SLOT0 = 1000;
+__device__ __forceinline__ unsigned long long gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+__device__ __forceinline__ void span_begin(const StepArgs& a, int slot) {
+  if (a.phase && threadIdx.x == 0) atomicMax(a.phase + slot * 8, ~gtimer());
+}
+__device__ __forceinline__ void span_end(const StepArgs& a, int slot) {  // every thread of the CTA
+  if (a.phase) {
+    __syncthreads();
+    if (threadIdx.x == 0) atomicMax(a.phase + slot * 8 + 1, gtimer());
+  }
+}
+
+__device__ __forceinline__ void prefetch_l1(const void* p) {
+  asm volatile("prefetch.global.L1 [%0];" ::"l"(p));
+}
+
+// Steering vector of agent g from its <=7 neighbours (in key order, Q8).  The
+// neighbours' lines are prefetched into L1 up front and the loop is kept
+// rolled: this code runs once per agent per step, so at small n its
+// instruction-fetch latency, not its arithmetic, is what the warps wait on.
 __device__ __forceinline__ V3 steer_agent(const StepArgs& a, V3 me, V3 fme, const int* nb,
                                           int cnt) {
-  V3 sep = v3(0.f, 0.f, 0.f), coh = v3(0.f, 0.f, 0.f), ali = v3(0.f, 0.f, 0.f);
 #pragma unroll
-  for (int k = 0; k < 7; ++k) {
-    if (k >= cnt) break;
-    int64_t j = nb[k];
+  for (int k = 0; k < 7; ++k)
+    if (k < cnt) {
+      prefetch_l1(pos_of(a.full, a.m, a.sdiv, nb[k]));
+      prefetch_l1(fwd_of(a.full, a.m, a.sdiv, nb[k]));
+    }
+  int q0 = nb[0], q1 = nb[1], q2 = nb[2], q3 = nb[3], q4 = nb[4], q5 = nb[5], q6 = nb[6];
+  V3 sep = v3(0.f, 0.f, 0.f), coh = v3(0.f, 0.f, 0.f), ali = v3(0.f, 0.f, 0.f);
+#pragma unroll 1
+  for (int k = 0; k < cnt; ++k) {
+    const int64_t j = q0;  // nb[k]: the list shifts down one slot per iteration
+    q0 = q1; q1 = q2; q2 = q3; q3 = q4; q4 = q5; q5 = q6;
     float4 pj = __ldg(pos_of(a.full, a.m, a.sdiv, j));
     float4 fj = __ldg(fwd_of(a.full, a.m, a.sdiv, j));
     V3 o = sub(v3(pj), me);  // A.position - me.position (Listing 5.3 line 7)

@@ -1,6 +1,7 @@
 // api.cu -- the C ABI of include/boids.h: handles, buffers, validation, the step
 // loop and host<->device state transfer.  No exception crosses the ABI.
 #include <cmath>
+#include <cstdlib>
 #include <cstring>
 #include <new>
 #include <string>
@@ -69,9 +70,12 @@ struct boids_ctx {
   float* qlim = nullptr;                  // warm path search limits [m]
   float4* sym_sp = nullptr;               // k_sym: agents in spatial order (x, y, z, limit) [sym_capacity]
   int32_t* sym_idx = nullptr;             // k_sym: their local indices [sym_capacity]
+  long long* sym_fb = nullptr;            // k_sym: per-CTA (range, cycles) of the last two launches [2][SYM_FB_LEN]
+  int sym_fb_par = 0;                     // which half the next launch writes
   int32_t* sym_rlist = nullptr;           // k_sym: agents routed to k_route this step [m]
   int32_t* sym_rcount = nullptr;          // ... and their number
   bool symmetric = true;                  // BOIDS_OPT_SYMMETRIC
+  bool balance = true;                    // BOIDS_OPT_BALANCE: k_sym split from the last launch's CTA times
   int32_t* pcnt = nullptr;
   unsigned long long* phase = nullptr;  // diagnostics (BOIDS_OPT_PHASES): per-CTA timestamps
   // grid mode (BOIDS_GRID): search grid and its binning buffers
@@ -184,6 +188,7 @@ void free_ctx(boids_ctx* c) {
   cudaFree(c->phase);
   cudaFree(c->sym_sp);
   cudaFree(c->sym_idx);
+  cudaFree(c->sym_fb);
   cudaFree(c->sym_rlist);
   cudaFree(c->sym_rcount);
   for (auto& r : c->recs) {
@@ -307,7 +312,8 @@ int create_impl(int64_t n, const boids_params* p, uint64_t seed, int32_t rank, i
              (rc = alloc((void**)&c->sym_rlist, m * sizeof(int32_t))) ||
              (rc = alloc((void**)&c->sym_rcount, sizeof(int32_t))) ||
              (!shard && ((rc = alloc((void**)&c->sym_sp, sym_capacity(c->nloc) * sizeof(float4))) ||
-                         (rc = alloc((void**)&c->sym_idx, sym_capacity(c->nloc) * sizeof(int32_t)))))) {
+                         (rc = alloc((void**)&c->sym_idx, sym_capacity(c->nloc) * sizeof(int32_t))) ||
+                         (rc = alloc((void**)&c->sym_fb, 2 * SYM_FB_LEN * sizeof(long long)))))) {
     free_ctx(c);
     return rc;
   }
@@ -317,6 +323,7 @@ int create_impl(int64_t n, const boids_params* p, uint64_t seed, int32_t rank, i
   if (e == cudaSuccess) e = cudaMemsetAsync(c->buf[0], 0, shard ? seg * world : seg, s);
   if (e == cudaSuccess) e = cudaMemsetAsync(c->buf[1], 0, seg, s);
   if (e == cudaSuccess) e = cudaMemsetAsync(c->cnt, 0xFF, m * sizeof(int32_t), s);  // -1: never searched
+  if (e == cudaSuccess && c->sym_fb) e = cudaMemsetAsync(c->sym_fb, 0, 2 * SYM_FB_LEN * sizeof(long long), s);
   if (e == cudaSuccess) e = cudaMemsetAsync(c->fstore, 0, m * sizeof(float4), s);
   if (e == cudaSuccess) e = cudaMemsetAsync(c->routed, 0, m, s);
   if (e == cudaSuccess) e = cudaMemsetAsync(c->nbr, 0xFF, m * 7 * sizeof(int32_t), s);
@@ -484,7 +491,12 @@ int one_step(boids_ctx* c, float dt) {
         StepArgs as = a;
         as.routed = c->routed;  // agents routed to k_route by k_sym_prep (k_select skips them)
         CK(cudaMemsetAsync(c->sym_rcount, 0, sizeof(int32_t), c->stream));
-        if ((rc = launch(c, 0, [&] { return launch_sym_scan(as, c->sym_sp, c->sym_idx, c->stream); }, 2)))
+        long long* fb_prev = c->sym_fb + (c->sym_fb_par ^ 1) * SYM_FB_LEN;
+        long long* fb_cur = c->sym_fb + c->sym_fb_par * SYM_FB_LEN;
+        c->sym_fb_par ^= 1;
+        if ((rc = launch(c, 0, [&] {
+               return launch_sym_scan(as, c->sym_sp, c->sym_idx, c->balance ? fb_prev : nullptr, fb_cur, c->stream);
+             }, 2)))
           return rc;
         if ((rc = launch(c, 1, [&] { return launch_warm_select(as, c->stream); }))) return rc;
         if ((rc = launch(c, 4, [&] { return launch_route(as, c->stream); }))) return rc;
@@ -507,6 +519,18 @@ int one_step(boids_ctx* c, float dt) {
   c->steps_taken++;
   return BOIDS_OK;
 }
+
+}  // namespace
+
+int boids::carveout_pct() {
+  static const int v = [] {
+    const char* e = getenv("BOIDS_CARVEOUT");
+    return e ? atoi(e) : 100;
+  }();
+  return v;
+}
+
+namespace {
 
 int check_dt(float dt) {
   if (!std::isfinite(dt) || dt < 0.f) return fail(BOIDS_EINVAL, "dt must be finite and >= 0");
@@ -580,6 +604,9 @@ BOIDS_API int boids_set_option(boids_ctx* c, int32_t opt, int64_t v) {
       return BOIDS_OK;
     case BOIDS_OPT_SYMMETRIC:
       c->symmetric = v != 0;
+      return BOIDS_OK;
+    case BOIDS_OPT_BALANCE:
+      c->balance = v != 0;
       return BOIDS_OK;
     case BOIDS_OPT_VOTE_U:
       if (v != 4 && v != 8) return fail(BOIDS_EINVAL, "vote width must be 4 or 8");

@@ -106,6 +106,28 @@ __device__ __forceinline__ void merge7(key_t (&A)[7], const key_t (&B)[7]) {
   for (int s = 0; s < 7; ++s) A[s] = S[s + 1];
 }
 
+// A := the 8 smallest keys of A u B, ascending (half-cleaner + 8-wide bitonic merge).
+__device__ __forceinline__ void merge8(key_t (&A)[8], const key_t (&B)[8]) {
+  key_t S[8];
+#pragma unroll
+  for (int s = 0; s < 8; ++s) S[s] = A[s] < B[7 - s] ? A[s] : B[7 - s];
+#pragma unroll
+  for (int i = 0; i < 4; ++i) cex(S[i], S[i + 4]);
+  cex(S[0], S[2]); cex(S[1], S[3]); cex(S[4], S[6]); cex(S[5], S[7]);
+  cex(S[0], S[1]); cex(S[2], S[3]); cex(S[4], S[5]); cex(S[6], S[7]);
+#pragma unroll
+  for (int s = 0; s < 8; ++s) A[s] = S[s];
+}
+__device__ __forceinline__ void insert8(key_t (&L)[8], key_t k) {
+#pragma unroll
+  for (int s = 7; s >= 1; --s) {
+    const key_t x = L[s - 1];
+    const key_t y = L[s] < k ? L[s] : k;
+    L[s] = k < x ? x : y;
+  }
+  L[0] = L[0] < k ? L[0] : k;
+}
+
 // ---- Appendix B: SplitMix64 streams --------------------------------------
 constexpr uint64_t SM64_GAMMA = 0x9E3779B97F4A7C15ull;
 __host__ __device__ __forceinline__ uint64_t sm64_mix(uint64_t z) {

@@ -127,6 +127,21 @@ struct GridArgs {
 // Does global agent g think at step t (think frequency k)?
 __host__ __device__ inline bool thinks(int64_t g, int64_t t, int32_t k) { return k <= 1 || (g + t) % k == 0; }
 
+// Every kernel of a step asks for the same L1/shared-memory split (the maximum
+// shared-memory carveout the TMA-ring kernels need), so consecutive kernels do
+// not make the SMs drain and reconfigure the split between launches.  Once per
+// kernel; BOIDS_CARVEOUT=<percent> overrides, -1 leaves the driver default.
+int carveout_pct();
+#define BOIDS_PREFER_SMEM(kern)                                                                  \
+  do {                                                                                           \
+    static const bool boids_once_ = [] {                                                         \
+      if (carveout_pct() >= 0)                                                                   \
+        cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, carveout_pct()); \
+      return true;                                                                               \
+    }();                                                                                         \
+    (void)boids_once_;                                                                           \
+  } while (0)
+
 // launchers (return the cudaError_t of the launch)
 cudaError_t launch_init(float4* out, float4* up4, float4* side4, int64_t m, int64_t lo,
                         int64_t nloc, const boids_params& p, uint64_t seed, cudaStream_t s);
@@ -157,7 +172,12 @@ cudaError_t launch_grid_far(const StepArgs& a, const GridArgs& g, cudaStream_t s
 int grid_chunk();
 cudaError_t launch_warm_select(const StepArgs& a, cudaStream_t s);
 int64_t sym_capacity(int64_t nloc);
-cudaError_t launch_sym_scan(const StepArgs& a, float4* sp, int* sidx, cudaStream_t s);
+// k_sym work-split feedback record: [0] grid, [1] items, then per CTA j
+// [2 + 3j] L0, [3 + 3j] L1, [4 + 3j] SM cycles the CTA took.
+constexpr int SYM_FB_MAX_CTAS = 1024;
+constexpr int SYM_FB_LEN = 2 + 3 * SYM_FB_MAX_CTAS;
+cudaError_t launch_sym_scan(const StepArgs& a, float4* sp, int* sidx, const long long* fb_prev, long long* fb_cur,
+                            cudaStream_t s);
 cudaError_t launch_route(const StepArgs& a, cudaStream_t s);
 int fused_auto_cluster(int64_t n_pad_total, int64_t nloc, int sm_count);
 

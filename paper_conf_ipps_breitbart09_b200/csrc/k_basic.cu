@@ -222,6 +222,7 @@ __global__ void __launch_bounds__(256) k_apply(StepArgs a) {
 
 cudaError_t launch_apply(const StepArgs& a, cudaStream_t s) {
   if (a.nloc <= 0) return cudaSuccess;
+  BOIDS_PREFER_SMEM(k_apply);
   k_apply<<<(unsigned)((a.nloc + 255) / 256), 256, 0, s>>>(a);
   return cudaGetLastError();
 }
@@ -271,12 +272,14 @@ __global__ void __launch_bounds__(1024) k_think_compact(StepArgs a, const int32_
 cudaError_t launch_think_compact(const StepArgs& a, const int32_t* qperm, int32_t* cold, int32_t* ncold,
                                  int32_t* warm, int32_t* nwarm, cudaStream_t s) {
   if (a.nloc <= 0) return cudaSuccess;
+  BOIDS_PREFER_SMEM(k_think_compact);
   k_think_compact<<<(unsigned)((a.nloc + 1023) / 1024), 1024, 0, s>>>(a, qperm, cold, ncold, warm, nwarm);
   return cudaGetLastError();
 }
 
 cudaError_t launch_update(const StepArgs& a, cudaStream_t s) {
   if (a.nloc <= 0) return cudaSuccess;
+  BOIDS_PREFER_SMEM(k_update);
   k_update<<<(unsigned)((a.nloc + 255) / 256), 256, 0, s>>>(a);
   return cudaGetLastError();
 }

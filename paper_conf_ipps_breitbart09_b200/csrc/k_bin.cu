@@ -215,6 +215,9 @@ cudaError_t launch_bin(const float4* full, int64_t m, const SliceDiv& sd, int64_
     k_bin_scan<<<1, SCAN_T, shm, s>>>(cnt, start, g.cells, items, nitems, chunk, counter, g.dim[0]);
     return cudaGetLastError();
   }
+  BOIDS_PREFER_SMEM(k_bin_count);
+  BOIDS_PREFER_SMEM(k_bin_scatter);
+  BOIDS_PREFER_SMEM(k_bin_scan);
   k_bin_count<<<blocks, 256, 0, s>>>(full, m, sd, j0, count, g, cellrank, cnt, spos == nullptr,
                                      spos == nullptr ? think_k : 1, think_t);
   cudaError_t e = cudaGetLastError();

@@ -379,6 +379,7 @@ cudaError_t launch_grid_far(const StepArgs& a, const GridArgs& g, cudaStream_t s
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  BOIDS_PREFER_SMEM(k_grid_far);
   k_grid_far<<<(unsigned)(4 * sms), FT, 0, s>>>(a, g);
   return cudaGetLastError();
 }

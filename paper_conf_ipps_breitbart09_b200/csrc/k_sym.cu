@@ -148,6 +148,58 @@ __device__ __forceinline__ int64_t sym_split(int64_t i, int64_t grid, int64_t np
   return (sym_prefix(lo, npad, qb) + off) / U * U;
 }
 
+// Feedback split (BOIDS_OPT_BALANCE).  The cost of an item is not uniform: the
+// slow path (passing pairs) concentrates where queries and candidates are near
+// each other in space -- on and next to the diagonal of a spatially sorted flock
+// -- and its weight depends on the flock's density.  The previous launch measured
+// every CTA's SM time for its range [L0_j, L1_j); read as a piecewise-constant
+// cost density over the item space, it gives a cumulative cost C(x), and CTA i
+// takes [C^-1(i T / G), C^-1((i + 1) T / G)), T = C(total), rounded to U.  The
+// flock moves little per step, so the density carries over.  Every CTA computes
+// the same boundaries from the same record, so the ranges tile the item space
+// exactly; only the partition changes, never a result.  Returns false (static
+// split) when the record is missing or from another launch shape.  Warp 0 only.
+__device__ bool fb_split(const long long* fb, int G, int64_t total, int i, int lane, int64_t& l0, int64_t& l1) {
+  if (fb == nullptr || G > SYM_FB_MAX_CTAS || fb[0] != G || fb[1] != total) return false;
+  const int per = (G + 31) / 32, j0 = min(G, lane * per), j1 = min(G, j0 + per);
+  double own = 0.0;
+  for (int j = j0; j < j1; ++j) own += (double)fb[4 + 3 * j];
+  double incl = own;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const double v = __shfl_up_sync(0xffffffffu, incl, o);
+    if (lane >= o) incl += v;
+  }
+  const double T = __shfl_sync(0xffffffffu, incl, 31), excl = incl - own;
+  if (!(T > 0.0)) return false;
+  auto bound = [&](int k) -> int64_t {
+    if (k <= 0) return 0;
+    if (k >= G) return total;
+    const double c = T * (double)k / (double)G;
+    const unsigned owner = __ballot_sync(0xffffffffu, j1 > j0 && excl <= c && c < incl);
+    const int src = owner ? __ffs(owner) - 1 : 31;
+    int64_t x = total;
+    if (lane == src) {
+      double cum = excl;
+      for (int j = j0; j < j1; ++j) {
+        const double t = (double)fb[4 + 3 * j];
+        if (c < cum + t) {
+          const int64_t a0 = fb[2 + 3 * j], a1 = fb[3 + 3 * j];
+          x = a0 + (int64_t)((c - cum) / t * (double)(a1 - a0));
+          break;
+        }
+        cum += t;
+      }
+    }
+    x = __shfl_sync(0xffffffffu, x, src);
+    x = x / U * U;
+    return x < 0 ? 0 : (x > total ? total : x);
+  };
+  l0 = bound(i);
+  l1 = bound(i + 1);
+  return true;
+}
+
 // Tile k of a CTA whose item range is [L0, L1): items [max(L0, A + k*CT), min(L1,
 // A + (k+1)*CT)) with A = L0 rounded down to CT.  Rows (npad - b*QB items) and
 // their starts S(b) are multiples of CT, so a tile never straddles two rows.
@@ -170,12 +222,28 @@ __device__ __forceinline__ TileDesc tile_desc(int k, int64_t L0, int64_t L1, int
 
 template <int NTS>
 __global__ void __launch_bounds__(NTS, NTS == 128 ? 4 : 1)
-    k_sym(StepArgs a, const float4* __restrict__ sp, const int* __restrict__ sidx, int64_t npad, int wd4) {
+    k_sym(StepArgs a, const float4* __restrict__ sp, const int* __restrict__ sidx, int64_t npad, int wd4,
+          const long long* __restrict__ fb_prev, long long* __restrict__ fb_cur) {
   constexpr int QBS = NTS * Q, NW = NTS / 32;
   extern __shared__ __align__(16) unsigned char smem_raw[];
   SymSmem<NTS>& sm = *reinterpret_cast<SymSmem<NTS>*>(smem_raw);
+  __shared__ int64_t s_range[2];
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-  const int64_t L0 = sym_split(blockIdx.x, gridDim.x, npad, QBS, wd4), L1 = sym_split(blockIdx.x + 1, gridDim.x, npad, QBS, wd4);
+  const long long c_start = clock64();
+  const int64_t total = sym_prefix(npad / QBS, npad, QBS);
+  if (warp == 0) {
+    int64_t l0, l1;
+    if (!fb_split(fb_prev, (int)gridDim.x, total, (int)blockIdx.x, lane, l0, l1)) {
+      l0 = sym_split(blockIdx.x, gridDim.x, npad, QBS, wd4);
+      l1 = sym_split(blockIdx.x + 1, gridDim.x, npad, QBS, wd4);
+    }
+    if (lane == 0) {
+      s_range[0] = l0;
+      s_range[1] = l1;
+    }
+  }
+  __syncthreads();
+  const int64_t L0 = s_range[0], L1 = s_range[1];
   const int ntiles = L1 > L0 ? (int)((L1 + CT - 1) / CT - L0 / CT) : 0;
   // Ring protocol: stage s = k % STAGES holds tile k.  full[s] completes when the
   // tile's bytes land (TMA complete_tx).  Each warp, when done with tile k,
@@ -314,6 +382,18 @@ __global__ void __launch_bounds__(NTS, NTS == 128 ? 4 : 1)
   }
   __syncwarp();
   flush(a, rec, wcount, lane);
+  if (fb_cur) {  // this CTA's range and SM time: the next launch's split (fb_split)
+    __syncthreads();
+    if (tid == 0) {
+      fb_cur[2 + 3 * blockIdx.x] = L0;
+      fb_cur[3 + 3 * blockIdx.x] = L1;
+      fb_cur[4 + 3 * blockIdx.x] = clock64() - c_start;
+      if (blockIdx.x == 0) {
+        fb_cur[0] = gridDim.x;
+        fb_cur[1] = total;
+      }
+    }
+  }
   if (a.stats && lane == 0) {
     atomicAdd(a.stats, (unsigned long long)slow_groups);
     atomicAdd(a.stats + 1, (unsigned long long)groups);
@@ -361,8 +441,8 @@ __device__ __forceinline__ float sym_t0(const StepArgs& a, int64_t qi, float4 me
 // full previous list: it wrapped to the far side of the world) would append
 // every in-radius pair -- hundreds -- to its hit buffer.  It is ROUTED instead:
 // limit -1 (no hits on either side in k_sym) and searched whole by k_route.
-__global__ void __launch_bounds__(256) k_sym_prep(StepArgs a, float4* __restrict__ sp, int* __restrict__ sidx,
-                                                   int64_t npad) {
+__device__ __forceinline__ void sym_prep_body(const StepArgs& a, float4* __restrict__ sp, int* __restrict__ sidx,
+                                              int64_t npad) {
   const int64_t p = (int64_t)blockIdx.x * 256 + threadIdx.x;
   if (p >= npad) return;
   if (p >= a.nloc) {
@@ -387,26 +467,11 @@ __global__ void __launch_bounds__(256) k_sym_prep(StepArgs a, float4* __restrict
   sidx[p] = qi;
 }
 
-// A := the 8 smallest keys of A u B, ascending (half-cleaner + 8-wide bitonic merge).
-__device__ __forceinline__ void merge8(key_t (&A)[8], const key_t (&B)[8]) {
-  key_t S[8];
-#pragma unroll
-  for (int s = 0; s < 8; ++s) S[s] = A[s] < B[7 - s] ? A[s] : B[7 - s];
-#pragma unroll
-  for (int i = 0; i < 4; ++i) cex(S[i], S[i + 4]);
-  cex(S[0], S[2]); cex(S[1], S[3]); cex(S[4], S[6]); cex(S[5], S[7]);
-  cex(S[0], S[1]); cex(S[2], S[3]); cex(S[4], S[5]); cex(S[6], S[7]);
-#pragma unroll
-  for (int s = 0; s < 8; ++s) A[s] = S[s];
-}
-__device__ __forceinline__ void insert8(key_t (&L)[8], key_t k) {
-#pragma unroll
-  for (int s = 7; s >= 1; --s) {
-    const key_t x = L[s - 1];
-    const key_t y = L[s] < k ? L[s] : k;
-    L[s] = k < x ? x : y;
-  }
-  L[0] = L[0] < k ? L[0] : k;
+__global__ void __launch_bounds__(256) k_sym_prep(StepArgs a, float4* __restrict__ sp, int* __restrict__ sidx,
+                                                   int64_t npad) {
+  span_begin(a, SPAN_SLOT0 + 0);
+  sym_prep_body(a, sp, sidx, npad);
+  span_end(a, SPAN_SLOT0 + 0);
 }
 
 // Routed agents (k_sym_prep): one CTA per agent searches all candidates (Listing
@@ -415,7 +480,7 @@ __device__ __forceinline__ void insert8(key_t (&L)[8], key_t k) {
 // them.  The CTA then finishes the agent -- list, 8th nearest (the next step's
 // warm-bound seed), steering, modification -- and k_select skips it.
 constexpr int RT = 512, RU = 16;
-__global__ void __launch_bounds__(RT) k_route(StepArgs a) {
+__device__ __forceinline__ void route_body(const StepArgs& a) {
   __shared__ key_t wl[RT / 32][8];
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int nr = *a.rcount;
@@ -489,6 +554,12 @@ __global__ void __launch_bounds__(RT) k_route(StepArgs a) {
   }
 }
 
+__global__ void __launch_bounds__(RT) k_route(StepArgs a) {
+  span_begin(a, SPAN_SLOT0 + 2);
+  route_body(a);
+  span_end(a, SPAN_SLOT0 + 2);
+}
+
 template <int NT>
 int sym_grid(int sms) {
   static int grid = 0;
@@ -503,9 +574,11 @@ int sym_grid(int sms) {
 }
 
 template <int NT>
-cudaError_t sym_with(const StepArgs& a, float4* sp, int* sidx, int sms, cudaStream_t s) {
+cudaError_t sym_with(const StepArgs& a, float4* sp, int* sidx, const long long* fb_prev, long long* fb_cur, int sms,
+                     cudaStream_t s) {
   constexpr int64_t QBS = NT * Q;
   const int64_t npad = (a.nloc + QBS - 1) / QBS * QBS;
+  BOIDS_PREFER_SMEM(k_sym_prep);
   k_sym_prep<<<(unsigned)((npad + 255) / 256), 256, 0, s>>>(a, sp, sidx, npad);
   if (cudaError_t e = cudaGetLastError()) return e;
   const int64_t nb = npad / QBS;
@@ -515,7 +588,7 @@ cudaError_t sym_with(const StepArgs& a, float4* sp, int* sidx, int sms, cudaStre
     const char* e = getenv("BOIDS_SYM_WD4");  // diagnostics: diagonal item weight x4
     return e ? atoi(e) : 6;  // measured best of 4..16 at C3 and C4
   }();
-  k_sym<NT><<<g, NT, sizeof(SymSmem<NT>), s>>>(a, sp, sidx, npad, wd4);
+  k_sym<NT><<<g, NT, sizeof(SymSmem<NT>), s>>>(a, sp, sidx, npad, wd4, fb_prev, g <= SYM_FB_MAX_CTAS ? fb_cur : nullptr);
   return cudaGetLastError();
 }
 
@@ -534,11 +607,13 @@ cudaError_t launch_route(const StepArgs& a, cudaStream_t s) {
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  BOIDS_PREFER_SMEM(k_route);
   k_route<<<(unsigned)std::min<int64_t>(a.nloc, 2LL * sms), RT, 0, s>>>(a);
   return cudaGetLastError();
 }
 
-cudaError_t launch_sym_scan(const StepArgs& a, float4* sp, int* sidx, cudaStream_t s) {
+cudaError_t launch_sym_scan(const StepArgs& a, float4* sp, int* sidx, const long long* fb_prev, long long* fb_cur,
+                            cudaStream_t s) {
   if (a.nloc <= 0) return cudaSuccess;
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
@@ -550,8 +625,8 @@ cudaError_t launch_sym_scan(const StepArgs& a, float4* sp, int* sidx, cudaStream
     const char* e = getenv("BOIDS_SYM_NT");  // diagnostics: force a CTA shape (128 or 512)
     return e ? atoi(e) : 0;
   }();
-  if (force == 512 || (force != 128 && tiles512 >= 2LL * sms)) return sym_with<512>(a, sp, sidx, sms, s);
-  return sym_with<128>(a, sp, sidx, sms, s);
+  if (force == 512 || (force != 128 && tiles512 >= 2LL * sms)) return sym_with<512>(a, sp, sidx, fb_prev, fb_cur, sms, s);
+  return sym_with<128>(a, sp, sidx, fb_prev, fb_cur, sms, s);
 }
 
 }  // namespace boids

@@ -197,6 +197,25 @@ def test_config_full_multi_step(pk, orc, cfg):
             assert bitexact(f.state(), o)
 
 
+@pytest.mark.parametrize("balance", [1, 0])
+def test_config_c3_feedback_split(pk, orc, balance):
+    """C3 (the north_star's n = 16384 brute-force case) for 12 steps: from the
+    second warm step on, k_sym cuts its work from the previous launch's measured
+    CTA times (BOIDS_OPT_BALANCE = 1), so the partition changes every step.  The
+    lists and states stay bit-exact with the oracle either way."""
+    c = W.CONFIGS["c3"]
+    p = pk.boids_default_params(init_mode=c.init_mode)
+    with pk.Flock(c.n, p, seed=1) as f:
+        from paper_conf_ipps_breitbart09_b200 import abi
+        abi.boids_set_option(f.h, abi.BOIDS_OPT_BALANCE, balance)
+        o = orc.init(c.n, _oparams(orc, p), seed=1)
+        for t in range(12):
+            o, o_idx, _, _ = orc.step(o, DT, _oparams(orc, p))
+            f.step(DT, 1)
+            np.testing.assert_array_equal(f.neighbors()[0], o_idx, err_msg=f"step {t}")
+            assert bitexact(f.state(), o), f"step {t}"
+
+
 def test_config_c4_sampled(pk, orc):
     """C4 (n=131072, WORLD init) at full size: GPU runs 2 steps from init in the
     bench's launch configuration; the oracle checks a seeded sample of agents of
