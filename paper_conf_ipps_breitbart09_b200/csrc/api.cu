@@ -391,6 +391,8 @@ StepArgs make_args(boids_ctx* c, float dt) {
   a.routed = c->p.think_every > 1 ? c->routed : nullptr;
   a.rlist = c->sym_rlist;  // warm brute-force steps route overflowed agents to k_route
   a.rcount = c->sym_rcount;
+  a.loc = c->loc_grid;
+  a.lstart = c->bstart;  // brute-force steps sort the queries (qperm) before any search
   return a;
 }
 

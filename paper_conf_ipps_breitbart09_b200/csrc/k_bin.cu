@@ -15,31 +15,9 @@
 // (sorted query blocks and candidate stream -> spatially coherent warps, far
 // fewer insertion-path entries; every pair is still evaluated) and the
 // search grid of BOIDS_GRID (cells >= r, see k_grid.cu).
-#include "internal.h"
+#include "cells.cuh"
 
 namespace boids {
-
-__device__ __forceinline__ uint32_t spread3(uint32_t x) {  // 10 bits -> every 3rd bit
-  x &= 0x3ff;
-  x = (x | (x << 16)) & 0x030000FF;
-  x = (x | (x << 8)) & 0x0300F00F;
-  x = (x | (x << 4)) & 0x030C30C3;
-  x = (x | (x << 2)) & 0x09249249;
-  return x;
-}
-
-__device__ __forceinline__ int cell_coord(float v, const BinGrid& g, int d) {
-  // floor((v - lo) * inv_h), clamped into [0, dim-1]; NaN handled by the caller
-  float t = (v - g.lo[d]) * g.inv_h;
-  int c = (int)floorf(t);
-  return c < 0 ? 0 : (c >= g.dim[d] ? g.dim[d] - 1 : c);
-}
-
-__device__ __forceinline__ int cell_of(float4 p, const BinGrid& g) {
-  int ix = cell_coord(p.x, g, 0), iy = cell_coord(p.y, g, 1), iz = cell_coord(p.z, g, 2);
-  if (g.morton) return (int)(spread3(ix) | (spread3(iy) << 1) | (spread3(iz) << 2));
-  return (iz * g.dim[1] + iy) * g.dim[0] + ix;
-}
 
 // Agents j in [j0, j0 + count) of the segmented buffer `full`.
 // keep_nan: bin agents with a NaN position into cell 0 (query binning: every

@@ -55,6 +55,46 @@ struct __align__(16) GridSmem {
   int nfar;              // queries that need more (routed to k_grid_far when few)
 };
 
+// A bound for a query whose warm bound reaches past the adjacent cells (a cold
+// step, an agent that wrapped to the diametric opposite point, or whose
+// neighbours did): the 7th smallest d2 to the other agents of its own cell,
+// which the binning of THIS step put together (current positions).  Real,
+// distinct agents, so an upper bound on the 7th key like t0; +inf with fewer
+// than 7.  It usually brings the query back within the adjacent cells, so it
+// is searched in its item instead of by k_grid_far.
+__device__ float cell_bound(const GridArgs& g, float4 me, int gi) {
+  auto coord = [&](float v, int d) {
+    const int c = (int)floorf((v - g.grid.lo[d]) * g.grid.inv_h);
+    return c < 0 ? 0 : (c >= g.grid.dim[d] ? g.grid.dim[d] - 1 : c);
+  };
+  float b[7];
+#pragma unroll
+  for (int k = 0; k < 7; ++k) b[k] = __int_as_float(0x7f800000);
+  if (!(me.x == me.x && me.y == me.y && me.z == me.z)) return b[6];
+  const int cell = (coord(me.z, 2) * g.grid.dim[1] + coord(me.y, 1)) * g.grid.dim[0] + coord(me.x, 0);
+  const int lo = __ldg(g.cstart + cell), hi = __ldg(g.cstart + cell + 1);
+  constexpr int G = 16;  // loads in flight
+  for (int k0 = lo; k0 < hi; k0 += G) {
+    float4 c[G];
+#pragma unroll
+    for (int k = 0; k < G; ++k)
+      c[k] = k0 + k < hi ? __ldg(g.spos + k0 + k) : make_float4(__int_as_float(0x7fc00000), 0.f, 0.f, 0.f);
+#pragma unroll
+    for (int k = 0; k < G; ++k) {
+      if (__float_as_int(c[k].w) == gi) continue;
+      float d = dist2(me.x, me.y, me.z, c[k]);
+      if (!(d == d)) continue;
+#pragma unroll
+      for (int t = 0; t < 7; ++t) {  // keep the 7 smallest, ascending
+        const float l = fminf(b[t], d);
+        d = fmaxf(b[t], d);
+        b[t] = l;
+      }
+    }
+  }
+  return b[6];
+}
+
 __device__ __forceinline__ int tile_count(const GridSmem& sm, int r, int off) {
   return min(CT, sm.range[r].y - (sm.range[r].x + off));
 }
@@ -132,6 +172,8 @@ __global__ void __launch_bounds__(NTG) k_grid(StepArgs a, GridArgs g) {
       pxy[q] = make_float2(me.x, me.y);
       pz[q] = me.z;
       lim[q] = fminf(r2_in, a.warm ? warm_bound(a, qi, me) : __int_as_float(0x7f800000));
+      if (qi < a.nloc && sqrtf(lim[q]) * g.grid.inv_h * (1.0f + 1.0f / 1024.0f) >= 1.0f)
+        lim[q] = fminf(lim[q], cell_bound(g, me, gq[q]));
 #pragma unroll
       for (int s = 0; s < 7; ++s) sm.lists[s * QBG + slot] = KEY_EMPTY;
     }
@@ -313,7 +355,8 @@ __global__ void __launch_bounds__(FT) k_grid_far(StepArgs a, GridArgs g) {
     const int qi = g.flist[f];
     const float4 me = __ldg(pos_of(a.full, a.m, a.sdiv, a.lo + qi));
     const int gi = (int)(a.lo + qi);
-    const float lim = fminf(r2_in, a.warm ? warm_bound(a, qi, me) : __int_as_float(0x7f800000));
+    const float lim = fminf(fminf(r2_in, a.warm ? warm_bound(a, qi, me) : __int_as_float(0x7f800000)),
+                            cell_bound(g, me, gi));
     if (tid == 0) {
       const int Rg = g.grid.reach;
       const float cells = sqrtf(lim) * g.grid.inv_h * (1.0f + 1.0f / 1024.0f);

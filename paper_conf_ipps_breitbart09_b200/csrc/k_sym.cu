@@ -24,6 +24,7 @@
 // Stream-K: the triangular item space sum_b (npad - b*QB) is cut into equal
 // contiguous ranges per CTA, as in k_scan.  Candidates and their original
 // indices stream through a TMA ring (cp.async.bulk + mbarrier).
+#include "cells.cuh"
 #include "step_common.cuh"
 #include "tma.cuh"
 
@@ -436,6 +437,50 @@ __device__ __forceinline__ float sym_t0(const StepArgs& a, int64_t qi, float4 me
   return nb[7] >= 0 ? m2 : m1;
 }
 
+// A second bound for an agent whose previous neighbours no longer bound it (t0
+// > r2: it wrapped to the diametric opposite point, or its neighbours
+// did): the 7th smallest current d2 to the agents around its cell in the
+// last spatial sort (WIN of them; qperm is in Morton order of the locality grid; lstart the
+// cells' starts), self excluded.  They are real, distinct agents, so it is an
+// upper bound on the 7th key like t0; +inf with fewer than 7 of them.  The
+// sort is up to BOIDS_OPT_RESORT steps old: only the bound's tightness depends
+// on that, never the result.
+constexpr int WIN = 64;
+__device__ float window_bound(const StepArgs& a, int qi, float4 me) {
+  const int n = (int)a.nloc;
+  if (!a.lstart || !a.qperm || n < 8 || !(me.x == me.x && me.y == me.y && me.z == me.z))
+    return __int_as_float(0x7f800000);
+  const int p0 = __ldg(a.lstart + cell_of(me, a.loc));
+  int lo = p0 - WIN / 2;
+  lo = lo > n - WIN ? n - WIN : lo;
+  lo = lo < 0 ? 0 : lo;
+  const int hi = lo + WIN < n ? lo + WIN : n;
+  float b[7];
+#pragma unroll
+  for (int k = 0; k < 7; ++k) b[k] = __int_as_float(0x7f800000);
+  constexpr int G = 16;  // loads in flight: the agents that take this path are scattered
+  for (int p0 = lo; p0 < hi; p0 += G) {
+    int j[G];
+#pragma unroll
+    for (int k = 0; k < G; ++k) j[k] = p0 + k < hi ? __ldg(a.qperm + p0 + k) : -1;
+    float4 q[G];
+#pragma unroll
+    for (int k = 0; k < G; ++k) q[k] = __ldg(pos_of(a.full, a.m, a.sdiv, a.lo + (j[k] < 0 ? 0 : j[k])));
+#pragma unroll
+    for (int k = 0; k < G; ++k) {
+      if (j[k] < 0 || j[k] == qi) continue;
+      float d = dist2(me.x, me.y, me.z, q[k]);
+#pragma unroll
+      for (int t = 0; t < 7; ++t) {  // keep the 7 smallest, ascending
+        const float lo_ = fminf(b[t], d);
+        d = fmaxf(b[t], d);
+        b[t] = lo_;
+      }
+    }
+  }
+  return b[6];
+}
+
 // sp[p] = (x, y, z, min(prev(r2), t0)) of agent sidx[p] = qperm[p]; phantoms beyond nloc.
 // An agent whose previous 7 neighbours are all out of range now (t0 >= r2 with a
 // full previous list: it wrapped to the far side of the world) would append
@@ -457,7 +502,8 @@ __device__ __forceinline__ void sym_prep_body(const StepArgs& a, float4* __restr
   int c = 0;
   const float t0 = sym_t0(a, qi, me, c);
   float lim = fminf(r2_in, t0);
-  if (c == 7 && t0 > r2_in && a.rlist) {
+  if (t0 > r2_in) lim = fminf(lim, window_bound(a, qi, me));
+  if (c == 7 && lim > r2_in && a.rlist) {
     a.rlist[atomicAdd(a.rcount, 1)] = qi;
     a.routed[qi] = 1;
     if (a.stats) atomicAdd(a.stats + 2, 1ull);

@@ -572,6 +572,7 @@ __device__ __forceinline__ void select4_body(const StepArgs& a) {
   const int64_t qi = wbase + lane;
   if (qi >= a.nloc) return;
   if (my_over) {  // overflowed buffer: k_route searches the agent whole after this kernel
+    if (a.stats) atomicAdd(a.stats + 2, 1ull);
     a.rlist[atomicAdd(a.rcount, 1)] = (int)qi;
     a.hitcnt[qi] = 0;
     a.pcnt[qi] = 0;
