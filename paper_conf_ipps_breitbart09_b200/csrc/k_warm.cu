@@ -491,87 +491,28 @@ __global__ void __launch_bounds__(NSEL) k_select(StepArgs a) {
   modify_agent(a, qi, v3(p4), f4, F);
 }
 
-// k_select for warm steps without think frequency (routing on).  A warp owns 32
-// agents, one per lane, and works in two phases:
-//  1. merge, SL lanes per agent (32 / SL agents per round): the lanes split the
-//     agent's hit buffer and partial lists, each keeps the 8 smallest keys, a
-//     shuffle butterfly over the SL lanes gives the agent's 8 smallest keys --
-//     the top-7 list (reading Q4) and the 8th nearest (the next step's
-//     warm-bound seed) -- which the owner lane collects;
-//  2. every lane steers and modifies its own agent.
-// Same lists and state as k_select: phase 1 hides the latency of the hit loads
-// one thread per agent walks serially; phase 2 keeps all 32 lanes on the
-// division- and square-root-heavy arithmetic.
-constexpr int SL = 4;
-__device__ __forceinline__ void select4_body(const StepArgs& a) {
-  const int lane = threadIdx.x & 31, sub = lane & (SL - 1);
-  const int64_t wbase = ((int64_t)blockIdx.x * NSEL + (threadIdx.x & ~31));  // first agent of this warp
-  key_t mine[8];
-#pragma unroll
-  for (int s = 0; s < 8; ++s) mine[s] = KEY_EMPTY;
-  bool my_over = false, my_routed = false;
-  // prefetch every line the four rounds read (lane sub: line sub of each agent's
-  // hit buffer, 4 x 16 keys >= HITS); the rounds themselves stay rolled, because
-  // at small n a warp's time goes to fetching instructions it runs only once
-#pragma unroll
-  for (int r = 0; r < SL; ++r) {
-    const int64_t qi = wbase + r * (32 / SL) + lane / SL;
-    if (qi < a.nloc && sub * 16 < a.hits_cap) prefetch_l1(a.hits + qi * a.hits_cap + sub * 16);
-  }
-#pragma unroll 1
-  for (int r = 0; r < SL; ++r) {
-    const int owner = r * (32 / SL) + lane / SL;  // lane that owns the agent this lane merges for
-    const int64_t qi = wbase + owner;
-    const bool valid = qi < a.nloc;
-    const bool routed = valid && a.routed && a.routed[qi];
-    const int c = valid ? a.hitcnt[qi] : 0;  // a routed agent has no hits
-    const int pc = valid ? a.pcnt[qi] : 0;
-    const bool active = valid && !routed;
-    const bool over = active && (c > a.hits_cap || pc > PSLOTS);
-    key_t L[8];
-#pragma unroll
-    for (int s = 0; s < 8; ++s) L[s] = KEY_EMPTY;
-    if (active && !over) {
-      const key_t* h = a.hits + qi * a.hits_cap;
-      int k = sub;
-      for (; k + SL < c; k += 2 * SL) {  // 2 loads in flight per lane
-        const key_t h0 = h[k], h1 = h[k + SL];
-        insert8(L, h0);
-        insert8(L, h1);
-      }
-      if (k < c) insert8(L, h[k]);
-      for (int p = sub; p < pc; p += SL) {  // rare: partial lists of unbounded agents (k_scan)
-        key_t B[8];
-#pragma unroll
-        for (int s = 0; s < 7; ++s) B[s] = a.partial[(qi * PSLOTS + p) * 7 + s];
-        B[7] = KEY_EMPTY;
-        merge8(L, B);
-      }
-    }
-#pragma unroll
-    for (int w = 1; w < SL; w <<= 1) {
-      key_t B[8];
-#pragma unroll
-      for (int s = 0; s < 8; ++s) B[s] = __shfl_xor_sync(0xffffffffu, L[s], w);
-      merge8(L, B);
-    }
-    // lane r*(32/SL) + g collects group g's result (from its lane g*SL)
-    const bool take = lane / (32 / SL) == r;
-    const int src = (lane % (32 / SL)) * SL;
-#pragma unroll
-    for (int s = 0; s < 8; ++s) {
-      const key_t v = __shfl_sync(0xffffffffu, L[s], src);
-      if (take) mine[s] = v;
-    }
-    const bool o = __shfl_sync(0xffffffffu, over, src), rt = __shfl_sync(0xffffffffu, routed, src);
-    if (take) {
-      my_over = o;
-      my_routed = rt;
-    }
-  }
-  const int64_t qi = wbase + lane;
+// k_select for warm steps without think frequency (routing on): one agent per
+// lane.  Its hit-buffer lines are prefetched into L1 before anything waits on
+// a load, the hits are inserted into a sorted top-8 (the 7-list of reading Q4
+// and the 8th nearest that seeds the next step's warm bound), then the lane
+// steers and modifies the agent.  Same lists and state as k_select; at small
+// n this kernel is one warp per SM sub-partition and pure latency, so what
+// counts is the length of its dependent chain, not its throughput.
+__device__ __forceinline__ void select1_body(const StepArgs& a) {
+  const int64_t qi = (int64_t)blockIdx.x * NSEL + threadIdx.x;
   if (qi >= a.nloc) return;
-  if (my_over) {  // overflowed buffer: k_route searches the agent whole after this kernel
+  const key_t* h = a.hits + qi * a.hits_cap;
+  prefetch_l1(h);
+  prefetch_l1(h + 16);
+  const bool routed = a.routed && a.routed[qi];
+  const int c = a.hitcnt[qi];  // a routed agent has no hits
+  const int pc = a.pcnt[qi];
+  if (routed) {  // routed by k_sym_prep: finished by k_route
+    a.routed[qi] = 0;
+    a.nbr8[qi] = -1;
+    return;
+  }
+  if (c > a.hits_cap || pc > PSLOTS) {  // overflowed buffer: k_route searches the agent whole after this kernel
     if (a.stats) atomicAdd(a.stats + 2, 1ull);
     a.rlist[atomicAdd(a.rcount, 1)] = (int)qi;
     a.hitcnt[qi] = 0;
@@ -579,19 +520,33 @@ __device__ __forceinline__ void select4_body(const StepArgs& a) {
     a.nbr8[qi] = -1;
     return;
   }
-  if (my_routed) {  // routed by k_sym_prep: finished by k_route
-    a.routed[qi] = 0;
-    a.nbr8[qi] = -1;
-    return;
+  key_t L[8];
+#pragma unroll
+  for (int s = 0; s < 8; ++s) L[s] = KEY_EMPTY;
+  int k = 0;
+  for (; k + 3 < c; k += 4) {  // 4 loads in flight
+    const key_t h0 = h[k], h1 = h[k + 1], h2 = h[k + 2], h3 = h[k + 3];
+    insert8(L, h0);
+    insert8(L, h1);
+    insert8(L, h2);
+    insert8(L, h3);
+  }
+  for (; k < c; ++k) insert8(L, h[k]);
+  for (int p = 0; p < pc; ++p) {  // rare: partial lists of unbounded agents (k_scan)
+    key_t B[8];
+#pragma unroll
+    for (int s = 0; s < 7; ++s) B[s] = a.partial[(qi * PSLOTS + p) * 7 + s];
+    B[7] = KEY_EMPTY;
+    merge8(L, B);
   }
   a.hitcnt[qi] = 0;  // ready for the next step
   a.pcnt[qi] = 0;
-  a.nbr8[qi] = mine[7] == KEY_EMPTY ? -1 : key_idx(mine[7]);
+  a.nbr8[qi] = L[7] == KEY_EMPTY ? -1 : key_idx(L[7]);
   int nb[7], cnt = 0;
 #pragma unroll
   for (int s = 0; s < 7; ++s) {
-    nb[s] = mine[s] == KEY_EMPTY ? -1 : key_idx(mine[s]);
-    cnt += mine[s] == KEY_EMPTY ? 0 : 1;
+    nb[s] = L[s] == KEY_EMPTY ? -1 : key_idx(L[s]);
+    cnt += L[s] == KEY_EMPTY ? 0 : 1;
   }
 #pragma unroll
   for (int s = 0; s < 7; ++s) a.nbr[qi * 7 + s] = nb[s];
@@ -602,9 +557,9 @@ __device__ __forceinline__ void select4_body(const StepArgs& a) {
   modify_agent(a, qi, v3(p4), f4, F);
 }
 
-__global__ void __launch_bounds__(NSEL) k_select4(StepArgs a) {
+__global__ void __launch_bounds__(NSEL) k_select1(StepArgs a) {
   span_begin(a, SPAN_SLOT0 + 1);
-  select4_body(a);
+  select1_body(a);
   span_end(a, SPAN_SLOT0 + 1);
 }
 
@@ -623,12 +578,21 @@ int scan_grid(int sms) {
   return grid;
 }
 
+// Smallest CTA share of the (query block, candidate) items (measured C1: 128 ->
+// 42.2, 32 -> 32.5, 16 -> 30.5 us/step; C2 unchanged).  At small n the scan
+// is latency-bound (a CTA's time is mostly its fixed prologue and TMA latency),
+// so spreading it over more SMs beats whole-tile shares.
+#ifndef BOIDS_SCAN_MIN
+#define BOIDS_SCAN_MIN 16
+#endif
+constexpr int64_t SCAN_MIN = BOIDS_SCAN_MIN;
+
 template <int NT>
 cudaError_t scan_with(const StepArgs& a, int sms, int64_t ncand, cudaStream_t s) {
   const int64_t nqb = (a.nloc + NT * Q - 1) / (NT * Q);
   const int64_t items = nqb * ncand;  // (query block, candidate) pairs; think mode: recomputed on device
   const int g = a.qcount ? scan_grid<NT>(sms)
-                         : (int)std::min<int64_t>(scan_grid<NT>(sms), (items + CT - 1) / CT);
+                         : (int)std::min<int64_t>(scan_grid<NT>(sms), (items + SCAN_MIN - 1) / SCAN_MIN);
   k_scan<NT><<<g, NT, sizeof(ScanSmem<NT>), s>>>(a, ncand, items);
   return cudaGetLastError();
 }
@@ -658,8 +622,8 @@ cudaError_t launch_warm_scan(const StepArgs& a, cudaStream_t s) {
 cudaError_t launch_warm_select(const StepArgs& a, cudaStream_t s) {
   if (a.nloc <= 0) return cudaSuccess;
   if (a.think_k <= 1 && a.rlist) {
-    BOIDS_PREFER_SMEM(k_select4);
-    k_select4<<<(unsigned)((a.nloc + NSEL - 1) / NSEL), NSEL, 0, s>>>(a);
+    BOIDS_PREFER_SMEM(k_select1);
+    k_select1<<<(unsigned)((a.nloc + NSEL - 1) / NSEL), NSEL, 0, s>>>(a);
     return cudaGetLastError();
   }
   BOIDS_PREFER_SMEM(k_select);

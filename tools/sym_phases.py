@@ -30,7 +30,7 @@ for name in sys.argv[1:] or ["c3"]:
     f.sync()
     raw = abi.boids_get_phases(f.h, 1024)
     spans = {}
-    for nm, slot in (("k_sym_prep", 1000), ("k_select4", 1001), ("k_route", 1002)):
+    for nm, slot in (("k_sym_prep", 1000), ("k_select1", 1001), ("k_route", 1002)):
         b, e = int(raw[slot, 0]), int(raw[slot, 1])
         if b and e:
             spans[nm] = ((~np.uint64(b)).astype(np.int64), e)
