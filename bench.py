@@ -249,7 +249,7 @@ def main():
     torch.cuda.synchronize()
 
     # ---------------- timed region: K steps, L2 flushed before each ----------------
-    abi.boids_set_option(h, abi.BOIDS_OPT_PROFILE, 1)
+    abi.boids_set_option(h, abi.BOIDS_OPT_PROFILE, 2)  # events around the search and update launches only
     abi.boids_get_profile(h, reset=True)
     info0 = abi.boids_info(h)
     launches0 = info0.launches

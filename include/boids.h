@@ -109,7 +109,9 @@ typedef struct boids_info_t {
 /* Options for boids_set_option. */
 #define BOIDS_OPT_RECORD_STEERING 1 /* 1: keep the last step's steering vectors (boids_get_steering) */
 #define BOIDS_OPT_KERNEL 2          /* BOIDS_KERNEL_* */
-#define BOIDS_OPT_PROFILE 3         /* 1: bracket each kernel launch with CUDA events (boids_get_profile) */
+#define BOIDS_OPT_PROFILE 3         /* 1: bracket each kernel launch with CUDA events (boids_get_profile);
+                                       2: only the search launches (and the update launches in think
+                                       mode): fewer event records inside a timed step; 0: off */
 #define BOIDS_OPT_CLUSTER 4         /* 0 = automatic, else force the fused kernel's cluster size (1..16) */
 #define BOIDS_OPT_RESORT 6          /* refresh the spatial order of the fused kernel's query blocks every
                                        `value` steps (default 8; results never depend on it) */

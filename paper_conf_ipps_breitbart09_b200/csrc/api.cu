@@ -103,7 +103,7 @@ struct boids_ctx {
   bool record_steering = false, steering_valid = false;
   int kernel = BOIDS_KERNEL_FUSED;
   int cluster_opt = 0;
-  bool profile = false;
+  int profile = 0;          // BOIDS_OPT_PROFILE level
   int64_t launches = 0;
   struct Rec {
     int cls;
@@ -214,14 +214,19 @@ cudaEvent_t get_event(boids_ctx* c) {
 template <class F>
 int launch(boids_ctx* c, int cls, F&& f, int kernels = 1) {
   cudaEvent_t a = nullptr, b = nullptr;
-  if (c->profile) {
+  // level 2: only the search classes (0, 3), plus the update (1) in think mode
+  // (k_apply / k_select carry that step's modification roofline) -- fewer event
+  // records in a timed step (each costs GPU time between dependent kernels)
+  const bool rec = c->profile == 1 ||
+                   (c->profile == 2 && (cls == 0 || cls == 3 || (cls == 1 && c->p.think_every > 1)));
+  if (rec) {
     a = get_event(c);
     b = get_event(c);
     CK(cudaEventRecord(a, c->stream));
   }
   CK(f());
   c->launches += kernels;
-  if (c->profile) {
+  if (rec) {
     CK(cudaEventRecord(b, c->stream));
     c->recs.push_back({cls, a, b});
   }
@@ -489,7 +494,11 @@ int one_step(boids_ctx* c, float dt) {
       // a single-GPU handle evaluates each unordered pair once (k_sym)
       // (below 8192 agents the step is latency-bound and the ordered-pair path,
       // with one launch less, is faster: measured C1/C2 55 vs 68 us)
-      if (c->symmetric && c->sym_sp && c->nloc >= 8192) {
+      static const int64_t sym_min = [] {
+        const char* e = getenv("BOIDS_SYM_MIN");  // diagnostics: smallest n on k_sym
+        return e ? atoll(e) : 8192LL;
+      }();
+      if (c->symmetric && c->sym_sp && c->nloc >= sym_min) {
         StepArgs as = a;
         as.routed = c->routed;  // agents routed to k_route by k_sym_prep (k_select skips them)
         CK(cudaMemsetAsync(c->sym_rcount, 0, sizeof(int32_t), c->stream));
@@ -602,7 +611,8 @@ BOIDS_API int boids_set_option(boids_ctx* c, int32_t opt, int64_t v) {
       c->kernel = (int)v;
       return BOIDS_OK;
     case BOIDS_OPT_PROFILE:
-      c->profile = v != 0;
+      if (v < 0 || v > 2) return fail(BOIDS_EINVAL, "profile level must be 0, 1 or 2");
+      c->profile = (int)v;
       return BOIDS_OK;
     case BOIDS_OPT_SYMMETRIC:
       c->symmetric = v != 0;

@@ -16,7 +16,7 @@ done
 timeout 300 python bench.py --impl reference > $OUT/bench_reference.json 2>&1
 if [ -z "$NO_NCU" ]; then
 for w in ${NCU_WORKLOADS:-c4 c3 c5}; do
-  K=k_sym; [ $w = c5 ] && K=k_grid
+  K=k_sym; [ $w = c5 ] && K=k_grid; [ $w = c1 ] && K=k_scan
   timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches_$w.csv \
      python bench.py --workload $w --steps 3 --warmup 3 --no-cpu-baseline --no-e2e > $OUT/ncu_launch_$w.log 2>&1
   timeout 1200 ncu --set full --clock-control none --import-source on -k $K -s 2 -c 1 -o $OUT/prof_$w \
