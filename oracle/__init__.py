@@ -44,6 +44,7 @@ class OracleParams(C.Structure):
         ("search_mode", C.c_int32),
         ("init_mode", C.c_int32),
         ("think_every", C.c_int32),
+        ("steer_mode", C.c_int32),
     ]
 
 
@@ -72,13 +73,14 @@ def lib():
         L.oracle_search_one.argtypes = [C.c_int64, f32p, C.c_float, C.c_int64, i32p, i32p]
         L.oracle_steer_one.argtypes = [f32p, f32p, C.c_int64, i32p, C.c_int32, P, f32p]
         L.oracle_modify_one.argtypes = [f32p, f32p, f32p, f32p, C.c_float, f32p, P, C.c_float,
-                                        f32p, f32p, f32p, f32p, f32p]
-        L.oracle_step.argtypes = [C.c_int64, P, C.c_float] + [f32p] * 5 + [f32p] * 5 + [i32p, i32p, f32p]
+                                        f32p, f32p, f32p, f32p, f32p, f32p]
+        L.oracle_step.argtypes = ([C.c_int64, P, C.c_float] + [f32p] * 5 + [f32p] * 5
+                                  + [i32p, i32p, f32p, f32p])
         L.oracle_step_sample.argtypes = ([C.c_int64, P, C.c_float] + [f32p] * 5 + [C.c_int64, i64p]
-                                         + [f32p] * 5 + [i32p, i32p, f32p])
+                                         + [f32p] * 5 + [i32p, i32p, f32p, f32p])
         L.oracle_step_think.argtypes = ([C.c_int64, P, C.c_float, C.c_int64] + [f32p] * 5 + [f32p] * 5
-                                        + [i32p, i32p, f32p, f32p])
-        L.oracle_run.argtypes = [C.c_int64, P, C.c_float, C.c_int32] + [f32p] * 5
+                                        + [i32p, i32p, f32p, f32p, f32p])
+        L.oracle_run.argtypes = [C.c_int64, P, C.c_float, C.c_int32] + [f32p] * 6
         L.oracle_run.restype = C.c_int
         _lib = L
     return _lib
@@ -98,7 +100,8 @@ def _f32(a, shape=None):
 
 
 class State(dict):
-    """Host AoS state: pos/fwd/up/side (n,3) float32 and speed (n,) float32."""
+    """Host AoS state: pos/fwd/up/side (n,3) float32 and speed (n,) float32; with
+    steer_mode 1 also acc (n,3), the smoothed accelerations (zero if absent)."""
 
     @property
     def n(self) -> int:
@@ -145,16 +148,31 @@ def steer_one(pos, fwd, i: int, idx7, cnt: int, params: OracleParams | None = No
     return F
 
 
-def modify_one(pos, fwd, up, side, speed, force, dt: float, params: OracleParams | None = None):
+def modify_one(pos, fwd, up, side, speed, force, dt: float, params: OracleParams | None = None, acc=None):
+    """acc: steer_mode 1 smoothed acceleration (3,) before the step; the result's
+    "acc" is the one after it."""
     p = params or default_params()
     outs = [np.empty(3, np.float32) for _ in range(4)] + [np.empty(1, np.float32)]
+    a = np.array(acc if acc is not None else np.zeros(3), np.float32).reshape(3)
     lib().oracle_modify_one(_f32(pos), _f32(fwd), _f32(up), _f32(side), C.c_float(speed),
-                            _f32(force), C.byref(p), C.c_float(dt), *outs)
-    return dict(pos=outs[0], fwd=outs[1], up=outs[2], side=outs[3], speed=float(outs[4][0]))
+                            _f32(force), C.byref(p), C.c_float(dt), *outs, a)
+    return dict(pos=outs[0], fwd=outs[1], up=outs[2], side=outs[3], speed=float(outs[4][0]), acc=a)
 
 
 def _state_arrays(s):
     return [_f32(s[k], (-1, 3)) for k in ("pos", "fwd", "up", "side")] + [_f32(s["speed"])]
+
+
+def _acc_in(s, n):
+    """A private copy of the smoothed accelerations (updated in place by the C side)."""
+    a = s.get("acc") if hasattr(s, "get") else None
+    return np.zeros((n, 3), np.float32) if a is None else np.array(a, np.float32, copy=True).reshape(n, 3)
+
+
+def _with_acc(out, acc, p):
+    if p.steer_mode == 1:
+        out["acc"] = acc
+    return out
 
 
 def step(s: State, dt: float, params: OracleParams | None = None):
@@ -168,9 +186,10 @@ def step(s: State, dt: float, params: OracleParams | None = None):
     idx = np.empty((n, 7), np.int32)
     cnt = np.empty(n, np.int32)
     F = np.empty((n, 3), np.float32)
+    acc = _acc_in(s, n)
     lib().oracle_step(n, C.byref(p), C.c_float(dt), *ins, out["pos"], out["fwd"], out["up"],
-                      out["side"], out["speed"], idx, cnt, F)
-    return out, idx, cnt, F
+                      out["side"], out["speed"], idx, cnt, F, acc)
+    return _with_acc(out, acc, p), idx, cnt, F
 
 
 def step_sample(s: State, agents, dt: float, params: OracleParams | None = None):
@@ -184,10 +203,11 @@ def step_sample(s: State, agents, dt: float, params: OracleParams | None = None)
     idx = np.empty((m, 7), np.int32)
     cnt = np.empty(m, np.int32)
     F = np.empty((m, 3), np.float32)
+    acc = np.ascontiguousarray(_acc_in(s, s.n)[agents])
     lib().oracle_step_sample(s.n, C.byref(p), C.c_float(dt), *_state_arrays(s), m, agents,
                              out["pos"], out["fwd"], out["up"], out["side"], out["speed"],
-                             idx, cnt, F)
-    return out, idx, cnt, F
+                             idx, cnt, F, acc)
+    return _with_acc(out, acc, p), idx, cnt, F
 
 
 def step_think(s: State, dt: float, t: int, fstore, idx7, cnt, params: OracleParams | None = None):
@@ -204,16 +224,18 @@ def step_think(s: State, dt: float, t: int, fstore, idx7, cnt, params: OraclePar
     c = np.array(cnt, np.int32, copy=True).reshape(n)
     fs = np.array(fstore, np.float32, copy=True).reshape(n, 3)
     F = np.empty((n, 3), np.float32)
+    acc = _acc_in(s, n)
     lib().oracle_step_think(n, C.byref(p), C.c_float(dt), t, *_state_arrays(s), out["pos"], out["fwd"],
-                            out["up"], out["side"], out["speed"], idx, c, fs, F)
-    return out, idx, c, fs, F
+                            out["up"], out["side"], out["speed"], idx, c, fs, F, acc)
+    return _with_acc(out, acc, p), idx, c, fs, F
 
 
 def run(s: State, dt: float, steps: int, params: OracleParams | None = None) -> State:
     p = params or default_params()
     s = State({k: np.array(v, np.float32, copy=True) for k, v in s.items()})
     arrs = _state_arrays(s)
-    rc = lib().oracle_run(s.n, C.byref(p), C.c_float(dt), steps, *arrs)
+    acc = _acc_in(s, s.n)
+    rc = lib().oracle_run(s.n, C.byref(p), C.c_float(dt), steps, *arrs, acc)
     if rc != 0:
         raise MemoryError("oracle_run")
-    return State(pos=arrs[0], fwd=arrs[1], up=arrs[2], side=arrs[3], speed=arrs[4])
+    return _with_acc(State(pos=arrs[0], fwd=arrs[1], up=arrs[2], side=arrs[3], speed=arrs[4]), acc, p)

@@ -26,6 +26,12 @@
  *   - synchronous (Jacobi) update: every output of step t is computed from
  *     the state of step t only (two substages; two kernels).
  *   - initial state: DESIGN.md Appendix B (the paper is silent).
+ *   - steer_mode 1 (the thesis's device code "is based on
+ *     the CPU version of OpenSteer"): OpenSteer 0.8.2's own flocking
+ *     instead of Listings 5.3-5.5 -- per-behaviour neighbourhood filters
+ *     (inBoidNeighborhood), averaged behaviours, adjustRawSteeringForce and
+ *     acceleration smoothing (blendIntoAccumulator) in the modification.
+ *     Restated from OpenSteer [ext], not from the paper: DESIGN.md Q20-Q24.
  *
  * Arithmetic (DESIGN.md Appendix A): IEEE binary32, round to nearest even,
  * every operation individually rounded, no fused multiply-add, evaluated in
@@ -59,6 +65,8 @@ typedef struct oracle_params {
   int32_t search_mode;  /* ignored by the oracle: every mode has one answer */
   int32_t init_mode;    /* 0 = ball of init_radius, 1 = ball of world_radius */
   int32_t think_every;  /* think frequency k; 1 = every agent thinks every step */
+  int32_t steer_mode;   /* 0 = the thesis's Listings 5.1-5.5 + reading Q10 (default);
+                           1 = OpenSteer 0.8.2 flocking [ext] (readings Q20-Q24) */
 } oracle_params;
 
 void oracle_default_params(oracle_params* p) {
@@ -76,6 +84,7 @@ void oracle_default_params(oracle_params* p) {
   p->search_mode = 0;
   p->init_mode = 0;
   p->think_every = 1;
+  p->steer_mode = 0;
 }
 
 /* ---------------- Appendix A vector helpers (each op rounded) ------------ */
@@ -221,9 +230,16 @@ void oracle_search(int64_t n, const float* pos3, float radius, int32_t* idx7, in
   for (int64_t i = 0; i < n; ++i) oracle_search_one(n, pos3, radius, i, idx7 + 7 * i, cnt + i);
 }
 
+static void oracle_steer_one_os(const float* pos3, const float* fwd3, int64_t i, const int32_t* idx7,
+                                int32_t cnt, const oracle_params* p, float* force3);
+
 /* ---------------- Listings 5.1, 5.3, 5.4, 5.5 steering -------------------- */
 void oracle_steer_one(const float* pos3, const float* fwd3, int64_t i, const int32_t* idx7,
                       int32_t cnt, const oracle_params* p, float* force3) {
+  if (p->steer_mode == 1) {
+    oracle_steer_one_os(pos3, fwd3, i, idx7, cnt, p, force3);
+    return;
+  }
   v3 me = v3_load(pos3, i);
   v3 fme = v3_load(fwd3, i);
   v3 sep = v3_make(0.0f, 0.0f, 0.0f);
@@ -251,17 +267,113 @@ void oracle_steer_one(const float* pos3, const float* fwd3, int64_t i, const int
   v3_store(force3, 0, F);
 }
 
+/* ---------------- steer_mode 1: OpenSteer 0.8.2 flocking [ext] -------------
+ * Boid::steerToFlock with SteerLibrary's steerForSeparation / Alignment /
+ * Cohesion over the same <= 7 neighbours (the thesis's list), each behaviour
+ * keeping only the neighbours inBoidNeighborhood(minDistance = 3 * radius
+ * (radius 0.5), maxDistance, cosMaxAngle) accepts (Q20-Q22). */
+#define OS_MIN_DIST 1.5f   /* 3 * SimpleVehicle radius 0.5 */
+#define OS_SEP_R 5.0f
+#define OS_SEP_COS (-0.707f)
+#define OS_ALI_R 7.5f
+#define OS_ALI_COS 0.7f
+#define OS_COH_R 9.0f
+#define OS_COH_COS (-0.15f)
+
+/* inBoidNeighborhood: inside minDistance -> yes; beyond maxDistance -> no;
+ * else forward . (offset / |offset|) > cosMaxAngle. */
+static int os_in_hood(v3 o, float d2, v3 fme, float min_d, float max_d, float cos_max) {
+  if (d2 < min_d * min_d) return 1;
+  if (d2 > max_d * max_d) return 0;
+  v3 unit = v3_divs(o, sqrtf(d2));
+  return v3_dot(fme, unit) > cos_max;
+}
+
+static void oracle_steer_one_os(const float* pos3, const float* fwd3, int64_t i, const int32_t* idx7,
+                                int32_t cnt, const oracle_params* p, float* force3) {
+  v3 me = v3_load(pos3, i);
+  v3 fme = v3_load(fwd3, i);
+  v3 sep = v3_make(0.0f, 0.0f, 0.0f), ali = sep, coh = sep;
+  int ns = 0, na = 0, nc = 0;
+  for (int k = 0; k < cnt; ++k) {               /* neighbours in key order (Q8) */
+    int64_t j = idx7[k];
+    v3 pj = v3_load(pos3, j);
+    v3 o = v3_sub(pj, me);                      /* offset = other.position - position */
+    float d2 = v3_dot(o, o);                    /* offset.lengthSquared() */
+    if (os_in_hood(o, d2, fme, OS_MIN_DIST, OS_SEP_R, OS_SEP_COS) && d2 > 0.0f) {
+      sep = v3_add(sep, v3_divs(o, -d2));       /* steering += offset / -distanceSquared */
+      ++ns;
+    }
+    if (os_in_hood(o, d2, fme, OS_MIN_DIST, OS_ALI_R, OS_ALI_COS)) {
+      ali = v3_add(ali, v3_load(fwd3, j));      /* steering += other.forward() */
+      ++na;
+    }
+    if (os_in_hood(o, d2, fme, OS_MIN_DIST, OS_COH_R, OS_COH_COS)) {
+      coh = v3_add(coh, pj);                    /* steering += other.position() */
+      ++nc;
+    }
+  }
+  if (ns > 0) sep = v3_normalize(v3_divs(sep, (float)ns));
+  if (na > 0) ali = v3_normalize(v3_sub(v3_divs(ali, (float)na), fme));
+  if (nc > 0) coh = v3_normalize(v3_sub(v3_divs(coh, (float)nc), me));
+  v3 sw = v3_scale(sep, p->w_separation);
+  v3 aw = v3_scale(ali, p->w_alignment);
+  v3 cw = v3_scale(coh, p->w_cohesion);
+  v3 F = v3_add(v3_add(sw, aw), cw);
+  v3_store(force3, 0, F);
+}
+
+/* x^20 as ((x^2)^2)^2)^2 * x^4, each product rounded (reading Q23 for pow(range, 20)). */
+static float os_pow20(float x) {
+  float x2 = x * x, x4 = x2 * x2, x8 = x4 * x4, x16 = x8 * x8;
+  return x16 * x4;
+}
+
+/* SimpleVehicle::adjustRawSteeringForce (Q23): below 0.2 maxSpeed the force is
+ * kept within a cone around forward (vecLimitDeviationAngleUtility, inside). */
+static v3 os_adjust_raw(v3 F, float speed, v3 fwd, const oracle_params* p) {
+  float max_adj = 0.2f * p->max_speed;
+  if (speed > max_adj || (F.x == 0.0f && F.y == 0.0f && F.z == 0.0f)) return F;
+  float range = speed / max_adj;
+  float cosine = 1.0f + (-1.0f - 1.0f) * os_pow20(range); /* interpolate(pow(range,20), 1, -1) */
+  float L = v3_len(F);
+  if (L == 0.0f) return F;
+  v3 dir = v3_divs(F, L);
+  if (v3_dot(dir, fwd) >= cosine) return F;
+  v3 perp = v3_sub(F, v3_scale(fwd, v3_dot(F, fwd)));  /* source.perpendicularComponent(basis) */
+  v3 uperp = v3_normalize(perp);
+  float perp_dist = sqrtf(1.0f - cosine * cosine);
+  v3 c0 = v3_scale(fwd, cosine);
+  v3 c1 = v3_scale(uperp, perp_dist);
+  return v3_scale(v3_add(c0, c1), L);
+}
+
 /* ---------------- modification substage (reading Q10-Q13) ----------------- */
+/* acc3: steer_mode 1 only -- the agent's smoothed acceleration, read and
+ * updated in place (OpenSteer's _smoothedAcceleration; only the agent itself
+ * uses it, so the in-place update keeps the step synchronous). */
 void oracle_modify_one(const float* p_in, const float* f_in, const float* u_in, const float* s_in,
                        float speed, const float* F_in, const oracle_params* p, float dt,
-                       float* p_out, float* f_out, float* u_out, float* s_out, float* speed_out) {
+                       float* p_out, float* f_out, float* u_out, float* s_out, float* speed_out,
+                       float* acc3) {
   v3 pos = v3_make(p_in[0], p_in[1], p_in[2]);
   v3 f = v3_make(f_in[0], f_in[1], f_in[2]);
   v3 u = v3_make(u_in[0], u_in[1], u_in[2]);
   v3 s = v3_make(s_in[0], s_in[1], s_in[2]);
   v3 F = v3_make(F_in[0], F_in[1], F_in[2]);
+  if (p->steer_mode == 1) F = os_adjust_raw(F, speed, f, p);  /* Q23 */
   v3 Fc = v3_trunc(F, p->max_force);           /* clamp force */
   v3 a = v3_divs(Fc, p->mass);                 /* a = F / m  (length = acceleration) */
+  if (p->steer_mode == 1) {                    /* blendIntoAccumulator (Q24) */
+    v3 sm = v3_load(acc3, 0);
+    if (dt > 0.0f) {
+      float rate = 9.0f * dt;                  /* clip(9 dt, 0.15, 0.4) */
+      rate = rate < 0.15f ? 0.15f : (rate > 0.4f ? 0.4f : rate);
+      sm = v3_add(sm, v3_scale(v3_sub(a, sm), rate));  /* interpolate(rate, smoothed, new) */
+      v3_store(acc3, 0, sm);
+    }
+    a = sm;
+  }
   v3 v = v3_scale(f, speed);                   /* velocity = forward * speed */
   v3 v1 = v3_add(v, v3_scale(a, dt));          /* integrate velocity */
   v3 v2 = v3_trunc(v1, p->max_speed);          /* clamp speed */
@@ -289,21 +401,23 @@ static void step_agent(int64_t n, const oracle_params* p, float dt, const float*
                        const float* fwd3, const float* up3, const float* side3,
                        const float* speed, int64_t i, float* pos_o, float* fwd_o, float* up_o,
                        float* side_o, float* speed_o, int32_t* idx7, int32_t* cnt,
-                       float* force3) {
+                       float* force3, float* acc3) {
   oracle_search_one(n, pos3, p->search_radius, i, idx7, cnt);
   oracle_steer_one(pos3, fwd3, i, idx7, *cnt, p, force3);
   oracle_modify_one(pos3 + 3 * i, fwd3 + 3 * i, up3 + 3 * i, side3 + 3 * i, speed[i], force3, p,
-                    dt, pos_o, fwd_o, up_o, side_o, speed_o);
+                    dt, pos_o, fwd_o, up_o, side_o, speed_o, acc3);
 }
 
 /* Whole step S_t -> S_{t+1}; outputs must not alias inputs (Jacobi update). */
+/* acc3 (n,3): steer_mode 1 smoothed accelerations, updated in place (ignored otherwise). */
 void oracle_step(int64_t n, const oracle_params* p, float dt, const float* pos3,
                  const float* fwd3, const float* up3, const float* side3, const float* speed,
                  float* pos_o, float* fwd_o, float* up_o, float* side_o, float* speed_o,
-                 int32_t* idx7, int32_t* cnt, float* force3) {
+                 int32_t* idx7, int32_t* cnt, float* force3, float* acc3) {
   for (int64_t i = 0; i < n; ++i)
     step_agent(n, p, dt, pos3, fwd3, up3, side3, speed, i, pos_o + 3 * i, fwd_o + 3 * i,
-               up_o + 3 * i, side_o + 3 * i, speed_o + i, idx7 + 7 * i, cnt + i, force3 + 3 * i);
+               up_o + 3 * i, side_o + 3 * i, speed_o + i, idx7 + 7 * i, cnt + i, force3 + 3 * i,
+               acc3 + 3 * i);
 }
 
 /* Sampled step: only the m agents listed in `agents` (outputs indexed 0..m-1). */
@@ -311,10 +425,11 @@ void oracle_step_sample(int64_t n, const oracle_params* p, float dt, const float
                         const float* fwd3, const float* up3, const float* side3,
                         const float* speed, int64_t m, const int64_t* agents, float* pos_o,
                         float* fwd_o, float* up_o, float* side_o, float* speed_o,
-                        int32_t* idx7, int32_t* cnt, float* force3) {
-  for (int64_t k = 0; k < m; ++k)
+                        int32_t* idx7, int32_t* cnt, float* force3, float* acc3) {
+  for (int64_t k = 0; k < m; ++k)  /* acc3 (m,3): the sampled agents' accelerations, in/out */
     step_agent(n, p, dt, pos3, fwd3, up3, side3, speed, agents[k], pos_o + 3 * k, fwd_o + 3 * k,
-               up_o + 3 * k, side_o + 3 * k, speed_o + k, idx7 + 7 * k, cnt + k, force3 + 3 * k);
+               up_o + 3 * k, side_o + 3 * k, speed_o + k, idx7 + 7 * k, cnt + k, force3 + 3 * k,
+               acc3 + 3 * k);
 }
 
 /* One synchronous step with think frequency k = p->think_every (sec 5.3:
@@ -328,7 +443,7 @@ void oracle_step_sample(int64_t n, const oracle_params* p, float dt, const float
 void oracle_step_think(int64_t n, const oracle_params* p, float dt, int64_t t, const float* pos3,
                        const float* fwd3, const float* up3, const float* side3, const float* speed,
                        float* pos_o, float* fwd_o, float* up_o, float* side_o, float* speed_o,
-                       int32_t* idx7, int32_t* cnt, float* fstore3, float* force3) {
+                       int32_t* idx7, int32_t* cnt, float* fstore3, float* force3, float* acc3) {
   int64_t k = p->think_every < 1 ? 1 : p->think_every;
   for (int64_t i = 0; i < n; ++i) {
     if ((i + t) % k == 0) {
@@ -339,13 +454,14 @@ void oracle_step_think(int64_t n, const oracle_params* p, float dt, int64_t t, c
     force3[3 * i + 1] = fstore3[3 * i + 1];
     force3[3 * i + 2] = fstore3[3 * i + 2];
     oracle_modify_one(pos3 + 3 * i, fwd3 + 3 * i, up3 + 3 * i, side3 + 3 * i, speed[i], force3 + 3 * i, p,
-                      dt, pos_o + 3 * i, fwd_o + 3 * i, up_o + 3 * i, side_o + 3 * i, speed_o + i);
+                      dt, pos_o + 3 * i, fwd_o + 3 * i, up_o + 3 * i, side_o + 3 * i, speed_o + i,
+                      acc3 + 3 * i);
   }
 }
 
 /* Many synchronous steps (S_t -> S_{t+steps}); state arrays updated in place. */
 int oracle_run(int64_t n, const oracle_params* p, float dt, int32_t steps, float* pos3,
-               float* fwd3, float* up3, float* side3, float* speed) {
+               float* fwd3, float* up3, float* side3, float* speed, float* acc3) {
   size_t v = (size_t)n * 3 * sizeof(float);
   float* buf = (float*)malloc(4 * v + (size_t)n * sizeof(float) + (size_t)n * 7 * sizeof(int32_t) +
                               (size_t)n * sizeof(int32_t) + v);
@@ -359,7 +475,7 @@ int oracle_run(int64_t n, const oracle_params* p, float dt, int32_t steps, float
   int32_t* cnt = idx + 7 * n;
   float* F = (float*)(cnt + n);
   for (int32_t t = 0; t < steps; ++t) {
-    oracle_step(n, p, dt, pos3, fwd3, up3, side3, speed, po, fo, uo, so, spo, idx, cnt, F);
+    oracle_step(n, p, dt, pos3, fwd3, up3, side3, speed, po, fo, uo, so, spo, idx, cnt, F, acc3);
     memcpy(pos3, po, v);
     memcpy(fwd3, fo, v);
     memcpy(up3, uo, v);
