@@ -76,7 +76,18 @@ typedef struct boids_params {
   int32_t think_every;   /* think frequency k >= 1 (skipThink, sec 5.3): agent i runs the
                             simulation substage at step t iff (i + t) mod k == 0 and otherwise
                             reuses its stored steering vector; every agent is modified.  1 */
+  int32_t steer_mode;    /* BOIDS_STEER_THESIS (default): steering of Listings 5.1-5.5 and the
+                            modification of reading Q10.  BOIDS_STEER_OPENSTEER: OpenSteer 0.8.2's
+                            flocking [ext] over the same <= 7 neighbours (
+                            "based on the CPU version of OpenSteer"): per-behaviour
+                            inBoidNeighborhood filters (radii 5 / 7.5 / 9, cos -0.707 / 0.7 / -0.15,
+                            always within 1.5), averaged behaviours, adjustRawSteeringForce below
+                            0.2 max_speed and acceleration smoothing (per-agent state, see
+                            boids_get_accel).  DESIGN.md readings Q20-Q24. */
 } boids_params;
+
+#define BOIDS_STEER_THESIS 0
+#define BOIDS_STEER_OPENSTEER 1
 
 typedef struct boids_ctx boids_ctx; /* opaque handle */
 
@@ -172,6 +183,14 @@ BOIDS_API int boids_get_state(boids_ctx* ctx, float* pos3, float* fwd3, float* u
  * pos3, fwd3, up3, speed must be non-NULL; side3 may be NULL (then zero).  Synchronises. */
 BOIDS_API int boids_set_state(boids_ctx* ctx, const float* pos3, const float* fwd3, const float* up3,
                     const float* side3, const float* speed);
+
+/* steer_mode BOIDS_STEER_OPENSTEER only: the smoothed accelerations
+ * (OpenSteer's _smoothedAcceleration, zero at creation) of the owned agents,
+ * host AoS float acc3[(hi - lo) * 3].  get: copies into caller memory and
+ * synchronises the handle's stream; set: copies from caller memory (used from
+ * the next step on).  BOIDS_EINVAL on a NULL argument or another steer_mode. */
+BOIDS_API int boids_get_accel(boids_ctx* ctx, float* acc3);
+BOIDS_API int boids_set_accel(boids_ctx* ctx, const float* acc3);
 
 /* Neighbour lists of the last step for the owned agents: idx7 = count*7 int32,
  * ascending by (d2, index), -1 padded; cnt = count int32, or -1 for an agent that

@@ -19,6 +19,7 @@ LIB_PATH = os.path.join(HERE, "libboids.so")
 BOIDS_OK, BOIDS_EINVAL, BOIDS_ECUDA, BOIDS_ENCCL, BOIDS_ENOMEM = 0, -1, -2, -3, -4
 BOIDS_BRUTE, BOIDS_GRID = 0, 1
 BOIDS_INIT_OPENSTEER, BOIDS_INIT_WORLD = 0, 1
+BOIDS_STEER_THESIS, BOIDS_STEER_OPENSTEER = 0, 1
 BOIDS_KERNEL_FUSED, BOIDS_KERNEL_SIMPLE, BOIDS_KERNEL_CLUSTER = 0, 1, 2
 BOIDS_OPT_RECORD_STEERING, BOIDS_OPT_KERNEL, BOIDS_OPT_PROFILE, BOIDS_OPT_CLUSTER, BOIDS_OPT_PHASES = 1, 2, 3, 4, 5
 BOIDS_OPT_RESORT, BOIDS_OPT_VOTE_U, BOIDS_OPT_SYMMETRIC, BOIDS_OPT_BALANCE = 6, 7, 8, 9
@@ -32,6 +33,7 @@ EXPORTS = (
     "boids_get_state", "boids_set_state", "boids_get_neighbors", "boids_get_steering",
     "boids_sync", "boids_info", "boids_get_profile", "boids_get_phases", "boids_destroy", "boids_last_error",
     "boids_get_think_state", "boids_set_think_state", "boids_readback_begin", "boids_readback_wait",
+    "boids_get_accel", "boids_set_accel",
 )
 
 
@@ -47,7 +49,7 @@ class boids_params(C.Structure):
         ("w_cohesion", C.c_float), ("max_force", C.c_float), ("max_speed", C.c_float),
         ("mass", C.c_float), ("world_radius", C.c_float), ("init_radius", C.c_float),
         ("init_speed_frac", C.c_float), ("max_neighbors", C.c_int32), ("search_mode", C.c_int32),
-        ("init_mode", C.c_int32), ("think_every", C.c_int32),
+        ("init_mode", C.c_int32), ("think_every", C.c_int32), ("steer_mode", C.c_int32),
     ]
 
 
@@ -86,6 +88,8 @@ def load(path: str = LIB_PATH):
         "boids_shard_buffers": (C.c_int, [vp, C.POINTER(vp), C.POINTER(vp), C.POINTER(i64)]),
         "boids_get_state": (C.c_int, [vp, fp, fp, fp, fp, fp]),
         "boids_set_state": (C.c_int, [vp, fp, fp, fp, fp, fp]),
+        "boids_get_accel": (C.c_int, [vp, fp]),
+        "boids_set_accel": (C.c_int, [vp, fp]),
         "boids_get_neighbors": (C.c_int, [vp, ip, ip]),
         "boids_get_steering": (C.c_int, [vp, fp]),
         "boids_sync": (C.c_int, [vp]),
@@ -204,6 +208,17 @@ def boids_set_state(h: int, state: dict):
     side = None if state.get("side") is None else _f32(state["side"], (cnt, 3))
     speed = _f32(state["speed"], (cnt,))
     _check(load().boids_set_state(h, _fptr(pos), _fptr(fwd), _fptr(up), _fptr(side), _fptr(speed)))
+
+
+def boids_get_accel(h: int):
+    """steer_mode BOIDS_STEER_OPENSTEER: smoothed accelerations (count, 3) of the owned agents."""
+    acc = np.empty((_count(h), 3), np.float32)
+    _check(load().boids_get_accel(h, _fptr(acc)))
+    return acc
+
+
+def boids_set_accel(h: int, acc):
+    _check(load().boids_set_accel(h, _fptr(_f32(acc, (_count(h), 3)))))
 
 
 def boids_get_neighbors(h: int):

@@ -31,12 +31,70 @@ __device__ __forceinline__ void prefetch_l1(const void* p) {
   asm volatile("prefetch.global.L1 [%0];" ::"l"(p));
 }
 
+// ---- steer_mode 1: OpenSteer 0.8.2 flocking [ext] (the
+// thesis's device code "is based on the CPU version of OpenSteer", P:434;
+// DESIGN.md Q20-Q24).  Inlined behind a uniform branch on steer_mode: an
+// out-of-line call taking StepArgs& put the kernel parameters on the stack of
+// every default kernel (measured +10 us per step at C1).
+constexpr float OS_MIN_DIST = 1.5f;  // 3 x SimpleVehicle radius 0.5
+// inBoidNeighborhood: inside min distance -> yes; beyond max -> no; else
+// forward . (offset / |offset|) > cos max angle
+__device__ __forceinline__ bool os_in_hood(V3 o, float d2, V3 fme, float max_d, float cos_max) {
+  if (d2 < __fmul_rn(OS_MIN_DIST, OS_MIN_DIST)) return true;
+  if (d2 > __fmul_rn(max_d, max_d)) return false;
+  return dot(fme, divs(o, __fsqrt_rn(d2))) > cos_max;
+}
+
+__device__ __forceinline__ V3 steer_agent_os(const StepArgs& a, V3 me, V3 fme, const int* nb, int cnt) {
+  V3 sep = v3(0.f, 0.f, 0.f), ali = sep, coh = sep;
+  int ns = 0, na = 0, nc = 0;
+  for (int k = 0; k < cnt; ++k) {  // neighbours in key order (Q8)
+    const int64_t j = nb[k];
+    const V3 pj = v3(__ldg(pos_of(a.full, a.m, a.sdiv, j)));
+    const V3 o = sub(pj, me);
+    const float d2 = dot(o, o);
+    if (os_in_hood(o, d2, fme, 5.0f, -0.707f) && d2 > 0.0f) {
+      sep = add(sep, divs(o, -d2));  // offset / -distanceSquared
+      ++ns;
+    }
+    if (os_in_hood(o, d2, fme, 7.5f, 0.7f)) {
+      ali = add(ali, v3(__ldg(fwd_of(a.full, a.m, a.sdiv, j))));
+      ++na;
+    }
+    if (os_in_hood(o, d2, fme, 9.0f, -0.15f)) {
+      coh = add(coh, pj);
+      ++nc;
+    }
+  }
+  if (ns > 0) sep = normalize(divs(sep, (float)ns));
+  if (na > 0) ali = normalize(sub(divs(ali, (float)na), fme));
+  if (nc > 0) coh = normalize(sub(divs(coh, (float)nc), me));
+  return add(add(scale(sep, a.p.w_separation), scale(ali, a.p.w_alignment)), scale(coh, a.p.w_cohesion));
+}
+
+// SimpleVehicle::adjustRawSteeringForce (Q23): below 0.2 maxSpeed the force is
+// kept within a cone of cos = interpolate(range^20, 1, -1) around forward.
+__device__ __forceinline__ V3 os_adjust_raw(V3 F, float speed, V3 fwd, float max_speed) {
+  const float max_adj = __fmul_rn(0.2f, max_speed);
+  if (speed > max_adj || (F.x == 0.0f && F.y == 0.0f && F.z == 0.0f)) return F;
+  const float r = __fdiv_rn(speed, max_adj);
+  const float r2 = __fmul_rn(r, r), r4 = __fmul_rn(r2, r2), r8 = __fmul_rn(r4, r4), r16 = __fmul_rn(r8, r8);
+  const float cosine = __fadd_rn(1.0f, __fmul_rn(-2.0f, __fmul_rn(r16, r4)));  // 1 + (-1 - 1) * r^20
+  const float L = len(F);
+  if (L == 0.0f) return F;
+  if (dot(divs(F, L), fwd) >= cosine) return F;
+  const V3 uperp = normalize(sub(F, scale(fwd, dot(F, fwd))));
+  const float perp_dist = __fsqrt_rn(__fsub_rn(1.0f, __fmul_rn(cosine, cosine)));
+  return scale(add(scale(fwd, cosine), scale(uperp, perp_dist)), L);
+}
+
 // Steering vector of agent g from its <=7 neighbours (in key order, Q8).  The
 // neighbours' lines are prefetched into L1 up front and the loop is kept
 // rolled: this code runs once per agent per step, so at small n its
 // instruction-fetch latency, not its arithmetic, is what the warps wait on.
 __device__ __forceinline__ V3 steer_agent(const StepArgs& a, V3 me, V3 fme, const int* nb,
                                           int cnt) {
+  if (a.p.steer_mode == BOIDS_STEER_OPENSTEER) return steer_agent_os(a, me, fme, nb, cnt);
 #pragma unroll
   for (int k = 0; k < 7; ++k)
     if (k < cnt) {
@@ -72,8 +130,20 @@ __device__ __forceinline__ void modify_agent(const StepArgs& a, int64_t i, V3 po
   float4 u4 = a.up4[i];
   float4 s4 = a.side4[i];
   V3 u = v3(u4), s = v3(s4);
-  V3 Fc = trunc_len(F, p.max_force);
+  // the recorded steering vector (force4) stays the raw one, as in the oracle
+  const V3 Fa = p.steer_mode == BOIDS_STEER_OPENSTEER ? os_adjust_raw(F, speed, f, p.max_speed) : F;
+  V3 Fc = trunc_len(Fa, p.max_force);
   V3 acc = divs(Fc, p.mass);
+  if (p.steer_mode == BOIDS_STEER_OPENSTEER) {  // blendIntoAccumulator (Q24); only agent i uses acc4[i]
+    V3 sm = v3(a.acc4[i]);
+    if (a.dt > 0.0f) {
+      float rate = __fmul_rn(9.0f, a.dt);  // clip(9 dt, 0.15, 0.4)
+      rate = rate < 0.15f ? 0.15f : (rate > 0.4f ? 0.4f : rate);
+      sm = add(sm, scale(sub(acc, sm), rate));
+      a.acc4[i] = make_float4(sm.x, sm.y, sm.z, 0.0f);
+    }
+    acc = sm;
+  }
   V3 v = scale(f, speed);
   V3 v1 = add(v, scale(acc, a.dt));
   V3 v2 = trunc_len(v1, p.max_speed);

@@ -62,6 +62,7 @@ struct boids_ctx {
   int32_t *bcnt = nullptr, *bstart = nullptr, *qperm = nullptr;
   float4* cand = nullptr;
   int64_t ncand = 0;
+  float4* acc4 = nullptr;               // steer_mode 1: smoothed accelerations [m]
   unsigned long long* stats = nullptr;  // fused-kernel insertion-path counters (device)
   unsigned long long* hits = nullptr;   // warm path hit buffers [m][HITS]
   int32_t* hitcnt = nullptr;            // warm path hit counts [m]
@@ -142,6 +143,8 @@ int validate(const boids_params* p) {
     return fail(BOIDS_EINVAL, "search_mode must be BOIDS_BRUTE or BOIDS_GRID");
   if (p->init_mode != BOIDS_INIT_OPENSTEER && p->init_mode != BOIDS_INIT_WORLD)
     return fail(BOIDS_EINVAL, "init_mode must be BOIDS_INIT_OPENSTEER or BOIDS_INIT_WORLD");
+  if (p->steer_mode != BOIDS_STEER_THESIS && p->steer_mode != BOIDS_STEER_OPENSTEER)
+    return fail(BOIDS_EINVAL, "steer_mode must be BOIDS_STEER_THESIS or BOIDS_STEER_OPENSTEER");
   return BOIDS_OK;
 }
 
@@ -152,6 +155,7 @@ void free_ctx(boids_ctx* c) {
   cudaFree(c->up4);
   cudaFree(c->side4);
   cudaFree(c->force4);
+  cudaFree(c->acc4);
   cudaFree(c->nbr);
   cudaFree(c->cnt);
   cudaFree(c->cellrank);
@@ -322,8 +326,13 @@ int create_impl(int64_t n, const boids_params* p, uint64_t seed, int32_t rank, i
     free_ctx(c);
     return rc;
   }
+  if (p->steer_mode == BOIDS_STEER_OPENSTEER && (rc = alloc((void**)&c->acc4, m * sizeof(float4)))) {
+    free_ctx(c);
+    return rc;
+  }
   cudaStream_t s = c->stream;
   cudaError_t e = cudaSuccess;
+  if (c->acc4) e = cudaMemsetAsync(c->acc4, 0, m * sizeof(float4), s);
   // phantoms in every segment of every buffer; then the owned agents
   if (e == cudaSuccess) e = cudaMemsetAsync(c->buf[0], 0, shard ? seg * world : seg, s);
   if (e == cudaSuccess) e = cudaMemsetAsync(c->buf[1], 0, seg, s);
@@ -397,6 +406,7 @@ StepArgs make_args(boids_ctx* c, float dt) {
   a.rlist = c->sym_rlist;  // warm brute-force steps route overflowed agents to k_route
   a.rcount = c->sym_rcount;
   a.loc = c->loc_grid;
+  a.acc4 = c->acc4;
   a.lstart = c->bstart;  // brute-force steps sort the queries (qperm) before any search
   return a;
 }
@@ -580,6 +590,7 @@ BOIDS_API void boids_default_params(boids_params* out) {
   out->search_mode = BOIDS_BRUTE;
   out->init_mode = BOIDS_INIT_OPENSTEER;
   out->think_every = 1;
+  out->steer_mode = BOIDS_STEER_THESIS;
 }
 
 BOIDS_API int boids_create(int64_t n, const boids_params* p, uint64_t seed, boids_ctx** out) {
@@ -736,6 +747,29 @@ BOIDS_API int boids_set_state(boids_ctx* c, const float* pos3, const float* fwd3
   // the last step until the next step.
   CK(cudaStreamSynchronize(c->stream));
   c->steering_valid = false;
+  return BOIDS_OK;
+}
+
+BOIDS_API int boids_get_accel(boids_ctx* c, float* acc3) {
+  if (!c) return fail(BOIDS_EINVAL, "NULL handle");
+  if (!acc3) return fail(BOIDS_EINVAL, "acc3 is NULL");
+  if (!c->acc4) return fail(BOIDS_EINVAL, "no acceleration state (steer_mode is not BOIDS_STEER_OPENSTEER)");
+  DeviceGuard g(c->dev);
+  // strided copy float4 -> packed float3 rows: the DMA engine converts the layout
+  CK(cudaMemcpy2DAsync(acc3, 3 * sizeof(float), c->acc4, sizeof(float4), 3 * sizeof(float), (size_t)c->nloc,
+                       cudaMemcpyDeviceToHost, c->stream));
+  CK(cudaStreamSynchronize(c->stream));
+  return BOIDS_OK;
+}
+
+BOIDS_API int boids_set_accel(boids_ctx* c, const float* acc3) {
+  if (!c) return fail(BOIDS_EINVAL, "NULL handle");
+  if (!acc3) return fail(BOIDS_EINVAL, "acc3 is NULL");
+  if (!c->acc4) return fail(BOIDS_EINVAL, "no acceleration state (steer_mode is not BOIDS_STEER_OPENSTEER)");
+  DeviceGuard g(c->dev);
+  CK(cudaMemcpy2DAsync(c->acc4, sizeof(float4), acc3, 3 * sizeof(float), 3 * sizeof(float), (size_t)c->nloc,
+                       cudaMemcpyHostToDevice, c->stream));
+  CK(cudaStreamSynchronize(c->stream));
   return BOIDS_OK;
 }
 

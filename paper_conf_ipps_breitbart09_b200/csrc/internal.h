@@ -106,6 +106,7 @@ struct StepArgs {
   int32_t* rlist;             // warm steps: agents finished by k_route (hit-buffer overflow, routed);
   int32_t* rcount;            // their number (zeroed before the step).  nullptr = warp re-search in k_select
   unsigned long long* phase;  // diagnostics: per-CTA %globaltimer stamps [grid][8], nullptr = off
+  float4* acc4;               // [m] steer_mode 1: smoothed accelerations (nullptr otherwise)
   BinGrid loc;                // locality (Morton) grid of the last query sort ...
   const int32_t* lstart;      // ... its cell starts in qperm (nullptr = none yet)
   float dt;
