@@ -519,7 +519,7 @@ int one_step(boids_ctx* c, float dt) {
                return launch_sym_scan(as, c->sym_sp, c->sym_idx, c->balance ? fb_prev : nullptr, fb_cur, c->stream);
              }, 2)))
           return rc;
-        if ((rc = launch(c, 1, [&] { return launch_warm_select(as, c->stream); }))) return rc;
+        if ((rc = launch(c, 1, [&] { return launch_warm_select(as, c->stream, false); }))) return rc;
         if ((rc = launch(c, 4, [&] { return launch_route(as, c->stream); }))) return rc;
       } else {
         CK(cudaMemsetAsync(c->sym_rcount, 0, sizeof(int32_t), c->stream));
@@ -542,6 +542,19 @@ int one_step(boids_ctx* c, float dt) {
 }
 
 }  // namespace
+
+bool boids::pdl_enabled() {
+  static const bool v = [] {
+    const char* e = getenv("BOIDS_PDL");
+    return !(e && atoi(e) == 0);
+  }();
+  return v;
+}
+
+bool boids::pdl_env(const char* name) {
+  const char* e = getenv(name);
+  return !(e && atoi(e) == 0);
+}
 
 int boids::carveout_pct() {
   static const int v = [] {

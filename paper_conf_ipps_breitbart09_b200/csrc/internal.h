@@ -1,5 +1,6 @@
 // internal.h -- private declarations shared by the CUDA translation units of libboids.
 #pragma once
+#include <utility>
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -145,6 +146,37 @@ int carveout_pct();
     (void)boids_once_;                                                                           \
   } while (0)
 
+// Programmatic dependent launch along a warm step's kernel chain (k_bound ->
+// k_scan / k_sym_prep -> k_sym -> k_select1 -> k_route): each of these kernels
+// lets its dependent be scheduled at once (pdl_trigger) and waits for its
+// predecessor's completion and memory (pdl_wait) before its first access to
+// step data, so launch latency and CTA rasterisation overlap the predecessor's
+// tail.  pdl_wait is a no-op for a kernel launched without the attribute.
+// BOIDS_PDL=0 turns the attribute off (diagnostics).
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" :::); }
+bool pdl_enabled();
+bool pdl_env(const char* name);  // diagnostics: getenv(name) != "0"
+template <typename... KArgs, typename... Args>
+cudaError_t launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t s, Args&&... args) {
+  return launch_pdl_if(true, kern, grid, block, smem, s, std::forward<Args>(args)...);
+}
+template <typename... KArgs, typename... Args>
+cudaError_t launch_pdl_if(bool use, void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t s,
+                          Args&&... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = use && pdl_enabled() ? 1 : 0;
+  return cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...);
+}
+
 // launchers (return the cudaError_t of the launch)
 cudaError_t launch_init(float4* out, float4* up4, float4* side4, int64_t m, int64_t lo,
                         int64_t nloc, const boids_params& p, uint64_t seed, cudaStream_t s);
@@ -173,7 +205,9 @@ cudaError_t launch_warm_scan(const StepArgs& a, cudaStream_t s);
 cudaError_t launch_grid(const StepArgs& a, const GridArgs& g, cudaStream_t s);
 cudaError_t launch_grid_far(const StepArgs& a, const GridArgs& g, cudaStream_t s);
 int grid_chunk();
-cudaError_t launch_warm_select(const StepArgs& a, cudaStream_t s);
+// pdl: launch k_select1 as a programmatic dependent of the scan.  Measured: a
+// gain after k_scan (C1 30 -> 25 us/step), a loss after k_sym (C3 97 -> 121).
+cudaError_t launch_warm_select(const StepArgs& a, cudaStream_t s, bool pdl = true);
 int64_t sym_capacity(int64_t nloc);
 // k_sym work-split feedback record: [0] grid, [1] items, then per CTA j
 // [2 + 3j] L0, [3 + 3j] L1, [4 + 3j] SM cycles the CTA took.

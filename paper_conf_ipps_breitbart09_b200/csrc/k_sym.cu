@@ -230,6 +230,7 @@ __global__ void __launch_bounds__(NTS, NTS == 128 ? 4 : 1)
   SymSmem<NTS>& sm = *reinterpret_cast<SymSmem<NTS>*>(smem_raw);
   __shared__ int64_t s_range[2];
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  pdl_wait();  // k_sym_prep's sp / limits (and the previous launch's feedback record)
   const long long c_start = clock64();
   const int64_t total = sym_prefix(npad / QBS, npad, QBS);
   if (warp == 0) {
@@ -515,6 +516,7 @@ __device__ __forceinline__ void sym_prep_body(const StepArgs& a, float4* __restr
 
 __global__ void __launch_bounds__(256) k_sym_prep(StepArgs a, float4* __restrict__ sp, int* __restrict__ sidx,
                                                    int64_t npad) {
+  pdl_trigger();  // k_sym may be scheduled now; it waits for this grid before reading sp
   span_begin(a, SPAN_SLOT0 + 0);
   sym_prep_body(a, sp, sidx, npad);
   span_end(a, SPAN_SLOT0 + 0);
@@ -601,6 +603,7 @@ __device__ __forceinline__ void route_body(const StepArgs& a) {
 }
 
 __global__ void __launch_bounds__(RT) k_route(StepArgs a) {
+  pdl_wait();  // k_select1's routing list
   span_begin(a, SPAN_SLOT0 + 2);
   route_body(a);
   span_end(a, SPAN_SLOT0 + 2);
@@ -634,8 +637,8 @@ cudaError_t sym_with(const StepArgs& a, float4* sp, int* sidx, const long long* 
     const char* e = getenv("BOIDS_SYM_WD4");  // diagnostics: diagonal item weight x4
     return e ? atoi(e) : 6;  // measured best of 4..16 at C3 and C4
   }();
-  k_sym<NT><<<g, NT, sizeof(SymSmem<NT>), s>>>(a, sp, sidx, npad, wd4, fb_prev, g <= SYM_FB_MAX_CTAS ? fb_cur : nullptr);
-  return cudaGetLastError();
+  return launch_pdl(k_sym<NT>, dim3(g), dim3(NT), sizeof(SymSmem<NT>), s, a, (const float4*)sp,
+                       (const int*)sidx, npad, wd4, fb_prev, g <= SYM_FB_MAX_CTAS ? fb_cur : nullptr);
 }
 
 }  // namespace
@@ -654,8 +657,7 @@ cudaError_t launch_route(const StepArgs& a, cudaStream_t s) {
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   BOIDS_PREFER_SMEM(k_route);
-  k_route<<<(unsigned)std::min<int64_t>(a.nloc, 2LL * sms), RT, 0, s>>>(a);
-  return cudaGetLastError();
+  return launch_pdl(k_route, dim3((unsigned)std::min<int64_t>(a.nloc, 2LL * sms)), dim3(RT), 0, s, a);
 }
 
 cudaError_t launch_sym_scan(const StepArgs& a, float4* sp, int* sidx, const long long* fb_prev, long long* fb_cur,

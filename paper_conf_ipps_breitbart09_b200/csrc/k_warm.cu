@@ -157,6 +157,8 @@ __device__ __forceinline__ void stamp_k(const StepArgs& a, int k) {
 
 template <int NTS>
 __global__ void __launch_bounds__(NTS, NTS == 128 ? 4 : 1) k_scan(StepArgs a, int64_t ncand, int64_t items) {
+  pdl_wait();  // k_bound's limits (think mode: the compacted query list)
+  pdl_trigger();
   if (a.qcount) {  // think mode: query slots counted on the device
     a.nq = *a.qcount;
     items = (a.nq + NTS * Q - 1) / (NTS * Q) * ncand;
@@ -364,6 +366,7 @@ __global__ void __launch_bounds__(NTS, NTS == 128 ? 4 : 1) k_scan(StepArgs a, in
 // scan, computed once per step (k_scan reads it instead of re-gathering the 8
 // previous neighbours in every CTA that shares the agent's query block).
 __global__ void __launch_bounds__(256) k_bound(StepArgs a) {
+  pdl_trigger();  // k_scan may be scheduled now; it waits for this grid before reading the limits
   const int64_t qi = (int64_t)blockIdx.x * 256 + threadIdx.x;
   if (qi >= a.nloc) return;
   const float r2 = __fmul_rn(a.p.search_radius, a.p.search_radius);
@@ -558,6 +561,7 @@ __device__ __forceinline__ void select1_body(const StepArgs& a) {
 }
 
 __global__ void __launch_bounds__(NSEL) k_select1(StepArgs a) {
+  pdl_wait();  // the scan's hit buffers
   span_begin(a, SPAN_SLOT0 + 1);
   select1_body(a);
   span_end(a, SPAN_SLOT0 + 1);
@@ -593,8 +597,7 @@ cudaError_t scan_with(const StepArgs& a, int sms, int64_t ncand, cudaStream_t s)
   const int64_t items = nqb * ncand;  // (query block, candidate) pairs; think mode: recomputed on device
   const int g = a.qcount ? scan_grid<NT>(sms)
                          : (int)std::min<int64_t>(scan_grid<NT>(sms), (items + SCAN_MIN - 1) / SCAN_MIN);
-  k_scan<NT><<<g, NT, sizeof(ScanSmem<NT>), s>>>(a, ncand, items);
-  return cudaGetLastError();
+  return launch_pdl(k_scan<NT>, dim3(g), dim3(NT), sizeof(ScanSmem<NT>), s, a, ncand, items);
 }
 
 #ifndef BOIDS_SCAN_BIG
@@ -619,12 +622,11 @@ cudaError_t launch_warm_scan(const StepArgs& a, cudaStream_t s) {
   return scan_with<128>(a, sms, ncand, s);
 }
 
-cudaError_t launch_warm_select(const StepArgs& a, cudaStream_t s) {
+cudaError_t launch_warm_select(const StepArgs& a, cudaStream_t s, bool pdl) {
   if (a.nloc <= 0) return cudaSuccess;
   if (a.think_k <= 1 && a.rlist) {
     BOIDS_PREFER_SMEM(k_select1);
-    k_select1<<<(unsigned)((a.nloc + NSEL - 1) / NSEL), NSEL, 0, s>>>(a);
-    return cudaGetLastError();
+    return launch_pdl_if(pdl, k_select1, dim3((unsigned)((a.nloc + NSEL - 1) / NSEL)), dim3(NSEL), 0, s, a);
   }
   BOIDS_PREFER_SMEM(k_select);
   k_select<<<(unsigned)((a.nloc + NSEL - 1) / NSEL), NSEL, 0, s>>>(a);

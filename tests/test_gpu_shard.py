@@ -52,11 +52,13 @@ def _emulated_run(pk, n, world, params, steps, seed=1):
             abi.boids_destroy(h)
 
 
-@pytest.mark.parametrize("mode,n,world", [(0, 3000, 2), (0, 5000, 3), (0, 1000, 8), (1, 20000, 4), (1, 777, 2)])
-def test_shard_emulation_bitidentical(boidslib, mode, n, world):
+@pytest.mark.parametrize("mode,n,world,steer", [(0, 3000, 2, 0), (0, 5000, 3, 0), (0, 1000, 8, 0), (1, 20000, 4, 0),
+                                                (1, 777, 2, 0), (0, 3000, 3, 1), (1, 5000, 2, 1)])
+def test_shard_emulation_bitidentical(boidslib, mode, n, world, steer):
+    """steer = 1: OpenSteer steering, whose smoothed accelerations live with the owner."""
     import paper_conf_ipps_breitbart09_b200 as pk
 
-    p = pk.boids_default_params(init_mode=1, search_mode=mode, world_radius=20.0)
+    p = pk.boids_default_params(init_mode=1, search_mode=mode, world_radius=20.0, steer_mode=steer)
     steps = 4
     got, got_nbr = _emulated_run(pk, n, world, p, steps)
     with pk.Flock(n, p, seed=1) as f:

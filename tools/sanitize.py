@@ -5,10 +5,11 @@ sys.path.insert(0, '.')
 import paper_conf_ipps_breitbart09_b200 as pk  # noqa: E402
 from paper_conf_ipps_breitbart09_b200 import abi  # noqa: E402
 
-for n in (1, 31, 1000, 1024):
+for n in (1, 31, 1000, 1024, 9000):
     for mode in (0, 1):
-        for kernel in ((0, 1, 2) if mode == 0 else (0,)):
-            p = pk.boids_default_params(search_mode=mode, init_mode=1, world_radius=15.0)
+        for kernel in ((0, 1, 2) if mode == 0 and n < 9000 else (0,)):
+            p = pk.boids_default_params(search_mode=mode, init_mode=1, world_radius=15.0,
+                                        steer_mode=1 if n == 1000 else 0)
             with pk.Flock(n, p, seed=3, kernel=kernel, record_steering=True) as f:
                 f.step(0.05, 3)
                 f.set_state(f.state())
