@@ -272,6 +272,32 @@ def test_config_c4_warm_sampled(pk, orc, sym):
             np.testing.assert_array_equal(g[k][ag], o[k])
 
 
+@pytest.mark.parametrize("n,search", [(300001, 0), (2500003, 1)])
+def test_large_ragged_warm_sampled(pk, orc, n, search):
+    """Beyond the bench sizes, ragged (n not a multiple of any tile or query
+    block): brute force at n = 300001 on k_sym (147 query blocks, stream-K,
+    feedback split) and the grid at n = 2.5M.  As in the C4 warm test: a cold
+    step on the oracle's initial state leaves lists, the input is replaced by a
+    jittered copy (workloads.jitter), and the warm step (bounds, window / cell
+    bounds, routing) is checked on 512 sampled agents against the oracle."""
+    p = pk.boids_default_params(init_mode=1, search_mode=search)
+    op = _oparams(orc, p)
+    ag = W.sample_agents(n, 512, seed=9)
+    s0 = orc.init(n, op, seed=2)
+    s1 = W.jitter({k: s0[k] for k in KEYS}, 0.05, seed=5)
+    with pk.Flock(n, p, seed=1, record_steering=True) as f:
+        f.set_state({k: s0[k] for k in KEYS})
+        f.step(DT, 1)
+        f.set_state(s1)
+        f.step(DT, 1)
+        g = f.state()
+        o, o_idx, _, o_F = orc.step_sample(orc.State(s1), ag, DT, op)
+        np.testing.assert_array_equal(f.neighbors()[0][ag], o_idx)
+        np.testing.assert_array_equal(f.steering()[ag], o_F)
+        for k in KEYS:
+            np.testing.assert_array_equal(g[k][ag], o[k])
+
+
 # --------------------------------------------------------------- edges
 def test_steps_zero_is_noop(pk):
     with pk.Flock(300, seed=2) as f:
