@@ -119,7 +119,7 @@ __device__ __forceinline__ void issue(GridSmem& sm, const GridArgs& g, uint32_t 
   tma_load_1d(sm.ring[s], g.spos + sm.range[r].x + off, cnt * (uint32_t)sizeof(float4), &sm.full[s]);
 }
 
-__global__ void __launch_bounds__(NTG) k_grid(StepArgs a, GridArgs g) {
+__global__ void __launch_bounds__(NTG, 5) k_grid(StepArgs a, GridArgs g) {  // 5 CTAs / SM: 3.38 -> 3.27 ms at C5 (4: 127 regs; 6: spills more, 3.33)
   __shared__ GridSmem sm;
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   if (tid == 0) {
