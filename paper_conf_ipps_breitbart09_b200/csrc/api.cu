@@ -75,6 +75,8 @@ struct boids_ctx {
   int sym_fb_par = 0;                     // which half the next launch writes
   int32_t* sym_rlist = nullptr;           // k_sym: agents routed to k_route this step [m]
   int32_t* sym_rcount = nullptr;          // ... and their number
+  unsigned long long* rpart = nullptr;    // k_route partial lists [m][16][8]
+  int32_t* rbcount = nullptr;             // k_route parts done per routed agent [m]
   bool symmetric = true;                  // BOIDS_OPT_SYMMETRIC
   bool balance = true;                    // BOIDS_OPT_BALANCE: k_sym split from the last launch's CTA times
   int32_t* pcnt = nullptr;
@@ -194,6 +196,8 @@ void free_ctx(boids_ctx* c) {
   cudaFree(c->sym_idx);
   cudaFree(c->sym_fb);
   cudaFree(c->sym_rlist);
+  cudaFree(c->rpart);
+  cudaFree(c->rbcount);
   cudaFree(c->sym_rcount);
   for (auto& r : c->recs) {
     cudaEventDestroy(r.a);
@@ -320,6 +324,8 @@ int create_impl(int64_t n, const boids_params* p, uint64_t seed, int32_t rank, i
              (rc = alloc((void**)&c->qlim, m * sizeof(float))) ||
              (rc = alloc((void**)&c->sym_rlist, m * sizeof(int32_t))) ||
              (rc = alloc((void**)&c->sym_rcount, sizeof(int32_t))) ||
+             (rc = alloc((void**)&c->rpart, (size_t)m * 16 * 8 * sizeof(unsigned long long))) ||
+             (rc = alloc((void**)&c->rbcount, (size_t)m * sizeof(int32_t))) ||
              (!shard && ((rc = alloc((void**)&c->sym_sp, sym_capacity(c->nloc) * sizeof(float4))) ||
                          (rc = alloc((void**)&c->sym_idx, sym_capacity(c->nloc) * sizeof(int32_t))) ||
                          (rc = alloc((void**)&c->sym_fb, 2 * SYM_FB_LEN * sizeof(long long)))))) {
@@ -338,6 +344,7 @@ int create_impl(int64_t n, const boids_params* p, uint64_t seed, int32_t rank, i
   if (e == cudaSuccess) e = cudaMemsetAsync(c->buf[1], 0, seg, s);
   if (e == cudaSuccess) e = cudaMemsetAsync(c->cnt, 0xFF, m * sizeof(int32_t), s);  // -1: never searched
   if (e == cudaSuccess && c->sym_fb) e = cudaMemsetAsync(c->sym_fb, 0, 2 * SYM_FB_LEN * sizeof(long long), s);
+  if (e == cudaSuccess && c->rbcount) e = cudaMemsetAsync(c->rbcount, 0, (size_t)m * sizeof(int32_t), s);
   if (e == cudaSuccess) e = cudaMemsetAsync(c->fstore, 0, m * sizeof(float4), s);
   if (e == cudaSuccess) e = cudaMemsetAsync(c->routed, 0, m, s);
   if (e == cudaSuccess) e = cudaMemsetAsync(c->nbr, 0xFF, m * 7 * sizeof(int32_t), s);
@@ -405,6 +412,8 @@ StepArgs make_args(boids_ctx* c, float dt) {
   a.routed = c->p.think_every > 1 ? c->routed : nullptr;
   a.rlist = c->sym_rlist;  // warm brute-force steps route overflowed agents to k_route
   a.rcount = c->sym_rcount;
+  a.rpart = c->rpart;
+  a.rbcount = c->rbcount;
   a.loc = c->loc_grid;
   a.acc4 = c->acc4;
   a.lstart = c->bstart;  // brute-force steps sort the queries (qperm) before any search

@@ -106,6 +106,8 @@ struct StepArgs {
                               // k_sym steps: 1 = routed to k_route by k_sym_prep
   int32_t* rlist;             // warm steps: agents finished by k_route (hit-buffer overflow, routed);
   int32_t* rcount;            // their number (zeroed before the step).  nullptr = warp re-search in k_select
+  unsigned long long* rpart;  // k_route: per routed agent, the top-8 of each candidate part [m][16][8]
+  int32_t* rbcount;           // k_route: parts finished per routed agent (zero between steps) [m]
   unsigned long long* phase;  // diagnostics: per-CTA %globaltimer stamps [grid][8], nullptr = off
   float4* acc4;               // [m] steer_mode 1: smoothed accelerations (nullptr otherwise)
   BinGrid loc;                // locality (Morton) grid of the last query sort ...

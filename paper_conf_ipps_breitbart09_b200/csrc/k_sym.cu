@@ -528,31 +528,41 @@ __global__ void __launch_bounds__(256) k_sym_prep(StepArgs a, float4* __restrict
 // them.  The CTA then finishes the agent -- list, 8th nearest (the next step's
 // warm-bound seed), steering, modification -- and k_select skips it.
 constexpr int RT = 512, RU = 16;
+constexpr int RP_MAX = 16;  // candidate parts per routed agent (few routed agents -> more CTAs each)
 __device__ __forceinline__ void route_body(const StepArgs& a) {
   __shared__ key_t wl[RT / 32][8];
+  __shared__ int s_last;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int nr = *a.rcount;
+  if (nr <= 0) return;
+  // P parts per agent so that a handful of routed agents still fills the GPU;
+  // the CTA that finishes an agent's last part merges the parts' top-8 lists
+  const int P = a.rpart ? max(1, min(RP_MAX, (int)(2 * gridDim.x / nr))) : 1;
+  const int64_t total = (int64_t)a.world * a.m;           // candidate slots (slot t = agent t)
+  const int64_t chunk = ((total + P - 1) / P + RT - 1) / RT * RT;
   const float r2 = __fmul_rn(a.p.search_radius, a.p.search_radius);
-  for (int r = blockIdx.x; r < nr; r += gridDim.x) {
+  for (int w = blockIdx.x; w < nr * P; w += gridDim.x) {
+    const int r = w / P, part = w - r * P;
     const int qi = a.rlist[r];
     const float4 me = __ldg(pos_of(a.full, a.m, a.sdiv, a.lo + qi));
     const int g = (int)(a.lo + qi);
     key_t A[8];
 #pragma unroll
     for (int s = 0; s < 8; ++s) A[s] = KEY_EMPTY;
-    // slice by slice (no per-candidate slice division); 16 independent loads in
-    // flight per thread: the candidates are L2-resident and this loop is
-    // latency-bound.  (Measured: k_fused on the compacted list instead costs
-    // 2.5-4 ms per step at C4 -- its grid is sized for all n.)
-    for (int sl = 0; sl < a.world; ++sl) {
-      const float4* base = a.full + (int64_t)sl * 2 * a.m;
-      const int jg0 = (int)((int64_t)sl * a.m);
-      for (int j0 = tid; j0 < (int)a.m; j0 += RT * RU) {
+    // slice by slice within this part (no per-candidate slice division); 16
+    // independent loads in flight per thread: the candidates are L2-resident
+    // and this loop is latency-bound
+    const int64_t c0 = part * chunk, c1 = min(total, c0 + chunk);
+    for (int64_t sl = c0 / a.m; sl * a.m < c1; ++sl) {
+      const float4* base = a.full + sl * 2 * a.m;
+      const int jg0 = (int)(sl * a.m);
+      const int jlo = (int)(max(c0, sl * a.m) - sl * a.m), jhi = (int)(min(c1, (sl + 1) * a.m) - sl * a.m);
+      for (int j0 = jlo + tid; j0 < jhi; j0 += RT * RU) {
         float4 c[RU];
 #pragma unroll
         for (int u = 0; u < RU; ++u) {
           const int j = j0 + RT * u;
-          c[u] = j < (int)a.m ? __ldg(base + j) : make_float4(__int_as_float(0x7fc00000), 0.f, 0.f, 0.f);
+          c[u] = j < jhi ? __ldg(base + j) : make_float4(__int_as_float(0x7fc00000), 0.f, 0.f, 0.f);
         }
 #pragma unroll
         for (int u = 0; u < RU; ++u) {
@@ -566,10 +576,10 @@ __device__ __forceinline__ void route_body(const StepArgs& a) {
       }
     }
 #pragma unroll
-    for (int w = 1; w < 32; w <<= 1) {
+    for (int o = 1; o < 32; o <<= 1) {
       key_t B[8];
 #pragma unroll
-      for (int s = 0; s < 8; ++s) B[s] = __shfl_xor_sync(0xffffffffu, A[s], w);
+      for (int s = 0; s < 8; ++s) B[s] = __shfl_xor_sync(0xffffffffu, A[s], o);
       merge8(A, B);
     }
     if (lane == 0)
@@ -577,26 +587,47 @@ __device__ __forceinline__ void route_body(const StepArgs& a) {
       for (int s = 0; s < 8; ++s) wl[warp][s] = A[s];
     __syncthreads();
     if (tid == 0) {
-      for (int w = 1; w < RT / 32; ++w) {
+      for (int v = 1; v < RT / 32; ++v) {
         key_t B[8];
 #pragma unroll
-        for (int s = 0; s < 8; ++s) B[s] = wl[w][s];
+        for (int s = 0; s < 8; ++s) B[s] = wl[v][s];
         merge8(A, B);
       }
-      a.nbr8[qi] = A[7] == KEY_EMPTY ? -1 : key_idx(A[7]);
-      int nb[7], cnt = 0;
+      s_last = 1;
+      if (P > 1) {  // publish this part; the last part's CTA merges all of them
 #pragma unroll
-      for (int s = 0; s < 7; ++s) {
-        nb[s] = A[s] == KEY_EMPTY ? -1 : key_idx(A[s]);
-        cnt += A[s] == KEY_EMPTY ? 0 : 1;
+        for (int s = 0; s < 8; ++s) a.rpart[((int64_t)r * RP_MAX + part) * 8 + s] = A[s];
+        __threadfence();
+        s_last = atomicAdd(a.rbcount + r, 1) == P - 1;
+        if (s_last) {
+          __threadfence();
+#pragma unroll
+          for (int s = 0; s < 8; ++s) A[s] = KEY_EMPTY;
+          for (int q = 0; q < P; ++q) {
+            key_t B[8];
+#pragma unroll
+            for (int s = 0; s < 8; ++s) B[s] = __ldcg(a.rpart + ((int64_t)r * RP_MAX + q) * 8 + s);
+            merge8(A, B);
+          }
+          a.rbcount[r] = 0;  // ready for the next step
+        }
       }
+      if (s_last) {
+        a.nbr8[qi] = A[7] == KEY_EMPTY ? -1 : key_idx(A[7]);
+        int nb[7], cnt = 0;
 #pragma unroll
-      for (int s = 0; s < 7; ++s) a.nbr[qi * 7 + s] = nb[s];
-      a.cnt[qi] = cnt;
-      const float4 f4 = __ldg(fwd_of(a.full, a.m, a.sdiv, a.lo + qi));
-      const V3 F = steer_agent(a, v3(me), v3(f4), nb, cnt);
-      if (a.think_k > 1) a.fstore[qi] = make_float4(F.x, F.y, F.z, 0.f);  // think mode: a warm thinker
-      modify_agent(a, qi, v3(me), f4, F);
+        for (int s = 0; s < 7; ++s) {
+          nb[s] = A[s] == KEY_EMPTY ? -1 : key_idx(A[s]);
+          cnt += A[s] == KEY_EMPTY ? 0 : 1;
+        }
+#pragma unroll
+        for (int s = 0; s < 7; ++s) a.nbr[qi * 7 + s] = nb[s];
+        a.cnt[qi] = cnt;
+        const float4 f4 = __ldg(fwd_of(a.full, a.m, a.sdiv, a.lo + qi));
+        const V3 F = steer_agent(a, v3(me), v3(f4), nb, cnt);
+        if (a.think_k > 1) a.fstore[qi] = make_float4(F.x, F.y, F.z, 0.f);  // think mode: a warm thinker
+        modify_agent(a, qi, v3(me), f4, F);
+      }
     }
     __syncthreads();
   }
