@@ -141,9 +141,20 @@ __global__ void __launch_bounds__(SCAN_T) k_bin_scan(int* __restrict__ cnt, int*
   extern __shared__ int sh[];  // C + C / 32 words, then (items) rows + rows / 32 + 1 words
   __shared__ int warp_sums[SCAN_T / 32];
   const int tid = threadIdx.x;
-  for (int i = tid; i < C; i += SCAN_T) {
-    sh[i + (i >> 5)] = cnt[i];
-    cnt[i] = 0;
+  // one CTA reads all C counts: 8 loads in flight per thread, or the loop waits
+  // one L2 round trip per element (C5: 39k cells, 42 -> a few us)
+  for (int i0 = tid; i0 < C; i0 += SCAN_T * 8) {
+    int v[8];
+#pragma unroll
+    for (int k = 0; k < 8; ++k) v[k] = i0 + k * SCAN_T < C ? cnt[i0 + k * SCAN_T] : 0;
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      const int i = i0 + k * SCAN_T;
+      if (i < C) {
+        sh[i + (i >> 5)] = v[k];
+        cnt[i] = 0;
+      }
+    }
   }
   __syncthreads();
   const int total = block_scan_runs(sh, C, warp_sums);
