@@ -75,6 +75,7 @@ struct boids_ctx {
   int sym_fb_par = 0;                     // which half the next launch writes
   int32_t* sym_rlist = nullptr;           // k_sym: agents routed to k_route this step [m]
   int32_t* sym_rcount = nullptr;          // ... and their number
+  int32_t* growbuf = nullptr;             // grid mode: row scratch of the many-CTA binning scan
   unsigned long long* rpart = nullptr;    // k_route partial lists [m][16][8]
   int32_t* rbcount = nullptr;             // k_route parts done per routed agent [m]
   bool symmetric = true;                  // BOIDS_OPT_SYMMETRIC
@@ -196,6 +197,7 @@ void free_ctx(boids_ctx* c) {
   cudaFree(c->sym_idx);
   cudaFree(c->sym_fb);
   cudaFree(c->sym_rlist);
+  cudaFree(c->growbuf);
   cudaFree(c->rpart);
   cudaFree(c->rbcount);
   cudaFree(c->sym_rcount);
@@ -310,6 +312,7 @@ int create_impl(int64_t n, const boids_params* p, uint64_t seed, int32_t rank, i
         (rc = alloc((void**)&c->gqstart, (C + 1) * sizeof(int32_t))) ||
         (rc = alloc((void**)&c->gitems, (size_t)(C + m / grid_chunk() + 2) * sizeof(int4))) ||
         (rc = alloc((void**)&c->gnitems, sizeof(int32_t))) ||
+        (rc = alloc((void**)&c->growbuf, (size_t)2 * (C / c->sgrid.dim[0] + 1) * sizeof(int32_t))) ||
         (rc = alloc((void**)&c->counter, sizeof(int32_t))) ||
         (rc = alloc((void**)&c->sym_rlist, m * sizeof(int32_t))) ||
         (rc = alloc((void**)&c->sym_rcount, sizeof(int32_t))) ||
@@ -443,12 +446,12 @@ int one_step(boids_ctx* c, float dt) {
            cudaError_t e = launch_bin(a.full, c->m, a.sdiv, 0, slots, c->sgrid, c->gcellrank, c->gcnt, c->gstart,
                                       c->spos, one ? c->qperm : nullptr, 0, c->stream, nullptr,
                                       one ? c->gitems : nullptr, one ? c->gnitems : nullptr, chunk,
-                                      one ? c->counter : nullptr);
+                                      one ? c->counter : nullptr, 1, 0, c->growbuf);
            if (e == cudaSuccess && !one)
              e = launch_bin(a.full, c->m, a.sdiv, c->lo, c->nloc, c->sgrid, c->gcellrank, c->gcnt, c->gqstart,
                             nullptr, c->qperm, (int)c->lo, c->stream, nullptr, c->gitems, c->gnitems, chunk,
                             c->counter,
-                            c->p.think_every, c->step_index);
+                            c->p.think_every, c->step_index, c->growbuf);
            return e;
          }, one ? 3 : 6)))
       return rc;

@@ -187,7 +187,8 @@ cudaError_t launch_fill_phantoms(float4* seg_base, int64_t m, int64_t nloc, int6
 cudaError_t launch_bin(const float4* full, int64_t m, const SliceDiv& sd, int64_t j0, int64_t count, const BinGrid& g,
                        int2* cellrank, int* cnt, int* start, float4* spos, int* perm, int perm_base,
                        cudaStream_t s, int* launches, int4* items = nullptr, int* nitems = nullptr, int chunk = 1,
-                       int* counter = nullptr, int think_k = 1, int64_t think_t = 0);
+                       int* counter = nullptr, int think_k = 1, int64_t think_t = 0,
+                       int* rowbuf = nullptr);  // [2 * rows] scratch: large grids scan on many CTAs
 BinGrid make_locality_grid(int64_t n, const boids_params& p);
 BinGrid make_search_grid(const boids_params& p);
 cudaError_t launch_fill_nan(float4* p, int64_t count, cudaStream_t s);

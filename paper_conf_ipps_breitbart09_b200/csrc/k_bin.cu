@@ -92,11 +92,12 @@ __device__ __forceinline__ int block_scan_runs(int* sh, int C, int* warp_sums) {
 // chunk-sized items of its own; a run spans at most MAX_SPAN cells.  Item = (first query slot, count, first cell,
 // last x - first x).  One thread per row; pass 0 counts, pass 1 writes.
 constexpr int MAX_SPAN = 8;  // cells per item: wider runs scan more candidates per query (think mode)
-__device__ __forceinline__ int row_items(const int* sh, int C, int total, int row, int D, int chunk, int4* out) {
+template <class StartOf>
+__device__ __forceinline__ int row_items_g(StartOf start_of, int C, int total, int row, int D, int chunk, int4* out) {
   int n = 0, acc = 0, xs = -1, q0 = 0;
   auto cnt_of = [&](int c, int& s0) {
-    s0 = sh[c + (c >> 5)];
-    const int s1 = c + 1 < C ? sh[(c + 1) + ((c + 1) >> 5)] : total;
+    s0 = start_of(c);
+    const int s1 = c + 1 < C ? start_of(c + 1) : total;
     return s1 - s0;
   };
   auto close = [&](int xe) {
@@ -129,6 +130,9 @@ __device__ __forceinline__ int row_items(const int* sh, int C, int total, int ro
   }
   close(D - 1);
   return n;
+}
+__device__ __forceinline__ int row_items(const int* sh, int C, int total, int row, int D, int chunk, int4* out) {
+  return row_items_g([&](int c) { return sh[c + (c >> 5)]; }, C, total, row, D, chunk, out);
 }
 
 // Exclusive scan of cnt[0..C) into start[0..C], start[C] = total; zeroes cnt.
@@ -173,6 +177,98 @@ __global__ void __launch_bounds__(SCAN_T) k_bin_scan(int* __restrict__ cnt, int*
   }
 }
 
+// ---- the same scan + work items over many CTAs, for large grids (C5: 39k
+// cells; one CTA took 42 us): one warp per grid row of D cells.
+//   rows1: row sums and the row's item count (rows are independent: an item
+//          never crosses a row);
+//   rows2: one CTA scans the row sums and item counts (rows << cells);
+//   rows3: cell starts = row base + in-row prefix, the row's items, cnt zeroed.
+constexpr int RW_WARPS = 8;
+constexpr int RW_MAXD = 256;  // cells per row handled this way (else the one-CTA scan)
+__device__ __forceinline__ int row_counts_to_smem(const int* cnt, int row, int D, int* rs, int lane) {
+  int sum = 0;
+  for (int x0 = 0; x0 < D; x0 += 32) {  // exclusive in-row prefix into rs[0..D], rs[D] = row total
+    const int x = x0 + lane;
+    const int k = x < D ? cnt[row * D + x] : 0;
+    int v = k;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int y = __shfl_up_sync(0xffffffffu, v, o);
+      if (lane >= o) v += y;
+    }
+    if (x < D) rs[x] = sum + v - k;
+    sum += __shfl_sync(0xffffffffu, v, 31);
+  }
+  if (lane == 0) rs[D] = sum;
+  __syncwarp();
+  return sum;
+}
+
+__global__ void __launch_bounds__(RW_WARPS * 32) k_bin_rows1(const int* __restrict__ cnt, int rows, int D,
+                                                             int chunk, int* __restrict__ rowsum,
+                                                             int* __restrict__ rowitems) {
+  __shared__ int rs[RW_WARPS][RW_MAXD + 1];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int row = blockIdx.x * RW_WARPS + warp;
+  if (row >= rows) return;
+  const int sum = row_counts_to_smem(cnt, row, D, rs[warp], lane);
+  if (lane == 0) {
+    rowsum[row] = sum;
+    // row_items over a (C = D, total = sum) view of this row's starts
+    const int* r = rs[warp];
+    if (rowitems) rowitems[row] = row_items_g([&](int c) { return r[c]; }, D, sum, 0, D, chunk, nullptr);
+  }
+}
+
+__global__ void __launch_bounds__(SCAN_T) k_bin_rows2(int* __restrict__ rowsum, int* __restrict__ rowitems, int rows,
+                                                     int* __restrict__ start, int C, int* __restrict__ nitems,
+                                                     int* __restrict__ counter) {
+  extern __shared__ int sh[];  // 2 x (rows + rows / 32 + 1)
+  __shared__ int warp_sums[SCAN_T / 32];
+  int* a = sh;
+  int* b = sh + rows + (rows >> 5) + 1;
+  for (int r = threadIdx.x; r < rows; r += SCAN_T) {
+    a[r + (r >> 5)] = rowsum[r];
+    if (rowitems) b[r + (r >> 5)] = rowitems[r];
+  }
+  __syncthreads();
+  const int total = block_scan_runs(a, rows, warp_sums);
+  const int n = rowitems ? block_scan_runs(b, rows, warp_sums) : 0;
+  for (int r = threadIdx.x; r < rows; r += SCAN_T) {
+    rowsum[r] = a[r + (r >> 5)];  // now the row's base
+    if (rowitems) rowitems[r] = b[r + (r >> 5)];
+  }
+  if (threadIdx.x == 0) {
+    start[C] = total;
+    if (nitems) *nitems = n;
+    if (counter) *counter = 0;
+  }
+}
+
+__global__ void __launch_bounds__(RW_WARPS * 32) k_bin_rows3(int* __restrict__ cnt, int rows, int D, int chunk,
+                                                             const int* __restrict__ rowbase,
+                                                             const int* __restrict__ itembase,
+                                                             int* __restrict__ start, int4* __restrict__ items) {
+  __shared__ int rs[RW_WARPS][RW_MAXD + 1];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int row = blockIdx.x * RW_WARPS + warp;
+  if (row >= rows) return;
+  const int sum = row_counts_to_smem(cnt, row, D, rs[warp], lane);
+  const int base = rowbase[row];
+  for (int x = lane; x < D; x += 32) {
+    start[row * D + x] = base + rs[warp][x];
+    cnt[row * D + x] = 0;
+  }
+  if (items && lane == 0) {
+    // the row's starts in absolute terms, then the same greedy items as the one-CTA scan
+    int* r = rs[warp];
+    for (int x = 0; x <= D; ++x) r[x] += base;
+    int4* out = items + itembase[row];
+    const int n = row_items_g([&](int c) { return r[c]; }, D, base + sum, 0, D, chunk, out);
+    for (int k = 0; k < n; ++k) out[k].z += row * D;  // cell index: row-local -> global
+  }
+}
+
 __global__ void k_bin_scatter(const float4* __restrict__ full, int64_t m, SliceDiv sd, int64_t j0, int64_t count,
                               const int2* __restrict__ cellrank, const int* __restrict__ start,
                               float4* __restrict__ spos, int* __restrict__ perm, int perm_base) {
@@ -192,7 +288,7 @@ __global__ void k_bin_scatter(const float4* __restrict__ full, int64_t m, SliceD
 cudaError_t launch_bin(const float4* full, int64_t m, const SliceDiv& sd, int64_t j0, int64_t count, const BinGrid& g,
                        int2* cellrank, int* cnt, int* start, float4* spos, int* perm, int perm_base,
                        cudaStream_t s, int* launches, int4* items, int* nitems, int chunk, int* counter,
-                       int think_k, int64_t think_t) {
+                       int think_k, int64_t think_t, int* rowbuf) {
   const unsigned blocks = (unsigned)((count + 255) / 256);
   const int rows = g.cells / g.dim[0];
   const size_t shm = (size_t)(g.cells + g.cells / 32 + 1 + (items ? rows + rows / 32 + 1 : 0)) * sizeof(int);
@@ -211,8 +307,26 @@ cudaError_t launch_bin(const float4* full, int64_t m, const SliceDiv& sd, int64_
                                      spos == nullptr ? think_k : 1, think_t);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return e;
-  k_bin_scan<<<1, SCAN_T, shm, s>>>(cnt, start, g.cells, items, nitems, chunk, counter, g.dim[0]);
-  if ((e = cudaGetLastError()) != cudaSuccess) return e;
+  const int D = g.dim[0];
+  if (rowbuf && g.cells > 16384 && D <= RW_MAXD && g.cells % D == 0) {  // large grid: many CTAs
+    const unsigned rb = (unsigned)((rows + RW_WARPS - 1) / RW_WARPS);
+    int* rowsum = rowbuf;
+    int* rowit = items ? rowbuf + rows : nullptr;
+    k_bin_rows1<<<rb, RW_WARPS * 32, 0, s>>>(cnt, rows, D, chunk, rowsum, rowit);
+    if ((e = cudaGetLastError()) != cudaSuccess) return e;
+    const size_t shm2 = (size_t)2 * (rows + rows / 32 + 1) * sizeof(int);
+    if (shm2 > 48 * 1024 &&
+        (e = cudaFuncSetAttribute(k_bin_rows2, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)shm2)) != cudaSuccess)
+      return e;
+    k_bin_rows2<<<1, SCAN_T, shm2, s>>>(rowsum, rowit, rows, start, g.cells, nitems, counter);
+    if ((e = cudaGetLastError()) != cudaSuccess) return e;
+    k_bin_rows3<<<rb, RW_WARPS * 32, 0, s>>>(cnt, rows, D, chunk, rowsum, rowit, start, items);
+    if ((e = cudaGetLastError()) != cudaSuccess) return e;
+    if (launches) *launches += 2;
+  } else {
+    k_bin_scan<<<1, SCAN_T, shm, s>>>(cnt, start, g.cells, items, nitems, chunk, counter, g.dim[0]);
+    if ((e = cudaGetLastError()) != cudaSuccess) return e;
+  }
   k_bin_scatter<<<blocks, 256, 0, s>>>(full, m, sd, j0, count, cellrank, start, spos, perm, perm_base);
   if (launches) *launches += 3;
   return cudaGetLastError();
