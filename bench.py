@@ -123,6 +123,29 @@ def cpu_oracle_rate(cfg: W.Config, agents: int, seed: int = 1):
     return len(ag) / dt, len(ag), dt
 
 
+def cpu_oracle_rate_threads(cfg: W.Config, agents_per_thread: int, threads: int, seed: int = 1):
+    """The same oracle over all host cores: the seeded sample split across
+    `threads` Python threads, each calling the C oracle (ctypes releases the GIL)
+    on its own slice of agents (the per-agent functions
+    partitioned over the cores, no GPU involved)."""
+    import threading
+
+    import oracle
+
+    p = oracle.default_params(init_mode=cfg.init_mode, search_mode=cfg.search_mode)
+    s = oracle.init(cfg.n, p, seed=seed)
+    ag = W.sample_agents(cfg.n, min(cfg.n, agents_per_thread * threads), seed=seed)
+    parts = np.array_split(ag, threads)
+    ts = [threading.Thread(target=oracle.step_sample, args=(s, part, float(W.DT), p)) for part in parts]
+    t = time.perf_counter()
+    for th in ts:
+        th.start()
+    for th in ts:
+        th.join()
+    dt = time.perf_counter() - t
+    return len(ag) / dt, len(ag), dt
+
+
 def cpu_sample_size(cfg: W.Config, seconds: float) -> int:
     """Agents per sample for ~`seconds` of oracle work (about 5 ns per candidate pair)."""
     return int(max(64, min(cfg.n, seconds / (5e-9 * cfg.n))))
@@ -399,6 +422,12 @@ def main():
         cpu = {"value": rate, "unit": UNIT, "cores": 1, "kind": "oracle",
                "sample": f"{agents} of {cfg.n} agents x 1 step (seeded sample of the config's initial state; "
                          f"each agent a full O(n) search + steer + modify), {secs:.1f} s single-threaded"}
+        ncores = len(os.sched_getaffinity(0)) if hasattr(os, "sched_getaffinity") else (os.cpu_count() or 1)
+        if ncores > 1:
+            r_all, a_all, s_all = cpu_oracle_rate_threads(cfg, max(16, m // 4), ncores)
+            cpu["all_cores"] = {"value": r_all, "unit": UNIT, "cores": ncores, "kind": "oracle",
+                                "sample": f"{a_all} sampled agents x 1 step split over {ncores} threads, "
+                                          f"{s_all:.1f} s"}
 
     if rank == 0:
         line = {
