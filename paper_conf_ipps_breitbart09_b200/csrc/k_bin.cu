@@ -91,9 +91,14 @@ __device__ __forceinline__ int block_scan_runs(int* sh, int C, int* warp_sums) {
 // `chunk` agents together; a cell with more than `chunk` agents is split into
 // chunk-sized items of its own; a run spans at most MAX_SPAN cells.  Item = (first query slot, count, first cell,
 // last x - first x).  One thread per row; pass 0 counts, pass 1 writes.
-constexpr int MAX_SPAN = 8;  // cells per item: wider runs scan more candidates per query (think mode)
+constexpr int MAX_SPAN = 8;  // cells per item: wider runs scan more candidates per query
+#ifndef BOIDS_THINK_SPAN
+#define BOIDS_THINK_SPAN 64
+#endif
+constexpr int THINK_SPAN = BOIDS_THINK_SPAN;  // ... in think mode: whole rows (C5 think 10: span 1 / 2 / 4 / 8 / 34 -> 5.77 / 3.99 / 3.18 / 2.90 / 2.71 ms; per-item cost dominates)
 template <class StartOf>
-__device__ __forceinline__ int row_items_g(StartOf start_of, int C, int total, int row, int D, int chunk, int4* out) {
+__device__ __forceinline__ int row_items_g(StartOf start_of, int C, int total, int row, int D, int chunk, int4* out,
+                                           int span = MAX_SPAN) {
   int n = 0, acc = 0, xs = -1, q0 = 0;
   auto cnt_of = [&](int c, int& s0) {
     s0 = start_of(c);
@@ -120,7 +125,7 @@ __device__ __forceinline__ int row_items_g(StartOf start_of, int C, int total, i
         ++n;
       }
     } else {
-      if (acc + k > chunk || (xs >= 0 && x - xs >= MAX_SPAN)) close(x - 1);
+      if (acc + k > chunk || (xs >= 0 && x - xs >= span)) close(x - 1);
       if (xs < 0) {
         xs = x;
         q0 = s0;
@@ -131,8 +136,9 @@ __device__ __forceinline__ int row_items_g(StartOf start_of, int C, int total, i
   close(D - 1);
   return n;
 }
-__device__ __forceinline__ int row_items(const int* sh, int C, int total, int row, int D, int chunk, int4* out) {
-  return row_items_g([&](int c) { return sh[c + (c >> 5)]; }, C, total, row, D, chunk, out);
+__device__ __forceinline__ int row_items(const int* sh, int C, int total, int row, int D, int chunk, int4* out,
+                                         int span) {
+  return row_items_g([&](int c) { return sh[c + (c >> 5)]; }, C, total, row, D, chunk, out, span);
 }
 
 // Exclusive scan of cnt[0..C) into start[0..C], start[C] = total; zeroes cnt.
@@ -141,7 +147,7 @@ __device__ __forceinline__ int row_items(const int* sh, int C, int total, int ro
 // items[0..*nitems), and the grid kernel's work counter is reset.
 __global__ void __launch_bounds__(SCAN_T) k_bin_scan(int* __restrict__ cnt, int* __restrict__ start, int C,
                                                     int4* __restrict__ items, int* __restrict__ nitems, int chunk,
-                                                    int* __restrict__ counter, int D) {
+                                                    int* __restrict__ counter, int D, int span) {
   extern __shared__ int sh[];  // C + C / 32 words, then (items) rows + rows / 32 + 1 words
   __shared__ int warp_sums[SCAN_T / 32];
   const int tid = threadIdx.x;
@@ -167,10 +173,10 @@ __global__ void __launch_bounds__(SCAN_T) k_bin_scan(int* __restrict__ cnt, int*
   if (!items) return;
   const int rows = C / D;
   int* rc = sh + C + (C >> 5) + 1;
-  for (int r = tid; r < rows; r += SCAN_T) rc[r + (r >> 5)] = row_items(sh, C, total, r, D, chunk, nullptr);
+  for (int r = tid; r < rows; r += SCAN_T) rc[r + (r >> 5)] = row_items(sh, C, total, r, D, chunk, nullptr, span);
   __syncthreads();
   const int n = block_scan_runs(rc, rows, warp_sums);
-  for (int r = tid; r < rows; r += SCAN_T) row_items(sh, C, total, r, D, chunk, items + rc[r + (r >> 5)]);
+  for (int r = tid; r < rows; r += SCAN_T) row_items(sh, C, total, r, D, chunk, items + rc[r + (r >> 5)], span);
   if (tid == 0) {
     *nitems = n;
     *counter = 0;
@@ -206,7 +212,7 @@ __device__ __forceinline__ int row_counts_to_smem(const int* cnt, int row, int D
 
 __global__ void __launch_bounds__(RW_WARPS * 32) k_bin_rows1(const int* __restrict__ cnt, int rows, int D,
                                                              int chunk, int* __restrict__ rowsum,
-                                                             int* __restrict__ rowitems) {
+                                                             int* __restrict__ rowitems, int span) {
   __shared__ int rs[RW_WARPS][RW_MAXD + 1];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int row = blockIdx.x * RW_WARPS + warp;
@@ -216,7 +222,7 @@ __global__ void __launch_bounds__(RW_WARPS * 32) k_bin_rows1(const int* __restri
     rowsum[row] = sum;
     // row_items over a (C = D, total = sum) view of this row's starts
     const int* r = rs[warp];
-    if (rowitems) rowitems[row] = row_items_g([&](int c) { return r[c]; }, D, sum, 0, D, chunk, nullptr);
+    if (rowitems) rowitems[row] = row_items_g([&](int c) { return r[c]; }, D, sum, 0, D, chunk, nullptr, span);
   }
 }
 
@@ -248,7 +254,8 @@ __global__ void __launch_bounds__(SCAN_T) k_bin_rows2(int* __restrict__ rowsum, 
 __global__ void __launch_bounds__(RW_WARPS * 32) k_bin_rows3(int* __restrict__ cnt, int rows, int D, int chunk,
                                                              const int* __restrict__ rowbase,
                                                              const int* __restrict__ itembase,
-                                                             int* __restrict__ start, int4* __restrict__ items) {
+                                                             int* __restrict__ start, int4* __restrict__ items,
+                                                             int span) {
   __shared__ int rs[RW_WARPS][RW_MAXD + 1];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int row = blockIdx.x * RW_WARPS + warp;
@@ -264,7 +271,7 @@ __global__ void __launch_bounds__(RW_WARPS * 32) k_bin_rows3(int* __restrict__ c
     int* r = rs[warp];
     for (int x = 0; x <= D; ++x) r[x] += base;
     int4* out = items + itembase[row];
-    const int n = row_items_g([&](int c) { return r[c]; }, D, base + sum, 0, D, chunk, out);
+    const int n = row_items_g([&](int c) { return r[c]; }, D, base + sum, 0, D, chunk, out, span);
     for (int k = 0; k < n; ++k) out[k].z += row * D;  // cell index: row-local -> global
   }
 }
@@ -291,13 +298,16 @@ cudaError_t launch_bin(const float4* full, int64_t m, const SliceDiv& sd, int64_
                        int think_k, int64_t think_t, int* rowbuf) {
   const unsigned blocks = (unsigned)((count + 255) / 256);
   const int rows = g.cells / g.dim[0];
+  // think mode: items hold only this step's thinkers (1/k of the agents); longer
+  // runs stream more candidates per query but amortise each item's fixed cost
+  const int span = think_k > 1 ? THINK_SPAN : MAX_SPAN;
   const size_t shm = (size_t)(g.cells + g.cells / 32 + 1 + (items ? rows + rows / 32 + 1 : 0)) * sizeof(int);
   if (shm > 48 * 1024) {
     cudaError_t e = cudaFuncSetAttribute(k_bin_scan, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)shm);
     if (e != cudaSuccess) return e;
   }
   if (count <= 0) {  // still publish an empty binning (starts, items, counter)
-    k_bin_scan<<<1, SCAN_T, shm, s>>>(cnt, start, g.cells, items, nitems, chunk, counter, g.dim[0]);
+    k_bin_scan<<<1, SCAN_T, shm, s>>>(cnt, start, g.cells, items, nitems, chunk, counter, g.dim[0], span);
     return cudaGetLastError();
   }
   BOIDS_PREFER_SMEM(k_bin_count);
@@ -312,7 +322,7 @@ cudaError_t launch_bin(const float4* full, int64_t m, const SliceDiv& sd, int64_
     const unsigned rb = (unsigned)((rows + RW_WARPS - 1) / RW_WARPS);
     int* rowsum = rowbuf;
     int* rowit = items ? rowbuf + rows : nullptr;
-    k_bin_rows1<<<rb, RW_WARPS * 32, 0, s>>>(cnt, rows, D, chunk, rowsum, rowit);
+    k_bin_rows1<<<rb, RW_WARPS * 32, 0, s>>>(cnt, rows, D, chunk, rowsum, rowit, span);
     if ((e = cudaGetLastError()) != cudaSuccess) return e;
     const size_t shm2 = (size_t)2 * (rows + rows / 32 + 1) * sizeof(int);
     if (shm2 > 48 * 1024 &&
@@ -320,11 +330,11 @@ cudaError_t launch_bin(const float4* full, int64_t m, const SliceDiv& sd, int64_
       return e;
     k_bin_rows2<<<1, SCAN_T, shm2, s>>>(rowsum, rowit, rows, start, g.cells, nitems, counter);
     if ((e = cudaGetLastError()) != cudaSuccess) return e;
-    k_bin_rows3<<<rb, RW_WARPS * 32, 0, s>>>(cnt, rows, D, chunk, rowsum, rowit, start, items);
+    k_bin_rows3<<<rb, RW_WARPS * 32, 0, s>>>(cnt, rows, D, chunk, rowsum, rowit, start, items, span);
     if ((e = cudaGetLastError()) != cudaSuccess) return e;
     if (launches) *launches += 2;
   } else {
-    k_bin_scan<<<1, SCAN_T, shm, s>>>(cnt, start, g.cells, items, nitems, chunk, counter, g.dim[0]);
+    k_bin_scan<<<1, SCAN_T, shm, s>>>(cnt, start, g.cells, items, nitems, chunk, counter, g.dim[0], span);
     if ((e = cudaGetLastError()) != cudaSuccess) return e;
   }
   k_bin_scatter<<<blocks, 256, 0, s>>>(full, m, sd, j0, count, cellrank, start, spos, perm, perm_base);
