@@ -16,6 +16,14 @@ for n in (1, 31, 1000, 1024, 9000):
                 f.step(0.05, 2)
                 f.neighbors(), f.steering(), f.sync()
     print("ok", n, flush=True)
+# grid with the default world: 39k search cells -> the many-CTA binning scan;
+# think mode (whole-row items)
+for think in (1, 3):
+    p = pk.boids_default_params(search_mode=1, init_mode=1, think_every=think)
+    with pk.Flock(3000, p, seed=4) as f:
+        f.step(0.05, 4)
+        f.sync()
+print("ok grid-large")
 # shard handles (emulated 2-rank all-gather is in tests; here one rank of 2)
 h = abi.boids_create_shard(1000, pk.boids_default_params(), 1, 1, 2)
 abi.boids_step_shard(h, 0.05)
