@@ -42,6 +42,21 @@ constexpr int CT = 256;         // candidates per tile (<= 4 KB bulk copy)
 constexpr int STAGES = 3;
 constexpr int U = 4;
 constexpr int FAR_MAX = 16;  // queries per item routed to k_grid_far
+// Query slot of (warp, q, lane).  Round-robin over the warps (BOIDS_GRID_RR=1):
+// an item with fewer than QBG queries still keeps every warp working, at the
+// cost of computing the padded slots; blocked (0): a warp's 4 x 32 queries are
+// consecutive and warps past the item's queries only keep the ring protocol
+// (measured: round-robin C5 4.13 vs blocked 3.25 ms/step -- the padded slots cost
+// more than the idle warps).
+#ifndef BOIDS_GRID_RR
+#define BOIDS_GRID_RR 0
+#endif
+__device__ __forceinline__ int qslot(int warp, int q, int lane) {
+  return BOIDS_GRID_RR ? q * NTG + warp * 32 + lane : warp * 32 * Q + q * 32 + lane;
+}
+__device__ __forceinline__ bool warp_has_queries(int warp, int qn) {
+  return BOIDS_GRID_RR ? warp * 32 < qn : warp * 32 * Q < qn;
+}
 
 struct __align__(16) GridSmem {
   float4 ring[STAGES][CT];
@@ -163,7 +178,7 @@ __global__ void __launch_bounds__(NTG, 5) k_grid(StepArgs a, GridArgs g) {  // 5
     int64_t qloc[Q];
 #pragma unroll
     for (int q = 0; q < Q; ++q) {
-      const int slot = warp * 32 * Q + q * 32 + lane;
+      const int slot = qslot(warp, q, lane);
       const int64_t qi = slot < qn ? (int64_t)__ldg(g.qperm + qs0 + slot) : a.nloc;
       qloc[q] = qi;
       gq[q] = (int)(a.lo + qi);
@@ -265,7 +280,7 @@ __global__ void __launch_bounds__(NTG, 5) k_grid(StepArgs a, GridArgs g) {  // 5
       const float4* tile = sm.ring[s];
       const int cnt = tile_count(sm, r, off);
       // warps without queries in this item only keep the ring protocol
-      for (int c = 0; c < (warp * 32 * Q < qn ? cnt : 0); c += U) {
+      for (int c = 0; c < (warp_has_queries(warp, qn) ? cnt : 0); c += U) {
         float4 cc[U];
         if (c + U <= cnt) {
 #pragma unroll
@@ -303,7 +318,7 @@ __global__ void __launch_bounds__(NTG, 5) k_grid(StepArgs a, GridArgs g) {  // 5
 #pragma unroll
             for (int q = 0; q < Q; ++q)
               if (d[q][u] <= lim[q] && j != gq[q])
-                lim[q] = fminf(lim[q], insert_smem7(&sm.lists[warp * 32 * Q + q * 32 + lane], QBG,
+                lim[q] = fminf(lim[q], insert_smem7(&sm.lists[qslot(warp, q, lane)], QBG,
                                                     make_key(d[q][u], j)));
           }
           limc = fmaxf(fmaxf(lim[0], lim[1]), fmaxf(lim[2], lim[3]));
@@ -322,7 +337,7 @@ __global__ void __launch_bounds__(NTG, 5) k_grid(StepArgs a, GridArgs g) {  // 5
     __syncwarp();
 #pragma unroll
     for (int q = 0; q < Q; ++q) {
-      const int slot = warp * 32 * Q + q * 32 + lane;
+      const int slot = qslot(warp, q, lane);
       if (slot < qn && qloc[q] < a.nloc) {
         key_t A[7];
 #pragma unroll
