@@ -46,6 +46,9 @@ constexpr int CT = 128;     // candidates per tile
 // ring a warp can run STAGES-1 tiles ahead, so each warp's hot tiles only cost
 // that warp.
 constexpr int STAGES = BOIDS_SYM_STAGES;
+// 256-thread CTAs run two per SM: the ring shrinks so two fit in shared memory
+template <int NT>
+__host__ __device__ constexpr int sym_stages() { return NT == 256 ? 12 : STAGES; }
 constexpr int U = 4;        // candidates per warp vote
 constexpr int WB = Q * U * 32;  // records per warp buffer: one vote group's maximum per side
 
@@ -57,11 +60,11 @@ struct __align__(8) Rec {
 
 template <int NT>
 struct __align__(16) SymSmem {
-  float4 ring[STAGES][CT];
-  int ridx[STAGES][CT];
+  float4 ring[sym_stages<NT>()][CT];
+  int ridx[sym_stages<NT>()][CT];
   Rec rec[NT / 32][WB];
-  uint64_t full[STAGES];
-  int rel[STAGES];  // warps done with the tile in the stage (the last one refills it)
+  uint64_t full[sym_stages<NT>()];
+  int rel[sym_stages<NT>()];  // warps done with the tile in the stage (the last one refills it)
 };
 
 // 8 records per lane per round: the atomics' round trips overlap.
@@ -222,10 +225,10 @@ __device__ __forceinline__ TileDesc tile_desc(int k, int64_t L0, int64_t L1, int
 }
 
 template <int NTS>
-__global__ void __launch_bounds__(NTS, NTS == 128 ? 4 : 1)
+__global__ void __launch_bounds__(NTS, NTS == 128 ? 4 : (NTS == 256 ? 2 : 1))
     k_sym(StepArgs a, const float4* __restrict__ sp, const int* __restrict__ sidx, int64_t npad, int wd4,
           const long long* __restrict__ fb_prev, long long* __restrict__ fb_cur) {
-  constexpr int QBS = NTS * Q, NW = NTS / 32;
+  constexpr int QBS = NTS * Q, NW = NTS / 32, SST = sym_stages<NTS>();
   extern __shared__ __align__(16) unsigned char smem_raw[];
   SymSmem<NTS>& sm = *reinterpret_cast<SymSmem<NTS>*>(smem_raw);
   __shared__ int64_t s_range[2];
@@ -247,14 +250,14 @@ __global__ void __launch_bounds__(NTS, NTS == 128 ? 4 : 1)
   __syncthreads();
   const int64_t L0 = s_range[0], L1 = s_range[1];
   const int ntiles = L1 > L0 ? (int)((L1 + CT - 1) / CT - L0 / CT) : 0;
-  // Ring protocol: stage s = k % STAGES holds tile k.  full[s] completes when the
+  // Ring protocol: stage s = k % SST holds tile k.  full[s] completes when the
   // tile's bytes land (TMA complete_tx).  Each warp, when done with tile k,
   // increments rel[s]; the LAST of the NW warps refills the stage with tile
-  // k + STAGES.  So the refill waits only for the slowest warp on that tile and
-  // no warp is the dedicated producer: warps drift up to STAGES - 1 tiles apart.
+  // k + SST.  So the refill waits only for the slowest warp on that tile and
+  // no warp is the dedicated producer: warps drift up to SST - 1 tiles apart.
   auto issue = [&](int k) {
     const TileDesc d = tile_desc(k, L0, L1, npad, QBS);
-    const int s = k % STAGES;
+    const int s = k % SST;
     const uint32_t n = (uint32_t)d.cnt;
     mbar_arrive_expect_tx(&sm.full[s], n * 20u);
     tma_load_1d(sm.ring[s], sp + d.jb, n * 16u, &sm.full[s]);
@@ -272,12 +275,12 @@ __global__ void __launch_bounds__(NTS, NTS == 128 ? 4 : 1)
       a.phase[blockIdx.x * 8 + 6] = 0;
     }
 #pragma unroll
-    for (int s = 0; s < STAGES; ++s) {
+    for (int s = 0; s < SST; ++s) {
       mbar_init(&sm.full[s], 1);
       sm.rel[s] = 0;
     }
     mbar_fence_init();
-    for (int k = 0; k < STAGES && k < ntiles; ++k) issue(k);
+    for (int k = 0; k < SST && k < ntiles; ++k) issue(k);
   }
   __syncthreads();
   Rec* rec = sm.rec[warp];
@@ -304,10 +307,10 @@ __global__ void __launch_bounds__(NTS, NTS == 128 ? 4 : 1)
       }
       limq = fmaxf(fmaxf(lim[0], lim[1]), fmaxf(lim[2], lim[3]));
     }
-    const int s = k % STAGES;
+    const int s = k % SST;
     long long tw0 = 0;
     if (a.phase) tw0 = clock64();
-    mbar_wait(&sm.full[s], (uint32_t)(k / STAGES) & 1u);
+    mbar_wait(&sm.full[s], (uint32_t)(k / SST) & 1u);
     if (a.phase) t_wait += clock64() - tw0;
     {
       const float4* tile = sm.ring[s];
@@ -369,15 +372,15 @@ __global__ void __launch_bounds__(NTS, NTS == 128 ? 4 : 1)
       }
     }
     __syncwarp();
-    if (lane == 0) {  // release stage s; the last warp refills it with tile k + STAGES
+    if (lane == 0) {  // release stage s; the last warp refills it with tile k + SST
       __threadfence_block();
       const int old = atomicAdd(&sm.rel[s], 1);
       if (old == NW - 1) {
         sm.rel[s] = 0;
         __threadfence_block();
-        if (k + STAGES < ntiles) {
+        if (k + SST < ntiles) {
           fence_proxy_async_smem();
-          issue(k + STAGES);
+          issue(k + SST);
         }
       }
     }
@@ -704,6 +707,7 @@ cudaError_t launch_sym_scan(const StepArgs& a, float4* sp, int* sidx, const long
     const char* e = getenv("BOIDS_SYM_NT");  // diagnostics: force a CTA shape (128 or 512)
     return e ? atoi(e) : 0;
   }();
+  if (force == 256) return sym_with<256>(a, sp, sidx, fb_prev, fb_cur, sms, s);
   if (force == 512 || (force != 128 && tiles512 >= 2LL * sms)) return sym_with<512>(a, sp, sidx, fb_prev, fb_cur, sms, s);
   return sym_with<128>(a, sp, sidx, fb_prev, fb_cur, sms, s);
 }
