@@ -134,6 +134,57 @@ __device__ __forceinline__ void issue(GridSmem& sm, const GridArgs& g, uint32_t 
   tma_load_1d(sm.ring[s], g.spos + sm.range[r].x + off, cnt * (uint32_t)sizeof(float4), &sm.full[s]);
 }
 
+// One tile of candidates against this thread's first QV queries (the rest of
+// the warp's groups hold no queries): distances, vote, rare exact insertion.
+template <int QV>
+__device__ __forceinline__ void grid_tile(const float4* tile, int cnt, const float2 (&pxy)[Q], const float (&pz)[Q],
+                                          float (&lim)[Q], float& limc, const int (&gq)[Q], key_t* lists, int warp,
+                                          int lane, unsigned& groups, unsigned& slow_groups) {
+  for (int c = 0; c < cnt; c += U) {
+    float4 cc[U];
+    if (c + U <= cnt) {
+#pragma unroll
+      for (int u = 0; u < U; ++u) cc[u] = tile[c + u];
+    } else {  // ragged tail of a range
+#pragma unroll
+      for (int u = 0; u < U; ++u)
+        cc[u] = c + u < cnt ? tile[c + u] : make_float4(__int_as_float(0x7fc00000), 0.f, 0.f, __int_as_float(-1));
+    }
+    // d2 = ((dx*dx) + (dy*dy)) + (dz*dz), every op rounded (Appendix A), packed
+    // FADD2/FMUL2 on the (x, y) pairs, scalar dz and sums (see k_sym.cu)
+    float d[QV][U];
+#pragma unroll
+    for (int u = 0; u < U; ++u)
+#pragma unroll
+      for (int q = 0; q < QV; ++q) {
+        const float2 dxy = __fadd2_rn(pxy[q], make_float2(-cc[u].x, -cc[u].y));
+        const float2 sq = __fmul2_rn(dxy, dxy);
+        const float dz = __fsub_rn(pz[q], cc[u].z);
+        d[q][u] = __fadd_rn(__fadd_rn(sq.x, sq.y), __fmul_rn(dz, dz));
+      }
+    float m = d[0][0];
+#pragma unroll
+    for (int q = 0; q < QV; ++q)
+#pragma unroll
+      for (int u = 0; u < U; ++u) m = fminf(m, d[q][u]);
+    ++groups;
+    if (__any_sync(0xffffffffu, m <= limc)) {
+      ++slow_groups;
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        const int j = __float_as_int(cc[u].w);  // original index
+#pragma unroll
+        for (int q = 0; q < QV; ++q)
+          if (d[q][u] <= lim[q] && j != gq[q])
+            lim[q] = fminf(lim[q], insert_smem7(&lists[qslot(warp, q, lane)], QBG, make_key(d[q][u], j)));
+      }
+      limc = lim[0];
+#pragma unroll
+      for (int q = 1; q < QV; ++q) limc = fmaxf(limc, lim[q]);
+    }
+  }
+}
+
 __global__ void __launch_bounds__(NTG, 5) k_grid(StepArgs a, GridArgs g) {  // 5 CTAs / SM: 3.38 -> 3.27 ms at C5 (4: 127 regs; 6: spills more, 3.33)
   __shared__ GridSmem sm;
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
@@ -266,7 +317,12 @@ __global__ void __launch_bounds__(NTG, 5) k_grid(StepArgs a, GridArgs g) {  // 5
     }
     __syncthreads();
     const int nr = sm.nrange;
-    float limc = fmaxf(fmaxf(lim[0], lim[1]), fmaxf(lim[2], lim[3]));
+    // query groups of 32 slots this warp holds queries in (blocked slots)
+    const int qv = BOIDS_GRID_RR ? (warp * 32 < qn ? Q : 0) : max(0, min(Q, (qn - warp * 32 * Q + 31) / 32));
+    float limc = 0.f;
+#pragma unroll
+    for (int q = 0; q < Q; ++q)
+      if (q < qv) limc = fmaxf(limc, lim[q]);
     __syncwarp();
 
     // consumers: walk the same tile sequence as the producer
@@ -279,51 +335,13 @@ __global__ void __launch_bounds__(NTG, 5) k_grid(StepArgs a, GridArgs g) {  // 5
       mbar_wait(&sm.full[s], (tc / STAGES) & 1u);
       const float4* tile = sm.ring[s];
       const int cnt = tile_count(sm, r, off);
-      // warps without queries in this item only keep the ring protocol
-      for (int c = 0; c < (warp_has_queries(warp, qn) ? cnt : 0); c += U) {
-        float4 cc[U];
-        if (c + U <= cnt) {
-#pragma unroll
-          for (int u = 0; u < U; ++u) cc[u] = tile[c + u];
-        } else {  // ragged tail of a range
-#pragma unroll
-          for (int u = 0; u < U; ++u)
-            cc[u] = c + u < cnt ? tile[c + u]
-                                : make_float4(__int_as_float(0x7fc00000), 0.f, 0.f, __int_as_float(-1));
-        }
-        float d[Q][U];
-#pragma unroll
-        for (int u = 0; u < U; ++u)
-#pragma unroll
-          for (int q = 0; q < Q; ++q) {
-            const float2 dxy = __fadd2_rn(pxy[q], make_float2(-cc[u].x, -cc[u].y));
-            const float2 sq = __fmul2_rn(dxy, dxy);
-            const float dz = __fsub_rn(pz[q], cc[u].z);
-            d[q][u] = __fadd_rn(__fadd_rn(sq.x, sq.y), __fmul_rn(dz, dz));
-          }
-        float mq[Q];
-#pragma unroll
-        for (int q = 0; q < Q; ++q) {
-          mq[q] = d[q][0];
-#pragma unroll
-          for (int u = 1; u < U; ++u) mq[q] = fminf(mq[q], d[q][u]);
-        }
-        const float m = fminf(fminf(mq[0], mq[1]), fminf(mq[2], mq[3]));
-        ++groups;
-        if (__any_sync(0xffffffffu, m <= limc)) {
-          ++slow_groups;
-#pragma unroll
-          for (int u = 0; u < U; ++u) {
-            const int j = __float_as_int(cc[u].w);  // original index
-#pragma unroll
-            for (int q = 0; q < Q; ++q)
-              if (d[q][u] <= lim[q] && j != gq[q])
-                lim[q] = fminf(lim[q], insert_smem7(&sm.lists[qslot(warp, q, lane)], QBG,
-                                                    make_key(d[q][u], j)));
-          }
-          limc = fmaxf(fmaxf(lim[0], lim[1]), fmaxf(lim[2], lim[3]));
-        }
-      }
+      // warps without queries in this item only keep the ring protocol; a warp
+      // computes only its query groups that hold queries (the item's last warp
+      // is usually partial: the padded groups cost work and loosen the vote)
+      if (qv == 4) grid_tile<4>(tile, cnt, pxy, pz, lim, limc, gq, sm.lists, warp, lane, groups, slow_groups);
+      else if (qv == 3) grid_tile<3>(tile, cnt, pxy, pz, lim, limc, gq, sm.lists, warp, lane, groups, slow_groups);
+      else if (qv == 2) grid_tile<2>(tile, cnt, pxy, pz, lim, limc, gq, sm.lists, warp, lane, groups, slow_groups);
+      else if (qv == 1) grid_tile<1>(tile, cnt, pxy, pz, lim, limc, gq, sm.lists, warp, lane, groups, slow_groups);
       __syncwarp();
       if (lane == 0) mbar_arrive(&sm.empty[s]);
       ++tc;
