@@ -363,7 +363,7 @@ __global__ void __launch_bounds__(NTS, NTS == 128 ? 4 : (NTS == 256 ? 2 : 1))
         }
       };
       if (!diag && cnt == CT) {  // full off-diagonal tile: constant trip count (the common case)
-#pragma unroll 2
+#pragma unroll 4  // measured: 1 / 2 / 4 / 8 -> C4 2.92 / 2.89 / 2.83 / 2.83 ms (bench pattern)
         for (int c = 0; c < CT; c += U) group(c, std::false_type{});
       } else if (!diag) {
         for (int c = 0; c < cnt; c += U) group(c, std::false_type{});
