@@ -449,7 +449,7 @@ __device__ __forceinline__ float sym_t0(const StepArgs& a, int64_t qi, float4 me
 // upper bound on the 7th key like t0; +inf with fewer than 7 of them.  The
 // sort is up to BOIDS_OPT_RESORT steps old: only the bound's tightness depends
 // on that, never the result.
-constexpr int WIN = 64;
+constexpr int WIN = 256;  // C4: 64 -> 11 routed agents per step, 256 -> 3 (route 32 -> 22 us, prep +17 us; net -0.5..1 %)
 __device__ float window_bound(const StepArgs& a, int qi, float4 me) {
   const int n = (int)a.nloc;
   if (!a.lstart || !a.qperm || n < 8 || !(me.x == me.x && me.y == me.y && me.z == me.z))
