@@ -272,6 +272,42 @@ def test_config_c4_warm_sampled(pk, orc, sym):
             np.testing.assert_array_equal(g[k][ag], o[k])
 
 
+def _spatial_ids(state, cells=64):
+    """Renumber the agents so ids follow space (sort by a coarse z, y, x cell,
+    then x): a reindex of the seeded state, no method arithmetic.  The bench's
+    ids are spatially random; here neighbours have nearby ids (measured to
+    change k_sym's timing, profiles/r1j/locality_probe.txt)."""
+    p = state["pos"]
+    lo, hi = p.min(0), p.max(0)
+    q = np.clip(((p - lo) / (hi - lo) * cells).astype(np.int64), 0, cells - 1)
+    perm = np.lexsort((p[:, 0], q[:, 0], q[:, 1], q[:, 2]))
+    return {k: np.ascontiguousarray(state[k][perm]) for k in KEYS}
+
+
+@pytest.mark.parametrize("search", [0, 1])
+def test_spatially_ordered_ids_warm_sampled(pk, orc, search):
+    """C4-size flock whose ids follow space (brute force on k_sym, and the grid):
+    cold step, jittered copy, warm step; 1024 sampled agents bit-exact against
+    the oracle (lists, steering, state)."""
+    c = W.CONFIGS["c4"]
+    p = pk.boids_default_params(init_mode=c.init_mode, search_mode=search)
+    op = _oparams(orc, p)
+    ag = W.sample_agents(c.n, 1024, seed=11)
+    s0 = _spatial_ids(orc.init(c.n, op, seed=1))
+    s1 = W.jitter(s0, 0.05, seed=6)
+    with pk.Flock(c.n, p, seed=1, record_steering=True) as f:
+        f.set_state(s0)
+        f.step(DT, 1)
+        f.set_state(s1)
+        f.step(DT, 1)
+        g = f.state()
+        o, o_idx, _, o_F = orc.step_sample(orc.State(s1), ag, DT, op)
+        np.testing.assert_array_equal(f.neighbors()[0][ag], o_idx)
+        np.testing.assert_array_equal(f.steering()[ag], o_F)
+        for k in KEYS:
+            np.testing.assert_array_equal(g[k][ag], o[k])
+
+
 @pytest.mark.parametrize("n,search", [(300001, 0), (2500003, 1)])
 def test_large_ragged_warm_sampled(pk, orc, n, search):
     """Beyond the bench sizes, ragged (n not a multiple of any tile or query
