@@ -147,15 +147,16 @@ def cpu_oracle_rate_threads(cfg: W.Config, agents_per_thread: int, threads: int,
 
 
 def cpu_sample_size(cfg: W.Config, seconds: float) -> int:
-    """Agents per sample for ~`seconds` of oracle work (about 5 ns per candidate pair)."""
-    return int(max(64, min(cfg.n, seconds / (5e-9 * cfg.n))))
+    """Agents per sample for ~`seconds` of oracle work (about 1 ns per candidate pair,
+    measured on the GPU box: profiles/r1j bench lines)."""
+    return int(max(64, min(cfg.n, seconds / (1e-9 * cfg.n))))
 
 
 def run_reference(args, cfg):
     rank, world, _ = env_rank()
     if rank != 0:
         return 0
-    m = cpu_sample_size(cfg, 1.5)
+    m = cpu_sample_size(cfg, 1.0)
     for _ in range(args.warmup):
         cpu_oracle_rate(cfg, max(64, m // 8))
     times, agents = [], 0
