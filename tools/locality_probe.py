@@ -40,11 +40,14 @@ for name in sys.argv[1:] or ["c5", "c4"]:
         f.sync()
         f.profile(reset=True)
         steps = 10
+        i0 = f.info()
         f.step(float(W.DT), steps)
         f.sync()
         prof = f.profile()
+        i1 = f.info()
         ms = sum(v[0] for v in prof.values())
         top = sorted(((v[0] / max(v[1], 1) * 1e3, k) for k, v in prof.items() if v[1]), reverse=True)[:4]
         print(f"{name} {order:6s} {ms / steps * 1e3:8.1f} us/step  agent-steps/s {c.n * steps / (ms / 1e3):.3e}  "
-              f"top {[(k, round(t, 1)) for t, k in top]}", flush=True)
+              f"top {[(k, round(t, 1)) for t, k in top]}  slow/vote {(i1.slow_groups - i0.slow_groups) / max(i1.vote_groups - i0.vote_groups, 1):.4f} "
+              f"vote_groups/step {(i1.vote_groups - i0.vote_groups) / steps:.3e} fallbacks/step {(i1.fallbacks - i0.fallbacks) / steps:.1f}", flush=True)
         f.close()
