@@ -5,6 +5,7 @@
 #include <cstring>
 #include <new>
 #include <string>
+#include <algorithm>
 #include <vector>
 
 #include "internal.h"
@@ -748,6 +749,40 @@ BOIDS_API int boids_get_state(boids_ctx* c, float* pos3, float* fwd3, float* up3
   return BOIDS_OK;
 }
 
+// The spatial query order (qperm) is a permutation of agent ids: after an upload
+// with another id <-> space arrangement it no longer groups nearby queries
+// (measured: C4 with Morton-renumbered ids 2.79 -> 3.60 ms/step until the next
+// refresh), so boids_set_state has it rebuilt on the next step -- unless the
+// upload keeps the arrangement (the usual case: the caller's copy of the last
+// state, moved a little).  Test: 256 strided pairs of consecutive qperm entries;
+// the order is kept if at least half of them are still within the search radius
+// of each other in the uploaded positions.  Only a performance decision.
+static bool order_still_spatial(boids_ctx* c, const float* pos3) {
+  const int64_t k = c->nloc;
+  if (!c->qperm || k < 64) return false;
+  const int64_t stride = std::max<int64_t>(1, (k - 1) / 256);
+  const int64_t cnt = std::min<int64_t>(256, (k - 1) / stride);
+  std::vector<int32_t> pr((size_t)(2 * cnt));
+  if (cudaMemcpy2DAsync(pr.data(), 2 * sizeof(int32_t), c->qperm, (size_t)stride * sizeof(int32_t),
+                        2 * sizeof(int32_t), (size_t)cnt, cudaMemcpyDeviceToHost, c->stream) != cudaSuccess ||
+      cudaStreamSynchronize(c->stream) != cudaSuccess)
+    return false;
+  const float r2 = c->p.search_radius * c->p.search_radius;
+  int64_t valid = 0, near = 0;
+  for (int64_t t = 0; t < cnt; ++t) {
+    const int64_t a = pr[2 * t], b = pr[2 * t + 1];
+    if (a < 0 || a >= k || b < 0 || b >= k) continue;
+    ++valid;
+    float d2 = 0.f;
+    for (int d = 0; d < 3; ++d) {
+      const float x = pos3[3 * a + d] - pos3[3 * b + d];
+      d2 += x * x;
+    }
+    near += d2 <= r2 ? 1 : 0;
+  }
+  return valid > 0 && 2 * near >= valid;
+}
+
 BOIDS_API int boids_set_state(boids_ctx* c, const float* pos3, const float* fwd3, const float* up3,
                     const float* side3, const float* speed) {
   if (!c) return fail(BOIDS_EINVAL, "NULL handle");
@@ -769,12 +804,8 @@ BOIDS_API int boids_set_state(boids_ctx* c, const float* pos3, const float* fwd3
   // smallest current distance to 7-8 distinct existing agents) is an upper bound
   // on the 7th neighbour distance for ANY positions, so the next step stays exact;
   // a poor bound only costs time.  boids_get_neighbors still reports the lists of
-  // the last step until the next step.  The spatial query order (qperm) is a
-  // permutation of agent ids: for a state with another id <-> space arrangement
-  // it no longer groups nearby queries (measured: C4 with Morton-renumbered ids
-  // 2.79 -> 3.60 ms/step over the next resort_every steps), so it is rebuilt on
-  // the next step.
-  c->since_sort = -1;
+  // the last step until the next step.
+  if (c->since_sort >= 0 && !order_still_spatial(c, pos3)) c->since_sort = -1;
   CK(cudaStreamSynchronize(c->stream));
   c->steering_valid = false;
   return BOIDS_OK;
