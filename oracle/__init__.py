@@ -80,6 +80,8 @@ def lib():
                                          + [f32p] * 5 + [i32p, i32p, f32p, f32p])
         L.oracle_step_think.argtypes = ([C.c_int64, P, C.c_float, C.c_int64] + [f32p] * 5 + [f32p] * 5
                                         + [i32p, i32p, f32p, f32p, f32p])
+        L.oracle_step_think_sample.argtypes = ([C.c_int64, P, C.c_float, C.c_int64] + [f32p] * 5
+                                               + [C.c_int64, i64p] + [f32p] * 5 + [i32p, i32p, f32p, f32p, f32p])
         L.oracle_run.argtypes = [C.c_int64, P, C.c_float, C.c_int32] + [f32p] * 6
         L.oracle_run.restype = C.c_int
         _lib = L
@@ -227,6 +229,27 @@ def step_think(s: State, dt: float, t: int, fstore, idx7, cnt, params: OraclePar
     acc = _acc_in(s, n)
     lib().oracle_step_think(n, C.byref(p), C.c_float(dt), t, *_state_arrays(s), out["pos"], out["fwd"],
                             out["up"], out["side"], out["speed"], idx, c, fs, F, acc)
+    return _with_acc(out, acc, p), idx, c, fs, F
+
+
+def step_think_sample(s: State, agents, dt: float, t: int, fstore, idx7=None, cnt=None,
+                      params: OracleParams | None = None):
+    """step_think evaluated only for `agents`.  fstore (len(agents), 3), idx7
+    (len(agents), 7), cnt (len(agents),) are the sampled agents' carried think
+    state (copied).  Returns (State, idx7, cnt, fstore, F_used) per sampled agent."""
+    p = params or default_params()
+    agents = np.ascontiguousarray(agents, np.int64)
+    m = agents.shape[0]
+    out = State(pos=np.empty((m, 3), np.float32), fwd=np.empty((m, 3), np.float32),
+                up=np.empty((m, 3), np.float32), side=np.empty((m, 3), np.float32),
+                speed=np.empty(m, np.float32))
+    idx = np.full((m, 7), -1, np.int32) if idx7 is None else np.array(idx7, np.int32, copy=True).reshape(m, 7)
+    c = np.full(m, -1, np.int32) if cnt is None else np.array(cnt, np.int32, copy=True).reshape(m)
+    fs = np.array(fstore, np.float32, copy=True).reshape(m, 3)
+    F = np.empty((m, 3), np.float32)
+    acc = np.ascontiguousarray(_acc_in(s, s.n)[agents])
+    lib().oracle_step_think_sample(s.n, C.byref(p), C.c_float(dt), t, *_state_arrays(s), m, agents, out["pos"],
+                                   out["fwd"], out["up"], out["side"], out["speed"], idx, c, fs, F, acc)
     return _with_acc(out, acc, p), idx, c, fs, F
 
 

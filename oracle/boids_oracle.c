@@ -39,7 +39,8 @@
  *
  * Pins (tests/test_oracle_*.py): brute-force sort on tiny flocks, tie and
  * boundary cases, invariants, closed-form steering/modification cases, the
- * wrap example, scipy cKDTree on tie-free inputs.  Parity unpinned: that the
+ * wrap example, scipy cKDTree on tie-free inputs, the local-space handedness
+ * (closed forms, the triple-product identity up' = n(u - (u.f')f'), det sign).  Parity unpinned: that the
  * DESIGN.md Table C1 constants and the Q10 modification arithmetic are what
  * the thesis actually ran (the paper prints neither).
  */
@@ -456,6 +457,31 @@ void oracle_step_think(int64_t n, const oracle_params* p, float dt, int64_t t, c
     oracle_modify_one(pos3 + 3 * i, fwd3 + 3 * i, up3 + 3 * i, side3 + 3 * i, speed[i], force3 + 3 * i, p,
                       dt, pos_o + 3 * i, fwd_o + 3 * i, up_o + 3 * i, side_o + 3 * i, speed_o + i,
                       acc3 + 3 * i);
+  }
+}
+
+/* oracle_step_think evaluated only for the m agents listed in `agents` (each
+ * thinker searched against all n): the same per-agent rule (reading
+ * Q15), for checking large flocks on a sample.  fstore3/force3/acc3/idx7/cnt
+ * and the outputs are per sampled agent (row s belongs to agents[s]). */
+void oracle_step_think_sample(int64_t n, const oracle_params* p, float dt, int64_t t, const float* pos3,
+                              const float* fwd3, const float* up3, const float* side3, const float* speed,
+                              int64_t m, const int64_t* agents, float* pos_o, float* fwd_o, float* up_o,
+                              float* side_o, float* speed_o, int32_t* idx7, int32_t* cnt, float* fstore3,
+                              float* force3, float* acc3) {
+  int64_t k = p->think_every < 1 ? 1 : p->think_every;
+  for (int64_t s = 0; s < m; ++s) {
+    int64_t i = agents[s];
+    if ((i + t) % k == 0) {
+      oracle_search_one(n, pos3, p->search_radius, i, idx7 + 7 * s, cnt + s);
+      oracle_steer_one(pos3, fwd3, i, idx7 + 7 * s, cnt[s], p, fstore3 + 3 * s);
+    }
+    force3[3 * s] = fstore3[3 * s];
+    force3[3 * s + 1] = fstore3[3 * s + 1];
+    force3[3 * s + 2] = fstore3[3 * s + 2];
+    oracle_modify_one(pos3 + 3 * i, fwd3 + 3 * i, up3 + 3 * i, side3 + 3 * i, speed[i], force3 + 3 * s, p,
+                      dt, pos_o + 3 * s, fwd_o + 3 * s, up_o + 3 * s, side_o + 3 * s, speed_o + s,
+                      acc3 + 3 * s);
   }
 }
 

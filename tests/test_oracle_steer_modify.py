@@ -240,3 +240,81 @@ def test_polarisation_rises(orc):
     a0 = local_alignment(s)
     a1 = local_alignment(orc.run(s, DT, 300))
     assert abs(a0) < 0.05 and a1 > a0 + 0.1
+
+
+# ---------------- local-space handedness (reading Q25) ----------------
+# OpenSteer's LocalSpace is right-handed [ext]: regenerateOrthonormalBasisUF sets
+# side = normalize(forward x up), then up = side x forward.  Two consequences
+# fixed by the vector algebra alone, not by the oracle's code:
+#   * up' = side x forward = (f x u) x f = u - (u . f) f (triple product): the new
+#     up is the OLD up projected onto the plane normal to the new forward -- it
+#     never flips (u' . u > 0 whenever u is not parallel to f);
+#   * det[side, up, forward] = (f x u) . (u x f) / |f x u| < 0, i.e. -1.
+# A swapped operand order in either cross product flips up' (first pin) or side
+# (the det sign); orthonormality alone (test_modify_invariants) cannot tell.
+
+
+def _det3(s, u, f):
+    return float(np.dot(np.asarray(s, np.float64), np.cross(np.asarray(u, np.float64), np.asarray(f, np.float64))))
+
+
+def test_local_space_closed_form(orc):
+    """f = (0,0,1), u = (0,1,0), F = 0: forward stays, side = f x u = (-1,0,0),
+    up = side x f = (0,1,0) -- exact (every product is 0 or +-1)."""
+    o = orc.modify_one([0, 0, 0], [0, 0, 1], [0, 1, 0], [0, 0, 0], 1.0, [0, 0, 0], 0.1)
+    assert o["fwd"].tolist() == [0, 0, 1]
+    assert o["side"].tolist() == [-1, 0, 0]
+    assert o["up"].tolist() == [0, 1, 0]
+    assert _det3(o["side"], o["up"], o["fwd"]) == -1.0
+
+
+def test_local_space_turn_closed_form(orc):
+    """Turning in the horizontal plane keeps up = (0,1,0): f = (1,0,0), speed 1,
+    F = (0,0,60) (clamped to 27), dt = 0.1 -> v = (1, 0, 2.7), f' = v / |v|;
+    up' must be exactly perpendicular to the turn plane, (0,1,0), and side' =
+    f' x up' = (-f'z, 0, f'x)."""
+    o = orc.modify_one([0, 0, 0], [1, 0, 0], [0, 1, 0], [0, 0, -1], 1.0, [0, 0, 60], 0.1)
+    f = np.asarray(o["fwd"], np.float64)
+    ref = np.array([1.0, 0.0, 2.7]) / np.linalg.norm([1.0, 0.0, 2.7])
+    np.testing.assert_allclose(f, ref, rtol=1e-6, atol=1e-7)
+    np.testing.assert_allclose(o["up"], [0, 1, 0], atol=1e-7)
+    np.testing.assert_allclose(o["side"], [-f[2], 0.0, f[0]], rtol=1e-6, atol=1e-7)
+    assert _det3(o["side"], o["up"], o["fwd"]) < 0
+
+
+@pytest.mark.parametrize("seed", range(5))
+def test_local_space_up_is_projected_old_up(orc, seed):
+    """Random frames and forces: up' = n^(u - (u . f') f') (triple-product
+    identity) and det[s', u', f'] = -1."""
+    rng = np.random.default_rng(100 + seed)
+    for _ in range(200):
+        f = unit(rng.standard_normal(3))
+        u = unit(np.cross(unit(rng.standard_normal(3)), f))
+        s = np.cross(f, u)
+        F = rng.standard_normal(3) * rng.uniform(1, 60)
+        o = orc.modify_one(rng.uniform(-20, 20, 3), f, u, s, rng.uniform(0.5, 9), F, DT)
+        f1 = np.asarray(o["fwd"], np.float64)
+        proj = unit(u - np.dot(u, f1) * f1)
+        if np.linalg.norm(u - np.dot(u, f1) * f1) < 1e-3:
+            continue  # new forward (nearly) parallel to the old up: reading Q13
+        np.testing.assert_allclose(o["up"], proj, atol=2e-5)
+        assert np.dot(o["up"], u) > 0
+        assert abs(_det3(o["side"], o["up"], o["fwd"]) + 1.0) < 1e-5
+
+
+@pytest.mark.parametrize("mode", [0, 1])
+def test_init_local_space_handedness(orc, mode):
+    """Appendix B: up0 = (0,1,0), side = n^(f x up0), up = side x f -- so up is
+    the world y axis projected normal to the forward (u . y > 0) and
+    det[side, up, fwd] = -1 for every agent."""
+    s = orc.init(5000, orc.default_params(init_mode=mode), seed=7)
+    f = s["fwd"].astype(np.float64)
+    y = np.array([0.0, 1.0, 0.0])
+    proj = y - (f @ y)[:, None] * f
+    ok = np.linalg.norm(proj, axis=1) > 1e-3
+    proj = proj[ok] / np.linalg.norm(proj[ok], axis=1)[:, None]
+    np.testing.assert_allclose(s["up"][ok], proj, atol=2e-5)
+    assert (s["up"][ok][:, 1] > 0).all()
+    det = np.einsum("ij,ij->i", s["side"].astype(np.float64),
+                    np.cross(s["up"].astype(np.float64), f))
+    np.testing.assert_allclose(det[ok], -1.0, atol=1e-5)

@@ -59,3 +59,21 @@ def test_every_agent_thinks_once_per_period(orc):
         s, idx, cnt, fs, F = orc.step_think(s, DT, t, fs, idx, cnt, p)
         thought += (np.any(fs != before, axis=1) | (cnt > 0)).astype(int) * ((np.arange(n) + t) % k == 0)
     assert (thought == 1).all()
+
+
+@pytest.mark.parametrize("k,t", [(10, 11), (4, 2)])
+def test_step_think_sample_matches_full(orc, k, t):
+    """The sampled form used for full-size GPU checks (C4/C5 think 10) is
+    step_think restricted to the sampled rows, with a nonzero stored force."""
+    n = 400
+    s = orc.State(W.ball_flock(n, seed=k * t, radius=10.0))
+    p = orc.default_params(think_every=k)
+    fs = W.random_forces(n, seed=3)
+    idx, cnt, _ = fresh(orc, n)
+    o, i2, c2, fs2, F = orc.step_think(s, DT, t, fs, idx, cnt, p)
+    ag = np.array([0, 1, 2, 9, 10, 11, 57, 123, 398, 399])
+    so, si, sc, sfs, sF = orc.step_think_sample(s, ag, DT, t, fs[ag], idx[ag], cnt[ag], p)
+    for key in ("pos", "fwd", "up", "side", "speed"):
+        assert np.array_equal(so[key], o[key][ag]), key
+    assert np.array_equal(si, i2[ag]) and np.array_equal(sc, c2[ag])
+    assert np.array_equal(sfs, fs2[ag]) and np.array_equal(sF, F[ag])

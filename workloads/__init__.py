@@ -119,3 +119,10 @@ def sample_agents(n: int, m: int, seed: int = 7) -> np.ndarray:
     if m > 1:
         s[1] = n - 1
     return np.unique(s).astype(np.int64)
+
+
+def random_forces(n: int, seed: int = 13, scale: float = 30.0) -> np.ndarray:
+    """Seeded steering vectors (n, 3) float32, Gaussian with per-axis std `scale`:
+    a stored-steering input for think-frequency checks (no method arithmetic)."""
+    rng = np.random.default_rng(seed)
+    return (rng.standard_normal((n, 3)) * scale).astype(np.float32)
