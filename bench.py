@@ -171,7 +171,7 @@ def run_reference(args, cfg):
         "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": total / args.steps * 1e3,
         "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f32",
-        "data": "synthetic", "config": config_dict(cfg, args.gpus),
+        "data": "synthetic", "config": dict(config_dict(cfg, args.gpus), think_every=max(1, args.think)),
         "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
         "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
@@ -305,7 +305,9 @@ def main():
     k_ms, k_n = prof[kname]
     k_ms_per = k_ms / max(k_n, 1)
     think = max(1, args.think)
-    sym = dist is None and not grid and think == 1 and not args.no_sym and args.kernel == 0
+    # the library reports which search path the timed steps ran (boids_info.last_path)
+    path = int(info1.last_path)
+    sym = path == abi.BOIDS_PATH_SYM
     if grid:  # algorithmic work of the grid search: pairs over the 27-cell stencils (device counter)
         pairs_per_launch = float(info1.grid_pairs - info0.grid_pairs) / max(k_n, 1)
         pairs_note = " (27-cell stencil candidates, device counter)"
@@ -327,10 +329,14 @@ def main():
             traffic = json.load(open(summ)).get(cfg.name, {}).get("dram_bytes_per_launch")
         except Exception:
             traffic = None
+    kernel_names = {abi.BOIDS_PATH_GRID: "k_grid (binned search + steer + modify)",
+                    abi.BOIDS_PATH_SYM: "k_sym_prep + k_sym (warm-step unordered-pair search)",
+                    abi.BOIDS_PATH_SCAN: "k_bound + k_scan (warm-step ordered-pair search)",
+                    abi.BOIDS_PATH_THINK: "k_bound + k_scan over this step's thinkers (k_fused for never-searched ones)",
+                    abi.BOIDS_PATH_FUSED: "k_fused (cold-step cluster kernel)",
+                    abi.BOIDS_PATH_SIMPLE: "k_search_simple (tiled search, thesis structure)"}
     roofline = {"bound": "alu",
-                "kernel": ("k_grid (binned search + steer + modify)" if grid else
-                           "k_sym_prep + k_sym (warm-step unordered-pair search)" if sym else
-                           "k_bound + k_scan (warm-step all-pairs search; k_fused on cold steps)"),
+                "kernel": kernel_names.get(path, f"path {path}"), "path": path,
                 "achieved": achieved, "peak": peak, "unit": "TFLOP/s", "frac": achieved / peak,
                 "traffic": traffic,
                 "peak_note": f"FP32 SIMT lane-ops: 148 SM x 128 lanes x {sm_max:.0f} MHz "
@@ -346,20 +352,63 @@ def main():
             "note": "n x n pairs of the thesis's formulation / the same kernel time: the rate an "
                     "ordered-pair kernel would need to match; not a hardware utilisation"}
 
-    # ---------------- the update (modification) kernel against HBM ----------------
-    u_ms, u_n = prof["update"]
+    # ---------------- update and binning kernels against HBM ----------------
+    # A separate profiled pass of K steps right after the timed region (events
+    # around EVERY launch would break the PDL chain of the timed steps): the
+    # update-class kernel (k_select1 on warm brute-force steps, k_apply in think
+    # mode) and the binning kernels, each against the measured copy bandwidth.
+    # Then the standalone update kernel k_update (B5: steering from the last
+    # step's lists + modification, one thread per agent) through
+    # boids_bench_update, L2 flushed before every launch.
+    hbm = float(pk_.get("hbm_gbs", 6552.0))
+    hbm_note = "hbm_gbs of MEASURED_PEAKS.json (copy bandwidth, measured)"
+    abi.boids_set_option(h, abi.BOIDS_OPT_PROFILE, 1)
+    abi.boids_get_profile(h, reset=True)
+    for k in range(args.steps):
+        flush.fill_(float(k))
+        step()
+    torch.cuda.synchronize()
+    prof1 = abi.boids_get_profile(h, reset=True)
+    abi.boids_set_option(h, abi.BOIDS_OPT_PROFILE, 0)
+    u_ms, u_n = prof1["update"]
     update_roofline = None
     if u_n:
-        hbm = float(pk_.get("hbm_gbs", 6552.0))
         if think > 1 and grid:  # k_apply: pos4 fwd4 up4 side4 fstore in (80 B), pos4 fwd4 up4 side4 out (64 B)
             name, per_agent = "k_apply (modification of every agent, think mode)", 144
-        else:  # k_select: hits in, own state in/out; its neighbour gathers hit L2
-            name, per_agent = "k_select (top-7 + steering + modification)", 128 + 8 * 10
+        else:  # k_select: ~10 hits (8 B) in, own state in (64 B) / out (64 B); neighbour gathers hit L2
+            name, per_agent = "k_select1 (top-7 of the hit buffer + steering + modification)", 128 + 8 * 10
         ub = per_agent * float(nloc) / (u_ms / u_n / 1e3) / 1e9
         update_roofline = {"bound": "hbm", "kernel": name, "achieved": ub, "peak": hbm, "unit": "GB/s",
-                           "frac": ub / hbm, "bytes_per_agent": per_agent,
-                           "kernel_ms_per_launch": u_ms / u_n,
-                           "peak_note": "hbm_gbs of MEASURED_PEAKS.json (copy bandwidth, measured)"}
+                           "frac": ub / hbm, "bytes_per_agent": per_agent, "launches": u_n,
+                           "kernel_ms_per_launch": u_ms / u_n, "peak_note": hbm_note,
+                           "measured": "profiled pass of K steps after the timed region, L2 flushed per step"}
+    b_ms, b_n = prof1["binning"]
+    binning_roofline = None
+    if b_n and grid:
+        # per agent: read pos4 (16) + write cell/rank (8) + read cell/rank (8) + read pos4 (16) + write the
+        # sorted record (16) + query permutation (4) + cell counts/starts (~2 x 4 per agent amortised)
+        per_agent = 76
+        steps_binned = args.steps
+        bb = per_agent * float(cfg.n) * steps_binned / (b_ms / 1e3) / 1e9
+        binning_roofline = {"bound": "hbm", "kernel": "k_bin_count + scan + scatter (counting sort by cell)",
+                            "achieved": bb, "peak": hbm, "unit": "GB/s", "frac": bb / hbm,
+                            "bytes_per_agent": per_agent, "ms_per_step": b_ms / steps_binned,
+                            "peak_note": hbm_note}
+    std_ms = []
+    for k in range(max(3, args.steps)):
+        flush.fill_(float(k))
+        std_ms.append(abi.boids_bench_update(h, dt, 1))
+    std_ms = float(np.median(std_ms))
+    per_std = 160  # reads pos4 fwd4 up4 side4 (64) + nbr 7 x 4 + cnt 4 (32); writes pos4 fwd4 up4 side4 (64)
+    sb = per_std * float(nloc) / (std_ms / 1e3) / 1e9
+    update_standalone = {"bound": "hbm", "kernel": "k_update (steering from the last lists + modification)",
+                         "achieved": sb, "peak": hbm, "unit": "GB/s", "frac": sb / hbm,
+                         "bytes_per_agent": per_std, "kernel_ms_per_launch": std_ms,
+                         "note": "boids_bench_update, median of launches, L2 flushed before each; the "
+                                 "neighbours' pos4/fwd4 gathers (up to 7 x 32 B) are not counted (L2 hits)",
+                         "peak_note": hbm_note}
+    if update_roofline is None:
+        update_roofline = dict(update_standalone)
 
     # ---------------- e2e through the C ABI with host buffers ----------------
     e2e = None
@@ -436,7 +485,8 @@ def main():
             "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
             "config": dict(config_dict(cfg, world), think_every=think), "roofline": roofline,
-            "update_roofline": update_roofline, "cpu_baseline": cpu, "e2e": e2e, "e2e_draw": e2e_draw,
+            "update_roofline": update_roofline, "update_standalone": update_standalone,
+            "binning_roofline": binning_roofline, "cpu_baseline": cpu, "e2e": e2e, "e2e_draw": e2e_draw,
             "gpu_launches": int(launches), "clocks": clocks,
             "kernel_profile_ms": {k: v[0] for k, v in prof.items() if v[1]},
             "thesis_context": "thesis v5 GPU (GeForce 8800 GTS) vs CPU (Athlon 64 3700+): ~42x at 4096 agents "

@@ -109,7 +109,19 @@ typedef struct boids_info_t {
   int64_t grid_pairs;  /* grid mode, cumulative: (query, candidate) pairs evaluated over the
                           27-cell stencils -- the grid search's algorithmic work */
   int64_t step_index;  /* steps taken by this handle (the t of the think schedule) */
+  int32_t last_path;   /* search path the last step ran (BOIDS_PATH_*; -1 before the first step) --
+                          what bench.py's roofline counts as the algorithmic work */
+  int32_t reserved0;
+  int64_t steps_sorted; /* cumulative: steps that rebuilt the spatial query order (binning) */
 } boids_info_t;
+
+/* boids_info_t.last_path */
+#define BOIDS_PATH_FUSED 0   /* cold step: k_fused (cluster kernel, ordered pairs n_local x n) */
+#define BOIDS_PATH_SCAN 1    /* warm step: k_bound + k_scan over ordered pairs n_local x n */
+#define BOIDS_PATH_SYM 2     /* warm step: k_sym_prep + k_sym over unordered pairs n(n-1)/2 */
+#define BOIDS_PATH_GRID 3    /* grid mode: binning + k_grid (+ k_grid_far) */
+#define BOIDS_PATH_SIMPLE 4  /* BOIDS_KERNEL_SIMPLE: k_search_simple + k_update */
+#define BOIDS_PATH_THINK 5   /* brute force, think mode: thinkers on k_bound + k_scan (cold ones k_fused) */
 
 #define BOIDS_KERNEL_FUSED 0   /* default: cold steps run the fused cluster kernel (search + merge +
                                   steer + modify); warm steps (previous lists known) run the
@@ -224,6 +236,16 @@ BOIDS_API int boids_readback_wait(boids_ctx* ctx);
  * set: fstore3 NULL keeps the stored vectors.  Both synchronise. */
 BOIDS_API int boids_get_think_state(boids_ctx* ctx, int64_t* step_index, float* fstore3);
 BOIDS_API int boids_set_think_state(boids_ctx* ctx, int64_t step_index, const float* fstore3);
+
+/* Measurement hook (SURVEY.md 8(d), B5 "update_standalone"): time `reps` launches
+ * of the standalone update kernel k_update -- steering from the neighbour lists
+ * of the last step (boids_get_neighbors) plus the modification substage, one
+ * thread per owned agent (the thesis's separate modification kernel, P:440,
+ * P:497-502) -- with CUDA events on the handle's stream, each launch alone.
+ * The kernel writes into private scratch buffers (copies of the frame), so the
+ * handle's state, lists and step index are unchanged.  *ms_per_launch = mean
+ * launch duration.  Synchronises.  EINVAL: NULL argument, reps < 1, bad dt. */
+BOIDS_API int boids_bench_update(boids_ctx* ctx, float dt, int32_t reps, double* ms_per_launch);
 
 /* Describe the handle (synchronises: it reads the device-side counters). */
 BOIDS_API int boids_info(boids_ctx* ctx, boids_info_t* out);

@@ -33,8 +33,10 @@ EXPORTS = (
     "boids_get_state", "boids_set_state", "boids_get_neighbors", "boids_get_steering",
     "boids_sync", "boids_info", "boids_get_profile", "boids_get_phases", "boids_destroy", "boids_last_error",
     "boids_get_think_state", "boids_set_think_state", "boids_readback_begin", "boids_readback_wait",
-    "boids_get_accel", "boids_set_accel",
+    "boids_get_accel", "boids_set_accel", "boids_bench_update",
 )
+# boids_info_t.last_path
+BOIDS_PATH_FUSED, BOIDS_PATH_SCAN, BOIDS_PATH_SYM, BOIDS_PATH_GRID, BOIDS_PATH_SIMPLE, BOIDS_PATH_THINK = range(6)
 
 
 class BoidsError(RuntimeError):
@@ -59,6 +61,7 @@ class boids_info_t(C.Structure):
         ("rank", C.c_int32), ("world", C.c_int32), ("kernel", C.c_int32), ("cluster", C.c_int32),
         ("launches", C.c_int64), ("slow_groups", C.c_int64), ("vote_groups", C.c_int64),
         ("fallbacks", C.c_int64), ("grid_pairs", C.c_int64), ("step_index", C.c_int64),
+        ("last_path", C.c_int32), ("reserved0", C.c_int32), ("steps_sorted", C.c_int64),
     ]
 
 
@@ -100,6 +103,7 @@ def load(path: str = LIB_PATH):
         "boids_readback_wait": (C.c_int, [vp]),
         "boids_get_think_state": (C.c_int, [vp, C.POINTER(i64), fp]),
         "boids_set_think_state": (C.c_int, [vp, i64, fp]),
+        "boids_bench_update": (C.c_int, [vp, f32, i32, C.POINTER(C.c_double)]),
         "boids_destroy": (None, [vp]),
         "boids_last_error": (C.c_char_p, []),
     }
@@ -273,6 +277,13 @@ def boids_get_think_state(h: int):
 def boids_set_think_state(h: int, step_index: int, fstore=None):
     F = None if fstore is None else _f32(fstore, (_count(h), 3))
     _check(load().boids_set_think_state(h, step_index, _fptr(F)))
+
+
+def boids_bench_update(h: int, dt: float, reps: int = 1) -> float:
+    """Mean duration (ms) of `reps` standalone k_update launches (state untouched)."""
+    ms = C.c_double()
+    _check(load().boids_bench_update(h, dt, reps, C.byref(ms)))
+    return ms.value
 
 
 def boids_destroy(h: int):

@@ -100,7 +100,11 @@ struct boids_ctx {
   float4* fstore = nullptr;         // [m] last steering vector per agent
   unsigned char* routed = nullptr;  // [m] 1 = searched by k_fused this step (think mode)
   int32_t *tcold = nullptr, *twarm = nullptr, *tcnt = nullptr;  // thinker lists and their counts
+  int* ocheck = nullptr;            // [2] boids_set_state's locality check (k_order_check)
+  float4* ubench = nullptr;         // boids_bench_update scratch: out [2m] | up [m] | side [m] | acc [m]
   int64_t step_index = 0, steps_taken = 0;
+  int32_t last_path = -1;  // BOIDS_PATH_* of the last step
+  int64_t steps_sorted = 0;
   int vote_u = 4;          // fused kernel: candidates per warp vote
   int resort_every = 8;    // refresh the spatial query order every this many steps
   int64_t since_sort = -1; // steps since the last refresh (-1: never sorted)
@@ -193,6 +197,8 @@ void free_ctx(boids_ctx* c) {
   cudaFree(c->tcold);
   cudaFree(c->twarm);
   cudaFree(c->tcnt);
+  cudaFree(c->ocheck);
+  cudaFree(c->ubench);
   cudaFree(c->phase);
   cudaFree(c->sym_sp);
   cudaFree(c->sym_idx);
@@ -300,7 +306,8 @@ int create_impl(int64_t n, const boids_params* p, uint64_t seed, int32_t rank, i
       (rc = alloc((void**)&c->routed, m)) ||
       (rc = alloc((void**)&c->tcold, m * sizeof(int32_t))) ||
       (rc = alloc((void**)&c->twarm, m * sizeof(int32_t))) ||
-      (rc = alloc((void**)&c->tcnt, 2 * sizeof(int32_t)))) {
+      (rc = alloc((void**)&c->tcnt, 2 * sizeof(int32_t))) ||
+      (rc = alloc((void**)&c->ocheck, 2 * sizeof(int)))) {
     free_ctx(c);
     return rc;
   }
@@ -470,10 +477,12 @@ int one_step(boids_ctx* c, float dt) {
     StepArgs ag = a;
     ag.store_only = think ? 1 : 0;
     CK(cudaMemsetAsync(c->sym_rcount, 0, sizeof(int32_t), c->stream));
+    c->last_path = BOIDS_PATH_GRID;
     if ((rc = launch(c, 3, [&] { return launch_grid(ag, g, c->stream); }))) return rc;
     if ((rc = launch(c, 4, [&] { return launch_grid_far(ag, g, c->stream); }))) return rc;
     if (think && (rc = launch(c, 1, [&] { return launch_apply(a, c->stream); }))) return rc;
   } else if (c->kernel == BOIDS_KERNEL_SIMPLE) {
+    c->last_path = BOIDS_PATH_SIMPLE;
     if ((rc = launch(c, 0, [&] { return launch_search_simple(a, c->stream); }))) return rc;
     if ((rc = launch(c, 1, [&] { return launch_update(a, c->stream); }))) return rc;
   } else {
@@ -487,11 +496,13 @@ int one_step(boids_ctx* c, float dt) {
            }, 3)))
         return rc;
       c->since_sort = 0;
+      c->steps_sorted++;
     }
     c->since_sort++;
     if (think) {
       // this step's thinkers, in spatial order, split into never-searched (cold)
       // and warm-bounded ones
+      c->last_path = BOIDS_PATH_THINK;
       CK(cudaMemsetAsync(c->tcnt, 0, 2 * sizeof(int32_t), c->stream));
       if ((rc = launch(c, 2, [&] {
              return launch_think_compact(a, c->qperm, c->tcold, c->tcnt, c->twarm, c->tcnt + 1, c->stream);
@@ -522,6 +533,7 @@ int one_step(boids_ctx* c, float dt) {
         return e ? atoll(e) : 8192LL;
       }();
       if (c->symmetric && c->sym_sp && c->nloc >= sym_min) {
+        c->last_path = BOIDS_PATH_SYM;
         StepArgs as = a;
         as.routed = c->routed;  // agents routed to k_route by k_sym_prep (k_select skips them)
         CK(cudaMemsetAsync(c->sym_rcount, 0, sizeof(int32_t), c->stream));
@@ -535,6 +547,7 @@ int one_step(boids_ctx* c, float dt) {
         if ((rc = launch(c, 1, [&] { return launch_warm_select(as, c->stream, false); }))) return rc;
         if ((rc = launch(c, 4, [&] { return launch_route(as, c->stream); }))) return rc;
       } else {
+        c->last_path = BOIDS_PATH_SCAN;
         CK(cudaMemsetAsync(c->sym_rcount, 0, sizeof(int32_t), c->stream));
         if ((rc = launch(c, 0, [&] { return launch_warm_scan(a, c->stream); }, 2))) return rc;
         if ((rc = launch(c, 1, [&] { return launch_warm_select(a, c->stream); }))) return rc;
@@ -542,6 +555,7 @@ int one_step(boids_ctx* c, float dt) {
       }
     } else {
       // cold step (no previous lists) or forced: the cluster kernel
+      c->last_path = BOIDS_PATH_FUSED;
       int cl = c->cluster_opt;
       if ((rc = launch(c, 0, [&] { return launch_fused(a, cl, c->stream); }))) return rc;
     }
@@ -754,34 +768,11 @@ BOIDS_API int boids_get_state(boids_ctx* c, float* pos3, float* fwd3, float* up3
 // (measured: C4 with Morton-renumbered ids 2.79 -> 3.60 ms/step until the next
 // refresh), so boids_set_state has it rebuilt on the next step -- unless the
 // upload keeps the arrangement (the usual case: the caller's copy of the last
-// state, moved a little).  Test: 256 strided pairs of consecutive qperm entries;
-// the order is kept if at least half of them are still within the search radius
-// of each other in the uploaded positions.  Only a performance decision.
-static bool order_still_spatial(boids_ctx* c, const float* pos3) {
-  const int64_t k = c->nloc;
-  if (!c->qperm || k < 64) return false;
-  const int64_t stride = std::max<int64_t>(1, (k - 1) / 256);
-  const int64_t cnt = std::min<int64_t>(256, (k - 1) / stride);
-  std::vector<int32_t> pr((size_t)(2 * cnt));
-  if (cudaMemcpy2DAsync(pr.data(), 2 * sizeof(int32_t), c->qperm, (size_t)stride * sizeof(int32_t),
-                        2 * sizeof(int32_t), (size_t)cnt, cudaMemcpyDeviceToHost, c->stream) != cudaSuccess ||
-      cudaStreamSynchronize(c->stream) != cudaSuccess)
-    return false;
-  const float r2 = c->p.search_radius * c->p.search_radius;
-  int64_t valid = 0, near = 0;
-  for (int64_t t = 0; t < cnt; ++t) {
-    const int64_t a = pr[2 * t], b = pr[2 * t + 1];
-    if (a < 0 || a >= k || b < 0 || b >= k) continue;
-    ++valid;
-    float d2 = 0.f;
-    for (int d = 0; d < 3; ++d) {
-      const float x = pos3[3 * a + d] - pos3[3 * b + d];
-      d2 += x * x;
-    }
-    near += d2 <= r2 ? 1 : 0;
-  }
-  return valid > 0 && 2 * near >= valid;
-}
+// state, moved a little).  Test (k_order_check, on the device, reading the
+// staged positions): 256 strided pairs of consecutive qperm entries; the order is
+// kept if at least half of them are still within the search radius of each
+// other.  Only a performance decision; its 8-byte result rides on set_state's
+// own synchronisation.
 
 BOIDS_API int boids_set_state(boids_ctx* c, const float* pos3, const float* fwd3, const float* up3,
                     const float* side3, const float* speed) {
@@ -805,8 +796,15 @@ BOIDS_API int boids_set_state(boids_ctx* c, const float* pos3, const float* fwd3
   // on the 7th neighbour distance for ANY positions, so the next step stays exact;
   // a poor bound only costs time.  boids_get_neighbors still reports the lists of
   // the last step until the next step.
-  if (c->since_sort >= 0 && !order_still_spatial(c, pos3)) c->since_sort = -1;
+  int chk[2] = {0, 0};
+  const bool check = c->since_sort >= 0 && c->qperm && k >= 64;
+  if (check) {
+    CK(launch_order_check(st, c->qperm, k, c->p.search_radius * c->p.search_radius, c->ocheck, c->stream));
+    c->launches++;
+    CK(cudaMemcpyAsync(chk, c->ocheck, sizeof(chk), cudaMemcpyDeviceToHost, c->stream));
+  }
   CK(cudaStreamSynchronize(c->stream));
+  if (c->since_sort >= 0 && !(check && chk[0] > 0 && 2 * chk[1] >= chk[0])) c->since_sort = -1;
   c->steering_valid = false;
   return BOIDS_OK;
 }
@@ -882,6 +880,9 @@ BOIDS_API int boids_info(boids_ctx* c, boids_info_t* o) {
   o->fallbacks = (int64_t)st[2];
   o->grid_pairs = (int64_t)st[3];
   o->step_index = c->step_index;
+  o->last_path = c->last_path;
+  o->reserved0 = 0;
+  o->steps_sorted = c->steps_sorted;
   return BOIDS_OK;
 }
 
@@ -915,6 +916,46 @@ BOIDS_API int boids_get_phases(boids_ctx* c, uint64_t* out, int64_t count) {
   DeviceGuard g(c->dev);
   CK(cudaMemcpyAsync(out, c->phase, count * sizeof(uint64_t), cudaMemcpyDeviceToHost, c->stream));
   CK(cudaStreamSynchronize(c->stream));
+  return BOIDS_OK;
+}
+
+BOIDS_API int boids_bench_update(boids_ctx* c, float dt, int32_t reps, double* ms_per_launch) {
+  if (!c || !ms_per_launch) return fail(BOIDS_EINVAL, "NULL argument");
+  if (reps < 1) return fail(BOIDS_EINVAL, "reps must be >= 1");
+  int rc = check_dt(dt);
+  if (rc) return rc;
+  DeviceGuard g(c->dev);
+  const int64_t m = c->m;
+  if (!c->ubench) CK(cudaMalloc((void**)&c->ubench, (size_t)5 * m * sizeof(float4)));
+  StepArgs a = make_args(c, dt);
+  float4* su = c->ubench + 2 * m;
+  float4* ss = c->ubench + 3 * m;
+  float4* sa = c->ubench + 4 * m;
+  // the kernel updates the frame (and OpenSteer's smoothed acceleration) in place:
+  // give it copies, so the handle's state is untouched
+  CK(cudaMemcpyAsync(su, c->up4, m * sizeof(float4), cudaMemcpyDeviceToDevice, c->stream));
+  CK(cudaMemcpyAsync(ss, c->side4, m * sizeof(float4), cudaMemcpyDeviceToDevice, c->stream));
+  if (c->acc4) CK(cudaMemcpyAsync(sa, c->acc4, m * sizeof(float4), cudaMemcpyDeviceToDevice, c->stream));
+  a.out = c->ubench;
+  a.up4 = su;
+  a.side4 = ss;
+  a.acc4 = c->acc4 ? sa : nullptr;
+  a.force4 = nullptr;
+  cudaEvent_t e0 = get_event(c), e1 = get_event(c);
+  double tot = 0.0;
+  for (int32_t r = 0; r < reps; ++r) {
+    CK(cudaEventRecord(e0, c->stream));
+    CK(launch_update(a, c->stream));
+    CK(cudaEventRecord(e1, c->stream));
+    CK(cudaEventSynchronize(e1));
+    float t = 0.f;
+    CK(cudaEventElapsedTime(&t, e0, e1));
+    tot += t;
+    c->launches++;
+  }
+  c->pool.push_back(e0);
+  c->pool.push_back(e1);
+  *ms_per_launch = tot / reps;
   return BOIDS_OK;
 }
 

@@ -197,6 +197,8 @@ cudaError_t launch_pack_draw(const float4* local, int64_t m, const float4* up4, 
                              float4* draw, cudaStream_t s);
 cudaError_t launch_state_in(const float* stage, bool has_side, int64_t k, float4* local, int64_t m, float4* up4,
                             float4* side4, cudaStream_t s);
+cudaError_t launch_order_check(const float* pos3, const int32_t* qperm, int64_t k, float r2, int* out,
+                               cudaStream_t s);
 cudaError_t launch_state_out(const float4* local, int64_t m, const float4* up4, const float4* side4, int64_t k,
                              float* stage, cudaStream_t s);
 cudaError_t launch_think_compact(const StepArgs& a, const int32_t* qperm, int32_t* cold, int32_t* ncold,

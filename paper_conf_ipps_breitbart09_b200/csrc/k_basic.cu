@@ -5,6 +5,7 @@
 // shared-memory position cache, Listing 6.2; separate modification
 // kernel) and doubles as the standalone HBM-bound update kernel of
 // SURVEY.md B5.  The default step is the fused kernel in k_fused.cu.
+#include <algorithm>
 #include "agent_update.cuh"
 
 namespace boids {
@@ -125,6 +126,45 @@ cudaError_t launch_state_out(const float4* local, int64_t m, const float4* up4, 
                              float* stage, cudaStream_t s) {
   if (k <= 0) return cudaSuccess;
   k_state_out<<<(unsigned)((k + 255) / 256), 256, 0, s>>>(local, m, up4, side4, k, stage);
+  return cudaGetLastError();
+}
+
+// boids_set_state's locality check (only a performance decision, never a
+// result): does the spatial query order qperm still group nearby agents in the
+// uploaded positions?  Up to 256 strided pairs of consecutive qperm entries;
+// out[0] = valid pairs, out[1] = pairs still within the search radius.  Reads
+// the positions from the staging buffer (AoS pos3 = stage[0 .. 3k)).
+__global__ void k_order_check(const float* __restrict__ pos3, const int32_t* __restrict__ qperm, int64_t k,
+                              int64_t stride, int64_t cnt, float r2, int* __restrict__ out) {
+  __shared__ int sv, sn;
+  if (threadIdx.x == 0) sv = sn = 0;
+  __syncthreads();
+  const int64_t t = threadIdx.x;
+  if (t < cnt) {
+    const int64_t a = qperm[t * stride], b = qperm[t * stride + 1];
+    if (a >= 0 && a < k && b >= 0 && b < k) {
+      float d2 = 0.f;
+      for (int d = 0; d < 3; ++d) {
+        const float x = __fsub_rn(pos3[3 * a + d], pos3[3 * b + d]);
+        d2 = __fadd_rn(d2, __fmul_rn(x, x));
+      }
+      atomicAdd(&sv, 1);
+      if (d2 <= r2) atomicAdd(&sn, 1);
+    }
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    out[0] = sv;
+    out[1] = sn;
+  }
+}
+
+cudaError_t launch_order_check(const float* pos3, const int32_t* qperm, int64_t k, float r2, int* out,
+                               cudaStream_t s) {
+  if (k < 2) return cudaMemsetAsync(out, 0, 2 * sizeof(int), s);
+  const int64_t stride = std::max<int64_t>(1, (k - 1) / 256);
+  const int64_t cnt = std::min<int64_t>(256, (k - 1) / stride);
+  k_order_check<<<1, 256, 0, s>>>(pos3, qperm, k, stride, cnt, r2, out);
   return cudaGetLastError();
 }
 

@@ -1,7 +1,8 @@
 // k_warm.cu -- the warm-start Boids step: k_scan (all pairs, stream-K balanced)
 // + k_select (top-7, steering, modification).  Used for every step whose
-// previous step left neighbour lists for all owned agents (the cold step -- the
-// first one, or the first after boids_set_state -- runs k_fused).
+// previous step left neighbour lists for all owned agents (only the cold step --
+// the very first one, before any lists exist -- runs k_fused; boids_set_state
+// keeps the lists as bound seeds, so the step after an upload is warm too).
 //
 // Why a second design.  With the warm threshold t0_i = max over the previous
 // step's 7 neighbours j of d2(i, j) at the CURRENT positions, the true 7th key

@@ -48,15 +48,17 @@ def test_struct_layout_matches_header(tmp_path):
 
     src = tmp_path / "probe.c"
     src.write_text('#include <stddef.h>\n#include <stdio.h>\n#include "boids.h"\n'
-                   'int main(void){printf("%zu %zu %zu %zu %zu\\n", sizeof(boids_params), '
+                   'int main(void){printf("%zu %zu %zu %zu %zu %zu %zu\\n", sizeof(boids_params), '
                    'offsetof(boids_params, think_every), sizeof(boids_info_t), '
-                   'offsetof(boids_info_t, cluster), offsetof(boids_info_t, step_index));return 0;}\n')
+                   'offsetof(boids_info_t, cluster), offsetof(boids_info_t, step_index), '
+                   'offsetof(boids_info_t, last_path), offsetof(boids_info_t, steps_sorted));return 0;}\n')
     exe = tmp_path / "probe"
     subprocess.check_call(["gcc", "-I", os.path.join(ROOT, "include"), str(src), "-o", str(exe)])
     got = list(map(int, subprocess.check_output([str(exe)], text=True).split()))
     assert got == [C.sizeof(abi.boids_params), abi.boids_params.think_every.offset,
                    C.sizeof(abi.boids_info_t), abi.boids_info_t.cluster.offset,
-                   abi.boids_info_t.step_index.offset]
+                   abi.boids_info_t.step_index.offset, abi.boids_info_t.last_path.offset,
+                   abi.boids_info_t.steps_sorted.offset]
 
 
 def test_default_params_match_design_table(boidslib, orc):

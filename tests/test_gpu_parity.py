@@ -445,26 +445,48 @@ def test_config_c5_sampled(pk, orc):
 
 
 # ----------------------------------------- double-buffered readback
-def test_readback_draw_matrix_double_buffered(pk):
+def test_readback_draw_matrix_double_buffered(pk, orc):
     """boids_readback_begin packs the 4x4 draw matrices (side, up, fwd, pos) of the
-    current state and copies them on a second stream while later steps run."""
+    current state and copies them on a second stream while later steps run; the
+    two alternating buffers must hold the oracle's states of the last two steps,
+    packed as rows (x, y, z, 0|0|0|1)."""
     import torch
 
     from paper_conf_ipps_breitbart09_b200 import abi
 
     n = 5000
     p = pk.boids_default_params(init_mode=1)
+    op = _oparams(orc, p)
     bufs = [torch.empty((n, 4, 4), dtype=torch.float32, pin_memory=True).numpy() for _ in range(2)]
-    with pk.Flock(n, p, seed=4) as f, pk.Flock(n, p, seed=4) as ref:
-        states = []
+    o = orc.init(n, op, seed=4)
+    states = []
+    with pk.Flock(n, p, seed=4) as f:
         for t in range(4):
             f.step(DT, 1)
             abi.boids_readback_begin(f.h, bufs[t % 2])  # waits for the previous copy only
-            ref.step(DT, 1)
-            states.append(ref.state())
+            o, _, _, _ = orc.step(o, DT, op)
+            states.append(o)
         abi.boids_readback_wait(f.h)
-        for t in (2, 3):  # the two buffers hold the last two steps
-            m, s = bufs[t % 2], states[t]
-            assert np.array_equal(m[:, 0, :3], s["side"]) and np.array_equal(m[:, 1, :3], s["up"])
-            assert np.array_equal(m[:, 2, :3], s["fwd"]) and np.array_equal(m[:, 3, :3], s["pos"])
-            assert (m[:, :3, 3] == 0).all() and (m[:, 3, 3] == 1).all()
+    for t in (2, 3):  # the two buffers hold the last two steps
+        m, s = bufs[t % 2], states[t]
+        expect = np.zeros((n, 4, 4), np.float32)
+        expect[:, 0, :3], expect[:, 1, :3], expect[:, 2, :3], expect[:, 3, :3] = s["side"], s["up"], s["fwd"], s["pos"]
+        expect[:, 3, 3] = 1.0
+        assert np.array_equal(m, expect), f"step {t}"
+
+
+@pytest.mark.parametrize("n", [64, 100, 300, 511, 512, 513])
+def test_set_state_between_steps_small_n(pk, orc, n):
+    """step, set_state, step at the sizes where boids_set_state's locality check
+    samples consecutive qperm entries with stride 1 (a strided copy
+    with pitch < width failed there and poisoned the next step); the second step
+    must succeed and match the oracle from the uploaded state."""
+    s = W.ball_flock(n, seed=n, radius=10.0)
+    with pk.Flock(n, seed=1, record_steering=True) as f:
+        f.step(DT, 2)
+        f.set_state(s)
+        f.step(DT, 1)
+        f.sync()
+        o_state, o_idx, _, o_F = orc.step(orc.State(s), DT)
+        np.testing.assert_array_equal(f.neighbors()[0], o_idx)
+        assert bitexact(f.state(), o_state) and np.array_equal(f.steering(), o_F)

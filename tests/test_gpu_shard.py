@@ -4,10 +4,12 @@
   0..G-1) in one process; the per-step NCCL all-gather is emulated by device
   copies of every rank's send slice into every rank's full buffer (the exact
   layout all_gather_into_tensor produces).  The gathered state after k steps
-  must be bit-identical to one single-rank handle: same per-agent arithmetic,
-  same (d2, index) order, whatever the partition.
+  and the last step's neighbour lists must be bit-identical to the CPU
+  oracle's k steps from its own Appendix-B init (same per-agent arithmetic,
+  same (d2, index) order, whatever the partition).
 * ShardedFlock over a real NCCL process group of size 1 (torch.distributed,
-  all_gather_into_tensor on zero-copy views of the library's buffers).
+  all_gather_into_tensor on zero-copy views of the library's buffers), against
+  the oracle the same way.
 """
 import os
 import socket
@@ -54,20 +56,28 @@ def _emulated_run(pk, n, world, params, steps, seed=1):
 
 @pytest.mark.parametrize("mode,n,world,steer", [(0, 3000, 2, 0), (0, 5000, 3, 0), (0, 1000, 8, 0), (1, 20000, 4, 0),
                                                 (1, 777, 2, 0), (0, 3000, 3, 1), (1, 5000, 2, 1)])
-def test_shard_emulation_bitidentical(boidslib, mode, n, world, steer):
+def test_shard_emulation_bitidentical(boidslib, orc, mode, n, world, steer):
     """steer = 1: OpenSteer steering, whose smoothed accelerations live with the owner."""
     import paper_conf_ipps_breitbart09_b200 as pk
 
     p = pk.boids_default_params(init_mode=1, search_mode=mode, world_radius=20.0, steer_mode=steer)
     steps = 4
     got, got_nbr = _emulated_run(pk, n, world, p, steps)
-    with pk.Flock(n, p, seed=1) as f:
-        f.step(DT, steps)
-        ref = f.state()
-        ref_nbr = f.neighbors()[0]
+    ref, ref_nbr = _oracle_run(orc, n, p, steps, seed=1)
     assert np.array_equal(got_nbr, ref_nbr)
     for k in KEYS:
         assert np.array_equal(got[k], ref[k]), k
+
+
+def _oracle_run(orc, n, p, steps, seed):
+    """The oracle's `steps` synchronous steps from its own Appendix-B init; returns
+    the state and the last step's neighbour lists."""
+    op = orc.default_params(**{name: getattr(p, name) for name, _ in p._fields_})
+    o = orc.init(n, op, seed=seed)
+    idx = None
+    for _ in range(steps):
+        o, idx, _, _ = orc.step(o, DT, op)
+    return o, idx
 
 
 def _free_port():
@@ -78,7 +88,7 @@ def _free_port():
     return p
 
 
-def test_sharded_flock_nccl_single_rank(boidslib):
+def test_sharded_flock_nccl_single_rank(boidslib, orc):
     import torch
     import torch.distributed as dist
 
@@ -97,10 +107,8 @@ def test_sharded_flock_nccl_single_rank(boidslib):
         got = sf.state()
         got_nbr = sf.neighbors()[0]
         sf.close()
-        with pk.Flock(n, p, seed=3) as f:
-            f.step(DT, 5)
-            ref = f.state()
-            assert np.array_equal(got_nbr, f.neighbors()[0])
+        ref, ref_nbr = _oracle_run(orc, n, p, 5, seed=3)
+        assert np.array_equal(got_nbr, ref_nbr)
         for k in KEYS:
             assert np.array_equal(got[k], ref[k]), k
     finally:
