@@ -339,7 +339,7 @@ int create_impl(int64_t n, const boids_params* p, uint64_t seed, int32_t rank, i
              (rc = alloc((void**)&c->rbcount, (size_t)m * sizeof(int32_t))) ||
              (!shard && ((rc = alloc((void**)&c->sym_sp, sym_capacity(c->nloc) * sizeof(float4))) ||
                          (rc = alloc((void**)&c->sym_idx, sym_capacity(c->nloc) * sizeof(int32_t))) ||
-                         (rc = alloc((void**)&c->sym_fb, 2 * SYM_FB_LEN * sizeof(long long)))))) {
+                         (rc = alloc((void**)&c->sym_fb, (2 * SYM_FB_LEN + SYM_FB_MAX_CTAS + 1) * sizeof(long long)))))) {
     free_ctx(c);
     return rc;
   }
@@ -541,7 +541,8 @@ int one_step(boids_ctx* c, float dt) {
         long long* fb_cur = c->sym_fb + c->sym_fb_par * SYM_FB_LEN;
         c->sym_fb_par ^= 1;
         if ((rc = launch(c, 0, [&] {
-               return launch_sym_scan(as, c->sym_sp, c->sym_idx, c->balance ? fb_prev : nullptr, fb_cur, c->stream);
+               return launch_sym_scan(as, c->sym_sp, c->sym_idx, c->balance ? fb_prev : nullptr, fb_cur,
+                                      c->sym_fb + 2 * SYM_FB_LEN, c->stream);
              }, 2)))
           return rc;
         if ((rc = launch(c, 1, [&] { return launch_warm_select(as, c->stream, false); }))) return rc;

@@ -218,8 +218,9 @@ int64_t sym_capacity(int64_t nloc);
 // [2 + 3j] L0, [3 + 3j] L1, [4 + 3j] SM cycles the CTA took.
 constexpr int SYM_FB_MAX_CTAS = 1024;
 constexpr int SYM_FB_LEN = 2 + 3 * SYM_FB_MAX_CTAS;
+// splits: [SYM_FB_MAX_CTAS + 1] int64 scratch: k_sym_prep writes every k_sym CTA's item range there
 cudaError_t launch_sym_scan(const StepArgs& a, float4* sp, int* sidx, const long long* fb_prev, long long* fb_cur,
-                            cudaStream_t s);
+                            long long* splits, cudaStream_t s);
 cudaError_t launch_route(const StepArgs& a, cudaStream_t s);
 int fused_auto_cluster(int64_t n_pad_total, int64_t nloc, int sm_count);
 

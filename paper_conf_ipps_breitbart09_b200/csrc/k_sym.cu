@@ -49,8 +49,9 @@ constexpr int STAGES = BOIDS_SYM_STAGES;
 // 256-thread CTAs run two per SM: the ring shrinks so two fit in shared memory
 template <int NT>
 __host__ __device__ constexpr int sym_stages() { return NT == 256 ? 12 : STAGES; }
-constexpr int U = 4;        // candidates per warp vote
-constexpr int WB = Q * U * 32;  // records per warp buffer: one vote group's maximum per side
+constexpr int U = 4;        // candidates per record-emission subgroup (the slow path)
+constexpr int UG = 8;       // candidates per warp vote (the fast path); item ranges are multiples of UG
+constexpr int WB = Q * U * 32;  // records per warp buffer: one subgroup's maximum per side
 
 struct __align__(8) Rec {
   int qi;  // local agent whose buffer receives the key
@@ -58,13 +59,22 @@ struct __align__(8) Rec {
   key_t key;
 };
 
+// Ring stages hold a tile as structure of arrays (x[CT], y[CT], z[CT], lim[CT],
+// index[CT]): a 16-byte shared load then gives four candidates' x (or y, z) --
+// two packed pairs for FADD2 with the query's coordinate as a broadcast operand.
 template <int NT>
 struct __align__(16) SymSmem {
-  float4 ring[sym_stages<NT>()][CT];
+  float rx[sym_stages<NT>()][CT];
+  float ry[sym_stages<NT>()][CT];
+  float rz[sym_stages<NT>()][CT];
+  float rw[sym_stages<NT>()][CT];
   int ridx[sym_stages<NT>()][CT];
   Rec rec[NT / 32][WB];
+  int qg[NT / 32][Q * 32];    // each warp's current query group: agent indices ...
+  float ql[NT / 32][Q * 32];  // ... and limits (read on the slow path only)
   uint64_t full[sym_stages<NT>()];
-  int rel[sym_stages<NT>()];  // warps done with the tile in the stage (the last one refills it)
+  int rel[sym_stages<NT>()];  // query groups done with the tile in the stage (the last one refills it)
+  int next_unit;              // work queue of (tile, query group) units
 };
 
 // 8 records per lane per round: the atomics' round trips overlap.
@@ -83,6 +93,17 @@ __device__ __forceinline__ void flush(const StepArgs& a, const Rec* rec, int n, 
     for (int k = 0; k < 8; ++k)
       if (slot[k] < a.hits_cap) a.hits[(int64_t)r[k].qi * a.hits_cap + slot[k]] = r[k].key;
   }
+}
+
+// A 16-byte shared-memory load the compiler cannot merge with an earlier load of
+// the same address: the slow path recomputes the fast path's distances from its
+// own loads, so nothing of the fast path stays live (in registers) across the vote.
+__device__ __forceinline__ float4 lds_fresh(const float* p) {
+  float4 v;
+  asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];"
+               : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w)
+               : "r"((unsigned)__cvta_generic_to_shared(p)));
+  return v;
 }
 
 // Items before query block b: S(b) = sum_{b' < b} (npad - b'*QB).
@@ -149,7 +170,7 @@ __device__ __forceinline__ int64_t sym_split(int64_t i, int64_t grid, int64_t np
   }
   const int64_t o = x - sw(lo), dw = (int64_t)wd4 * qb;
   const int64_t off = o < dw ? o / wd4 : qb + (o - dw) / 4;
-  return (sym_prefix(lo, npad, qb) + off) / U * U;
+  return (sym_prefix(lo, npad, qb) + off) / UG * UG;
 }
 
 // Feedback split (BOIDS_OPT_BALANCE).  The cost of an item is not uniform: the
@@ -159,49 +180,68 @@ __device__ __forceinline__ int64_t sym_split(int64_t i, int64_t grid, int64_t np
 // every CTA's SM time for its range [L0_j, L1_j); read as a piecewise-constant
 // cost density over the item space, it gives a cumulative cost C(x), and CTA i
 // takes [C^-1(i T / G), C^-1((i + 1) T / G)), T = C(total), rounded to U.  The
-// flock moves little per step, so the density carries over.  Every CTA computes
-// the same boundaries from the same record, so the ranges tile the item space
-// exactly; only the partition changes, never a result.  Returns false (static
-// split) when the record is missing or from another launch shape.  Warp 0 only.
-__device__ bool fb_split(const long long* fb, int G, int64_t total, int i, int lane, int64_t& l0, int64_t& l1) {
-  if (fb == nullptr || G > SYM_FB_MAX_CTAS || fb[0] != G || fb[1] != total) return false;
-  const int per = (G + 31) / 32, j0 = min(G, lane * per), j1 = min(G, j0 + per);
-  double own = 0.0;
-  for (int j = j0; j < j1; ++j) own += (double)fb[4 + 3 * j];
-  double incl = own;
+// flock moves little per step, so the density carries over.  Only the partition
+// changes, never a result.  Without a usable record (first launch, another
+// launch shape) the static weighted split (sym_split) is used.
+//
+// k_sym_prep's block 0 computes all G + 1 boundaries into `splits` (one
+// thread per boundary, binary search over a shared-memory prefix of the costs),
+// off k_sym's critical path: k_sym's CTAs then read their two boundaries.
+__device__ void compute_splits(const long long* __restrict__ fb, int G, int64_t total, int64_t npad, int64_t qb,
+                               int wd4, long long* __restrict__ splits) {
+  __shared__ double pre[SYM_FB_MAX_CTAS];
+  __shared__ double wsum[32];
+  __shared__ int ok;
+  const int tid = threadIdx.x, nt = blockDim.x, lane = tid & 31, warp = tid >> 5;
+  if (tid == 0) ok = fb != nullptr && G <= SYM_FB_MAX_CTAS && fb[0] == G && fb[1] == total;
+  __syncthreads();
+  if (ok) {  // inclusive prefix of the measured CTA costs (block scan over per-thread chunks)
+    const int per = (G + nt - 1) / nt, j0 = min(G, tid * per), j1 = min(G, j0 + per);
+    double own = 0.0;
+    for (int j = j0; j < j1; ++j) own += (double)fb[4 + 3 * j];
+    double incl = own;
 #pragma unroll
-  for (int o = 1; o < 32; o <<= 1) {
-    const double v = __shfl_up_sync(0xffffffffu, incl, o);
-    if (lane >= o) incl += v;
-  }
-  const double T = __shfl_sync(0xffffffffu, incl, 31), excl = incl - own;
-  if (!(T > 0.0)) return false;
-  auto bound = [&](int k) -> int64_t {
-    if (k <= 0) return 0;
-    if (k >= G) return total;
-    const double c = T * (double)k / (double)G;
-    const unsigned owner = __ballot_sync(0xffffffffu, j1 > j0 && excl <= c && c < incl);
-    const int src = owner ? __ffs(owner) - 1 : 31;
-    int64_t x = total;
-    if (lane == src) {
-      double cum = excl;
-      for (int j = j0; j < j1; ++j) {
-        const double t = (double)fb[4 + 3 * j];
-        if (c < cum + t) {
-          const int64_t a0 = fb[2 + 3 * j], a1 = fb[3 + 3 * j];
-          x = a0 + (int64_t)((c - cum) / t * (double)(a1 - a0));
-          break;
-        }
-        cum += t;
-      }
+    for (int o = 1; o < 32; o <<= 1) {
+      const double v = __shfl_up_sync(0xffffffffu, incl, o);
+      if (lane >= o) incl += v;
     }
-    x = __shfl_sync(0xffffffffu, x, src);
-    x = x / U * U;
-    return x < 0 ? 0 : (x > total ? total : x);
-  };
-  l0 = bound(i);
-  l1 = bound(i + 1);
-  return true;
+    if (lane == 31) wsum[warp] = incl;
+    __syncthreads();
+    double woff = 0.0;
+    for (int w = 0; w < warp; ++w) woff += wsum[w];
+    double run = woff + incl - own;
+    for (int j = j0; j < j1; ++j) {
+      run += (double)fb[4 + 3 * j];
+      pre[j] = run;
+    }
+    __syncthreads();
+    if (tid == 0 && !(pre[G - 1] > 0.0)) ok = 0;
+    __syncthreads();
+  }
+  const double T = ok ? pre[G - 1] : 0.0;
+  for (int k = tid; k <= G; k += nt) {
+    int64_t x;
+    if (k == 0) {
+      x = 0;
+    } else if (k == G) {
+      x = total;
+    } else if (ok) {
+      const double c = T * (double)k / (double)G;
+      int lo = 0, hi = G - 1;  // first j with pre[j] > c
+      while (lo < hi) {
+        const int mid = (lo + hi) >> 1;
+        if (pre[mid] > c) hi = mid; else lo = mid + 1;
+      }
+      const double t = (double)fb[4 + 3 * lo], cum = pre[lo] - t;
+      const int64_t a0 = fb[2 + 3 * lo], a1 = fb[3 + 3 * lo];
+      x = t > 0.0 ? a0 + (int64_t)((c - cum) / t * (double)(a1 - a0)) : a0;
+      x = x / UG * UG;
+      x = x < 0 ? 0 : (x > total ? total : x);
+    } else {
+      x = sym_split(k, G, npad, qb, wd4);
+    }
+    splits[k] = x;
+  }
 }
 
 // Tile k of a CTA whose item range is [L0, L1): items [max(L0, A + k*CT), min(L1,
@@ -215,9 +255,10 @@ struct TileDesc {
 __device__ __forceinline__ TileDesc tile_desc(int k, int64_t L0, int64_t L1, int64_t npad, int64_t qb) {
   const int64_t A = L0 / CT * CT;
   const int64_t Ls = max(L0, A + (int64_t)k * CT), Le = min(L1, A + (int64_t)(k + 1) * CT);
-  // row: largest b with S(b) <= Ls; S is increasing and concave -> solve, then fix up
-  const double nb2 = (double)npad / (double)qb + 0.5;
-  int64_t b = (int64_t)(nb2 - sqrt(fmax(0.0, nb2 * nb2 - 2.0 * (double)Ls / (double)qb)));
+  // row: largest b with S(b) <= Ls; S is increasing and concave -> solve in fp32
+  // (a few ulps off at most: the integer fix-ups below make it exact), then fix up
+  const float nb2 = (float)npad / (float)qb + 0.5f;
+  int64_t b = (int64_t)(nb2 - sqrtf(fmaxf(0.f, nb2 * nb2 - 2.f * (float)Ls / (float)qb)));
   b = b < 0 ? 0 : b;
   while (b > 0 && sym_prefix(b, npad, qb) > Ls) --b;
   while (sym_prefix(b + 1, npad, qb) <= Ls) ++b;
@@ -226,41 +267,49 @@ __device__ __forceinline__ TileDesc tile_desc(int k, int64_t L0, int64_t L1, int
 
 template <int NTS>
 __global__ void __launch_bounds__(NTS, NTS == 128 ? 4 : (NTS == 256 ? 2 : 1))
-    k_sym(StepArgs a, const float4* __restrict__ sp, const int* __restrict__ sidx, int64_t npad, int wd4,
-          const long long* __restrict__ fb_prev, long long* __restrict__ fb_cur) {
+    k_sym(StepArgs a, const float* __restrict__ spf, int64_t cap, const int* __restrict__ sidx, int64_t npad,
+          const long long* __restrict__ splits, long long* __restrict__ fb_cur) {
   constexpr int QBS = NTS * Q, NW = NTS / 32, SST = sym_stages<NTS>();
   extern __shared__ __align__(16) unsigned char smem_raw[];
   SymSmem<NTS>& sm = *reinterpret_cast<SymSmem<NTS>*>(smem_raw);
   __shared__ int64_t s_range[2];
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   pdl_wait();  // k_sym_prep's sp / limits (and the previous launch's feedback record)
-  const long long c_start = clock64();
+  __shared__ long long s_cstart;
+  __shared__ unsigned long long s_tw[NTS / 32], s_ts[NTS / 32];  // diagnostics (a.phase): per-warp wait / emit cycles
+  if (tid == 0) s_cstart = clock64();
+  if (tid < NTS / 32) s_tw[tid] = s_ts[tid] = 0;
   const int64_t total = sym_prefix(npad / QBS, npad, QBS);
-  if (warp == 0) {
-    int64_t l0, l1;
-    if (!fb_split(fb_prev, (int)gridDim.x, total, (int)blockIdx.x, lane, l0, l1)) {
-      l0 = sym_split(blockIdx.x, gridDim.x, npad, QBS, wd4);
-      l1 = sym_split(blockIdx.x + 1, gridDim.x, npad, QBS, wd4);
-    }
-    if (lane == 0) {
-      s_range[0] = l0;
-      s_range[1] = l1;
-    }
-  }
+  if (tid < 2) s_range[tid] = splits[blockIdx.x + tid];  // k_sym_prep's boundaries (compute_splits)
   __syncthreads();
   const int64_t L0 = s_range[0], L1 = s_range[1];
   const int ntiles = L1 > L0 ? (int)((L1 + CT - 1) / CT - L0 / CT) : 0;
+  // Work units.  Unit u = (tile k = u / NW, query group w = u % NW): the 128
+  // candidates of tile k against the 4 x 32 queries [w*128, (w+1)*128) of tile
+  // k's query block.  Warps take units from a shared counter, in order, instead
+  // of each warp owning one query group: the slow path of a tile (passing pairs,
+  // record emission) concentrates in the query group next to it in space -- on
+  // the diagonal, tile k is hot for group k only -- and with fixed groups that
+  // one warp set the CTA's end while the others waited at the final barrier
+  // (C3: stall_barrier 20 % of samples).  Taken dynamically, hot units spread
+  // over whichever warps are free.
+  //
   // Ring protocol: stage s = k % SST holds tile k.  full[s] completes when the
-  // tile's bytes land (TMA complete_tx).  Each warp, when done with tile k,
-  // increments rel[s]; the LAST of the NW warps refills the stage with tile
-  // k + SST.  So the refill waits only for the slowest warp on that tile and
-  // no warp is the dedicated producer: warps drift up to SST - 1 tiles apart.
+  // tile's bytes land (TMA complete_tx).  Each finished unit of tile k
+  // increments rel[s]; the unit that completes the tile's NW query groups
+  // refills the stage with tile k + SST.  A warp takes a new unit only after
+  // finishing its current one, so at most NW units are open: a unit of tile
+  // k + SST can only be taken once tile k's units are all taken, and its wait
+  // on full[s] (parity of k + SST) cannot be satisfied by tile k's phase.
   auto issue = [&](int k) {
     const TileDesc d = tile_desc(k, L0, L1, npad, QBS);
     const int s = k % SST;
     const uint32_t n = (uint32_t)d.cnt;
     mbar_arrive_expect_tx(&sm.full[s], n * 20u);
-    tma_load_1d(sm.ring[s], sp + d.jb, n * 16u, &sm.full[s]);
+    tma_load_1d(sm.rx[s], spf + d.jb, n * 4u, &sm.full[s]);
+    tma_load_1d(sm.ry[s], spf + cap + d.jb, n * 4u, &sm.full[s]);
+    tma_load_1d(sm.rz[s], spf + 2 * cap + d.jb, n * 4u, &sm.full[s]);
+    tma_load_1d(sm.rw[s], spf + 3 * cap + d.jb, n * 4u, &sm.full[s]);
     tma_load_1d(sm.ridx[s], sidx + d.jb, n * 4u, &sm.full[s]);
   };
   if (tid == 0) {
@@ -279,100 +328,166 @@ __global__ void __launch_bounds__(NTS, NTS == 128 ? 4 : (NTS == 256 ? 2 : 1))
       mbar_init(&sm.full[s], 1);
       sm.rel[s] = 0;
     }
+    sm.next_unit = 0;
     mbar_fence_init();
-    for (int k = 0; k < SST && k < ntiles; ++k) issue(k);
+  }
+  if (warp == 0) {  // the first SST tiles, one lane each
+    __syncwarp();
+    for (int k = lane; k < SST && k < ntiles; k += 32) issue(k);
   }
   __syncthreads();
   Rec* rec = sm.rec[warp];
   int wcount = 0;
   unsigned slow_groups = 0, groups = 0;
-  long long t_wait = 0, t_slow = 0;  // diagnostics (a.phase): cycles in full-barrier waits / emits
   int64_t cur_b = -1;
-  float2 pxy[Q];
-  float pz[Q], lim[Q], limq = 0.f;
-  int gq[Q], qpos[Q];
-  for (int k = 0; k < ntiles; ++k) {
+  int cur_w = -1;
+  float px[Q], py[Q], pz[Q], limq = 0.f;
+  int qbase = 0;  // sorted position of the thread's query 0 (query q: qbase + 32 q)
+  int* wqg = sm.qg[warp];
+  float* wql = sm.ql[warp];
+  const float INF = __int_as_float(0x7f800000);
+  const int nunits = ntiles * NW;
+  for (;;) {
+    int u = 0;
+    if (lane == 0) u = atomicAdd(&sm.next_unit, 1);
+    u = __shfl_sync(0xffffffffu, u, 0);
+    if (u >= nunits) break;
+    const int k = u / NW, wq = u - k * NW;
     const TileDesc td = tile_desc(k, L0, L1, npad, QBS);
-    if (td.b != cur_b) {  // this warp's 4 x 32 queries of row b (spatially compact)
+    if (td.b != cur_b || wq != cur_w) {  // query group wq of row b: 4 x 32 spatially compact queries
       cur_b = td.b;
+      cur_w = wq;
+      qbase = (int)(cur_b * QBS + wq * 32 * Q + lane);
+      float lq[Q];
+      __syncwarp();  // the previous group's slow path is done with wqg / wql
 #pragma unroll
       for (int q = 0; q < Q; ++q) {
-        const int p = (int)(cur_b * QBS + warp * 32 * Q + q * 32 + lane);
-        const float4 me = __ldg(sp + p);
-        qpos[q] = p;
-        gq[q] = __ldg(sidx + p);
-        pxy[q] = make_float2(me.x, me.y);
-        pz[q] = me.z;
-        lim[q] = me.w;
+        const int p = qbase + q * 32;
+        wqg[q * 32 + lane] = __ldg(sidx + p);
+        px[q] = __ldg(spf + p);
+        py[q] = __ldg(spf + cap + p);
+        pz[q] = __ldg(spf + 2 * cap + p);
+        lq[q] = __ldg(spf + 3 * cap + p);
+        wql[q * 32 + lane] = lq[q];
       }
-      limq = fmaxf(fmaxf(lim[0], lim[1]), fmaxf(lim[2], lim[3]));
+      limq = fmaxf(fmaxf(lq[0], lq[1]), fmaxf(lq[2], lq[3]));
     }
     const int s = k % SST;
     long long tw0 = 0;
     if (a.phase) tw0 = clock64();
     mbar_wait(&sm.full[s], (uint32_t)(k / SST) & 1u);
-    if (a.phase) t_wait += clock64() - tw0;
+    if (a.phase && lane == 0) s_tw[warp] += clock64() - tw0;
     {
-      const float4* tile = sm.ring[s];
+      const float* tx = sm.rx[s];
+      const float* ty = sm.ry[s];
+      const float* tz = sm.rz[s];
+      const float* tw = sm.rw[s];
       const int* tidx = sm.ridx[s];
-      const int jb = (int)td.jb, cnt = td.cnt;
+      const int jb = (int)td.jb;
+      const int cnt = td.cnt;  // a multiple of UG
       const bool diag = td.jb < (cur_b + 1) * QBS;  // candidates of the query block itself
-      auto group = [&](const int c, auto diag_c) {
+      // d2 of query q to candidates (c + 2p, c + 2p + 1), reading Q3: the x, y, z
+      // differences of the two pairs in one FADD2 each (query coordinate broadcast),
+      // their squares in one FMUL2 each, the sums ((dx dx) + (dy dy)) + (dz dz) scalar
+      // -- never a packed add of packed products, which ptxas would contract into FFMA2.
+      auto dist_pair = [&](int q, float4 X, float4 Y, float4 Z, int hi, float& d0, float& d1) {
+        const float2 cx = hi ? make_float2(X.z, X.w) : make_float2(X.x, X.y);
+        const float2 cy = hi ? make_float2(Y.z, Y.w) : make_float2(Y.x, Y.y);
+        const float2 cz = hi ? make_float2(Z.z, Z.w) : make_float2(Z.x, Z.y);
+        const float2 dx = __fadd2_rn(make_float2(px[q], px[q]), make_float2(-cx.x, -cx.y));
+        const float2 dy = __fadd2_rn(make_float2(py[q], py[q]), make_float2(-cy.x, -cy.y));
+        const float2 dz = __fadd2_rn(make_float2(pz[q], pz[q]), make_float2(-cz.x, -cz.y));
+        const float2 x2 = __fmul2_rn(dx, dx), y2 = __fmul2_rn(dy, dy), z2 = __fmul2_rn(dz, dz);
+        d0 = __fadd_rn(__fadd_rn(x2.x, y2.x), z2.x);
+        d1 = __fadd_rn(__fadd_rn(x2.y, y2.y), z2.y);
+      };
+      // Slow path of one subgroup of U = 4 candidates (c .. c+3): recompute its
+      // 16 distances (the same arithmetic, so the same floats as the fast path),
+      // test them against the exact limits, append the passing keys.
+      auto slow4 = [&](const int c, auto diag_c) {
         constexpr bool DIAG = decltype(diag_c)::value;
-        float4 cc[U];
-#pragma unroll
-        for (int u = 0; u < U; ++u) cc[u] = tile[c + u];
+        const float4 X = lds_fresh(tx + c);
+        const float4 Y = lds_fresh(ty + c);
+        const float4 Z = lds_fresh(tz + c);
+        const float4 W = lds_fresh(tw + c);
+        const float cw[U] = {W.x, W.y, W.z, W.w};
         float d[Q][U];
 #pragma unroll
-        for (int u = 0; u < U; ++u)
+        for (int q = 0; q < Q; ++q) {
+          dist_pair(q, X, Y, Z, 0, d[q][0], d[q][1]);
+          dist_pair(q, X, Y, Z, 1, d[q][2], d[q][3]);
+        }
+        int cidx[U], gq[Q];
+        float lim[Q];
 #pragma unroll
-          for (int q = 0; q < Q; ++q) {
-            const float2 dxy = __fadd2_rn(pxy[q], make_float2(-cc[u].x, -cc[u].y));
-            const float2 sq = __fmul2_rn(dxy, dxy);
-            const float dz = __fsub_rn(pz[q], cc[u].z);
-            d[q][u] = __fadd_rn(__fadd_rn(sq.x, sq.y), __fmul_rn(dz, dz));
+        for (int u = 0; u < U; ++u) cidx[u] = tidx[c + u];
+#pragma unroll
+        for (int q = 0; q < Q; ++q) {
+          gq[q] = wqg[q * 32 + lane];
+          lim[q] = wql[q * 32 + lane];
+        }
+        unsigned qb = 0, cb = 0;
+#pragma unroll
+        for (int q = 0; q < Q; ++q)
+#pragma unroll
+          for (int u = 0; u < U; ++u) {
+            if (d[q][u] <= lim[q] && (!DIAG || jb + c + u != qbase + q * 32)) qb |= 1u << (q * U + u);
+            if (!DIAG && d[q][u] <= cw[u]) cb |= 1u << (q * U + u);
           }
+        long long ts0 = 0;
+        if (a.phase) ts0 = clock64();
+        emit<0>(a, rec, wcount, lane, qb, d, gq, cidx);
+        if (!DIAG) emit<1>(a, rec, wcount, lane, cb, d, gq, cidx);
+        if (a.phase && lane == 0) s_ts[warp] += clock64() - ts0;
+      };
+      // Fast path of one vote group of UG = 8 candidates: only the minimum of the
+      // 32 distances per lane, against the largest limit that could accept a pair
+      // (the thread's queries', and on off-diagonal tiles the candidates' too);
+      // one warp vote -- nearly always false -- decides whether the slow path runs.
+      auto group = [&](const int c, auto diag_c) {
+        constexpr bool DIAG = decltype(diag_c)::value;
+        const float4 X0 = *reinterpret_cast<const float4*>(tx + c);
+        const float4 X1 = *reinterpret_cast<const float4*>(tx + c + 4);
+        const float4 Y0 = *reinterpret_cast<const float4*>(ty + c);
+        const float4 Y1 = *reinterpret_cast<const float4*>(ty + c + 4);
+        const float4 Z0 = *reinterpret_cast<const float4*>(tz + c);
+        const float4 Z1 = *reinterpret_cast<const float4*>(tz + c + 4);
         float mq[Q];
 #pragma unroll
         for (int q = 0; q < Q; ++q) {
-          mq[q] = d[q][0];
-#pragma unroll
-          for (int u = 1; u < U; ++u) mq[q] = fminf(mq[q], d[q][u]);
+          float e0, e1, e2, e3, e4, e5, e6, e7;
+          dist_pair(q, X0, Y0, Z0, 0, e0, e1);
+          dist_pair(q, X0, Y0, Z0, 1, e2, e3);
+          dist_pair(q, X1, Y1, Z1, 0, e4, e5);
+          dist_pair(q, X1, Y1, Z1, 1, e6, e7);
+          mq[q] = fminf(fminf(fminf(e0, e1), fminf(e2, e3)), fminf(fminf(e4, e5), fminf(e6, e7)));
         }
         const float m = fminf(fminf(mq[0], mq[1]), fminf(mq[2], mq[3]));  // NaN (phantoms) ignored
-        const float thr = DIAG ? limq : fmaxf(fmaxf(limq, fmaxf(cc[0].w, cc[1].w)), fmaxf(cc[2].w, cc[3].w));
+        float thr = limq;
+        if (!DIAG) {
+          const float4 W0 = *reinterpret_cast<const float4*>(tw + c);
+          const float4 W1 = *reinterpret_cast<const float4*>(tw + c + 4);
+          thr = fmaxf(fmaxf(fmaxf(thr, fmaxf(W0.x, W0.y)), fmaxf(W0.z, W0.w)),
+                      fmaxf(fmaxf(W1.x, W1.y), fmaxf(W1.z, W1.w)));
+        }
         ++groups;
         if (__any_sync(0xffffffffu, m <= thr)) {  // rare, warp-uniform
           ++slow_groups;
-          int cidx[U];
-#pragma unroll
-          for (int u = 0; u < U; ++u) cidx[u] = tidx[c + u];
-          unsigned qb = 0, cb = 0;
-#pragma unroll
-          for (int q = 0; q < Q; ++q)
-#pragma unroll
-            for (int u = 0; u < U; ++u) {
-              if (d[q][u] <= lim[q] && (!DIAG || jb + c + u != qpos[q])) qb |= 1u << (q * U + u);
-              if (!DIAG && d[q][u] <= cc[u].w) cb |= 1u << (q * U + u);
-            }
-          long long ts0 = 0;
-          if (a.phase) ts0 = clock64();
-          emit<0>(a, rec, wcount, lane, qb, d, gq, cidx);
-          if (!DIAG) emit<1>(a, rec, wcount, lane, cb, d, gq, cidx);
-          if (a.phase) t_slow += clock64() - ts0;
+#pragma unroll 1
+          for (int c4 = c; c4 < c + UG; c4 += U) slow4(c4, diag_c);
         }
       };
       if (!diag && cnt == CT) {  // full off-diagonal tile: constant trip count (the common case)
-#pragma unroll 4  // measured: 1 / 2 / 4 / 8 -> C4 2.92 / 2.89 / 2.83 / 2.83 ms (bench pattern)
-        for (int c = 0; c < CT; c += U) group(c, std::false_type{});
+#pragma unroll 1
+        for (int c = 0; c < CT; c += UG) group(c, std::false_type{});
       } else if (!diag) {
-        for (int c = 0; c < cnt; c += U) group(c, std::false_type{});
+        for (int c = 0; c < cnt; c += UG) group(c, std::false_type{});
       } else {
-        for (int c = 0; c < cnt; c += U) group(c, std::true_type{});
+        for (int c = 0; c < cnt; c += UG) group(c, std::true_type{});
       }
     }
     __syncwarp();
-    if (lane == 0) {  // release stage s; the last warp refills it with tile k + SST
+    if (lane == 0) {  // this query group is done with stage s; the tile's last one refills it
       __threadfence_block();
       const int old = atomicAdd(&sm.rel[s], 1);
       if (old == NW - 1) {
@@ -387,12 +502,12 @@ __global__ void __launch_bounds__(NTS, NTS == 128 ? 4 : (NTS == 256 ? 2 : 1))
   }
   __syncwarp();
   flush(a, rec, wcount, lane);
-  if (fb_cur) {  // this CTA's range and SM time: the next launch's split (fb_split)
+  if (fb_cur) {  // this CTA's range and SM time: the next launch's split (compute_splits)
     __syncthreads();
     if (tid == 0) {
       fb_cur[2 + 3 * blockIdx.x] = L0;
       fb_cur[3 + 3 * blockIdx.x] = L1;
-      fb_cur[4 + 3 * blockIdx.x] = clock64() - c_start;
+      fb_cur[4 + 3 * blockIdx.x] = clock64() - s_cstart;
       if (blockIdx.x == 0) {
         fb_cur[0] = gridDim.x;
         fb_cur[1] = total;
@@ -406,9 +521,9 @@ __global__ void __launch_bounds__(NTS, NTS == 128 ? 4 : (NTS == 256 ? 2 : 1))
   if (a.phase) {
     if (lane == 0) {
       atomicAdd(a.phase + blockIdx.x * 8 + 4, (unsigned long long)slow_groups);
-      atomicMax(a.phase + blockIdx.x * 8 + 5, (unsigned long long)t_wait);  // [5] max wait cycles of a warp
-      atomicMax(a.phase + blockIdx.x * 8 + 6, (unsigned long long)t_slow);  // [6] max emit cycles of a warp
-      if (warp == 0) a.phase[blockIdx.x * 8 + 7] = (unsigned long long)t_wait;  // [7] warp 0 wait
+      atomicMax(a.phase + blockIdx.x * 8 + 5, s_tw[warp]);  // [5] max wait cycles of a warp
+      atomicMax(a.phase + blockIdx.x * 8 + 6, s_ts[warp]);  // [6] max emit cycles of a warp
+      if (warp == 0) a.phase[blockIdx.x * 8 + 7] = s_tw[0];  // [7] warp 0 wait
     }
     __syncthreads();
     if (tid == 0) {
@@ -485,17 +600,22 @@ __device__ float window_bound(const StepArgs& a, int qi, float4 me) {
   return b[6];
 }
 
-// sp[p] = (x, y, z, min(prev(r2), t0)) of agent sidx[p] = qperm[p]; phantoms beyond nloc.
+// Structure of arrays over the sorted positions p: spf[p], spf[cap + p], spf[2 cap + p] = x, y, z and
+// spf[3 cap + p] = min(prev(r2), t0) of agent sidx[p] = qperm[p]; phantoms beyond nloc.
 // An agent whose previous 7 neighbours are all out of range now (t0 >= r2 with a
 // full previous list: it wrapped to the far side of the world) would append
 // every in-radius pair -- hundreds -- to its hit buffer.  It is ROUTED instead:
 // limit -1 (no hits on either side in k_sym) and searched whole by k_route.
-__device__ __forceinline__ void sym_prep_body(const StepArgs& a, float4* __restrict__ sp, int* __restrict__ sidx,
-                                              int64_t npad) {
+__device__ __forceinline__ void sym_prep_body(const StepArgs& a, float* __restrict__ spf, int64_t cap,
+                                              int* __restrict__ sidx, int64_t npad) {
   const int64_t p = (int64_t)blockIdx.x * 256 + threadIdx.x;
   if (p >= npad) return;
   if (p >= a.nloc) {
-    sp[p] = make_float4(__int_as_float(0x7fc00000), __int_as_float(0x7fc00000), __int_as_float(0x7fc00000), -1.f);
+    const float nan = __int_as_float(0x7fc00000);
+    spf[p] = nan;
+    spf[cap + p] = nan;
+    spf[2 * cap + p] = nan;
+    spf[3 * cap + p] = -1.f;
     sidx[p] = -1;
     return;
   }
@@ -513,15 +633,22 @@ __device__ __forceinline__ void sym_prep_body(const StepArgs& a, float4* __restr
     if (a.stats) atomicAdd(a.stats + 2, 1ull);
     lim = -1.f;
   }
-  sp[p] = make_float4(me.x, me.y, me.z, lim);
+  spf[p] = me.x;
+  spf[cap + p] = me.y;
+  spf[2 * cap + p] = me.z;
+  spf[3 * cap + p] = lim;
   sidx[p] = qi;
 }
 
-__global__ void __launch_bounds__(256) k_sym_prep(StepArgs a, float4* __restrict__ sp, int* __restrict__ sidx,
-                                                   int64_t npad) {
+__global__ void __launch_bounds__(256) k_sym_prep(StepArgs a, float* __restrict__ spf, int64_t cap,
+                                                   int* __restrict__ sidx, int64_t npad, int64_t qb, int G, int wd4,
+                                                   const long long* __restrict__ fb_prev,
+                                                   long long* __restrict__ splits) {
   pdl_trigger();  // k_sym may be scheduled now; it waits for this grid before reading sp
   span_begin(a, SPAN_SLOT0 + 0);
-  sym_prep_body(a, sp, sidx, npad);
+  if (blockIdx.x == gridDim.x - 1)  // the last block (fewest real agents) also cuts k_sym's work
+    compute_splits(fb_prev, G, sym_prefix(npad / qb, npad, qb), npad, qb, wd4, splits);
+  sym_prep_body(a, spf, cap, sidx, npad);
   span_end(a, SPAN_SLOT0 + 0);
 }
 
@@ -657,22 +784,24 @@ int sym_grid(int sms) {
 }
 
 template <int NT>
-cudaError_t sym_with(const StepArgs& a, float4* sp, int* sidx, const long long* fb_prev, long long* fb_cur, int sms,
-                     cudaStream_t s) {
+cudaError_t sym_with(const StepArgs& a, float4* sp, int* sidx, const long long* fb_prev, long long* fb_cur,
+                     long long* splits, int sms, cudaStream_t s) {
   constexpr int64_t QBS = NT * Q;
   const int64_t npad = (a.nloc + QBS - 1) / QBS * QBS;
-  BOIDS_PREFER_SMEM(k_sym_prep);
-  k_sym_prep<<<(unsigned)((npad + 255) / 256), 256, 0, s>>>(a, sp, sidx, npad);
-  if (cudaError_t e = cudaGetLastError()) return e;
   const int64_t nb = npad / QBS;
   const int64_t items = nb * npad - QBS * (nb * (nb - 1) / 2);
-  const int g = (int)std::min<int64_t>(sym_grid<NT>(sms), (items + CT - 1) / CT);
+  const int g = (int)std::min<int64_t>(std::min<int64_t>(sym_grid<NT>(sms), (items + CT - 1) / CT), SYM_FB_MAX_CTAS);
   static const int wd4 = [] {
     const char* e = getenv("BOIDS_SYM_WD4");  // diagnostics: diagonal item weight x4
     return e ? atoi(e) : 6;  // measured best of 4..16 at C3 and C4
   }();
-  return launch_pdl(k_sym<NT>, dim3(g), dim3(NT), sizeof(SymSmem<NT>), s, a, (const float4*)sp,
-                       (const int*)sidx, npad, wd4, fb_prev, g <= SYM_FB_MAX_CTAS ? fb_cur : nullptr);
+  BOIDS_PREFER_SMEM(k_sym_prep);
+  const int64_t cap = sym_capacity(a.nloc);  // sp holds 4 * cap floats: x[cap] | y[cap] | z[cap] | lim[cap]
+  float* spf = reinterpret_cast<float*>(sp);
+  k_sym_prep<<<(unsigned)((npad + 255) / 256), 256, 0, s>>>(a, spf, cap, sidx, npad, QBS, g, wd4, fb_prev, splits);
+  if (cudaError_t e = cudaGetLastError()) return e;
+  return launch_pdl(k_sym<NT>, dim3(g), dim3(NT), sizeof(SymSmem<NT>), s, a, (const float*)spf, cap,
+                    (const int*)sidx, npad, (const long long*)splits, fb_cur);
 }
 
 }  // namespace
@@ -695,7 +824,7 @@ cudaError_t launch_route(const StepArgs& a, cudaStream_t s) {
 }
 
 cudaError_t launch_sym_scan(const StepArgs& a, float4* sp, int* sidx, const long long* fb_prev, long long* fb_cur,
-                            cudaStream_t s) {
+                            long long* splits, cudaStream_t s) {
   if (a.nloc <= 0) return cudaSuccess;
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
@@ -707,9 +836,9 @@ cudaError_t launch_sym_scan(const StepArgs& a, float4* sp, int* sidx, const long
     const char* e = getenv("BOIDS_SYM_NT");  // diagnostics: force a CTA shape (128 or 512)
     return e ? atoi(e) : 0;
   }();
-  if (force == 256) return sym_with<256>(a, sp, sidx, fb_prev, fb_cur, sms, s);
-  if (force == 512 || (force != 128 && tiles512 >= 2LL * sms)) return sym_with<512>(a, sp, sidx, fb_prev, fb_cur, sms, s);
-  return sym_with<128>(a, sp, sidx, fb_prev, fb_cur, sms, s);
+  if (force == 256) return sym_with<256>(a, sp, sidx, fb_prev, fb_cur, splits, sms, s);
+  if (force == 512 || (force != 128 && tiles512 >= 2LL * sms)) return sym_with<512>(a, sp, sidx, fb_prev, fb_cur, splits, sms, s);
+  return sym_with<128>(a, sp, sidx, fb_prev, fb_cur, splits, sms, s);
 }
 
 }  // namespace boids
