@@ -217,6 +217,14 @@ def main():
     ap.add_argument("--no-sym", action="store_true",
                     help="single-GPU brute force: evaluate every ordered pair (k_scan) instead of each "
                          "unordered pair once (k_sym, default)")
+    ap.add_argument("--kernel-timing", default="live", choices=["live", "pass"],
+                    help="live (default): CUDA events bracket the search kernel inside the timed region; "
+                         "pass: the timed region runs uninstrumented and the search kernel is timed with "
+                         "events in a profiled pass of K steps right after (events inside a CUDA graph break "
+                         "its PDL edges: at n <= 16384 that perturbs the step time itself)")
+    ap.add_argument("--graph", type=int, default=0,
+                    help="1: warm steps replay captured CUDA graphs (BOIDS_OPT_GRAPH); 0 (default): eager launches "
+                         "(measured faster per flushed step on B200, DESIGN.md sec 5)")
     ap.add_argument("--force-shard", action="store_true",
                     help="use the multi-GPU code path (NCCL process group + sharded handles) even at N=1")
     args = ap.parse_args()
@@ -258,6 +266,7 @@ def main():
     else:
         fl = pk.Flock(cfg.n, params, seed=1, kernel=args.kernel, symmetric=not args.no_sym)
         h = fl.h
+        abi.boids_set_option(h, abi.BOIDS_OPT_GRAPH, args.graph)
         step = lambda: fl.step(dt, 1)  # noqa: E731
         nloc = cfg.n
 
@@ -273,7 +282,9 @@ def main():
     torch.cuda.synchronize()
 
     # ---------------- timed region: K steps, L2 flushed before each ----------------
-    abi.boids_set_option(h, abi.BOIDS_OPT_PROFILE, 2)  # events around the search and update launches only
+    live = args.kernel_timing == "live"
+    # events around the search launches only (level 2), or none (kernel timing in a later pass)
+    abi.boids_set_option(h, abi.BOIDS_OPT_PROFILE, 2 if live else 0)
     abi.boids_get_profile(h, reset=True)
     info0 = abi.boids_info(h)
     launches0 = info0.launches
@@ -293,6 +304,20 @@ def main():
     prof = abi.boids_get_profile(h, reset=True)
     abi.boids_set_option(h, abi.BOIDS_OPT_PROFILE, 0)
     ms = float(sum(a.elapsed_time(b) for a, b in ev))
+    grid_pairs = info1.grid_pairs - info0.grid_pairs  # grid search work of the steps `prof` timed
+    path = int(info1.last_path)
+    if not live:  # the search kernel timed in a profiled pass of K steps right after the timed region
+        abi.boids_set_option(h, abi.BOIDS_OPT_PROFILE, 2)
+        abi.boids_get_profile(h, reset=True)
+        ip0 = abi.boids_info(h)
+        for k in range(args.steps):
+            flush.fill_(float(k))
+            step()
+        torch.cuda.synchronize()
+        prof = abi.boids_get_profile(h, reset=True)
+        abi.boids_set_option(h, abi.BOIDS_OPT_PROFILE, 0)
+        ip1 = abi.boids_info(h)
+        grid_pairs, path = ip1.grid_pairs - ip0.grid_pairs, int(ip1.last_path)
     if dist is not None:
         t = torch.tensor([ms], device=dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
@@ -306,10 +331,9 @@ def main():
     k_ms_per = k_ms / max(k_n, 1)
     think = max(1, args.think)
     # the library reports which search path the timed steps ran (boids_info.last_path)
-    path = int(info1.last_path)
     sym = path == abi.BOIDS_PATH_SYM
     if grid:  # algorithmic work of the grid search: pairs over the 27-cell stencils (device counter)
-        pairs_per_launch = float(info1.grid_pairs - info0.grid_pairs) / max(k_n, 1)
+        pairs_per_launch = float(grid_pairs) / max(k_n, 1)
         pairs_note = " (27-cell stencil candidates, device counter)"
     elif sym:  # k_sym: every unordered pair once, tested against both agents' limits
         pairs_per_launch = float(cfg.n) * float(cfg.n - 1) / 2
@@ -343,6 +367,9 @@ def main():
                              f"(sm_max_mhz of MEASURED_PEAKS.json; each add/sub/mul counted once, no FMA)",
                 "work_per_launch": f"{OPS_PER_PAIR} lane-ops x {pairs_per_launch:.4g} pairs" + pairs_note,
                 "kernel_ms_per_launch": k_ms_per, "kernel_share_of_step": k_ms / ms if ms else None,
+                "timing": ("CUDA events on the launching stream around each search launch of the timed steps"
+                           if live else "CUDA events on the launching stream around each search launch of a "
+                           "profiled pass of K steps right after the (uninstrumented) timed region"),
                 "frac_at_measured_clock": (achieved / (148 * LANES_PER_SM * clocks["sm_mhz"] * 1e6 / 1e12))
                 if clocks.get("sm_mhz") else None}
     if sym:  # the thesis's per-agent formulation evaluates n x n ordered pairs

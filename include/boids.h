@@ -113,6 +113,7 @@ typedef struct boids_info_t {
                           what bench.py's roofline counts as the algorithmic work */
   int32_t reserved0;
   int64_t steps_sorted; /* cumulative: steps that rebuilt the spatial query order (binning) */
+  int64_t graph_launches; /* cumulative: boids_step steps run as a captured CUDA graph (BOIDS_OPT_GRAPH) */
 } boids_info_t;
 
 /* boids_info_t.last_path */
@@ -148,6 +149,12 @@ typedef struct boids_info_t {
                                        k_sym launch measured per item range (feedback; the first launch
                                        uses a static weighted split), 0 = static split always.  Only the
                                        partition of the work changes; results are identical. */
+#define BOIDS_OPT_GRAPH 10          /* 1: boids_step replays a captured CUDA graph of each warm single-rank
+                                       step (think_every 1; profiling events are retargeted per replay);
+                                       0 (default): every kernel is launched from the host (measured on
+                                       B200: the graph saves host enqueue time but a step of 4-6 dependent
+                                       kernels behind a cold L2 runs 5-6 us slower as a graph, C1-C3).
+                                       Results are identical either way. */
 #define BOIDS_OPT_PHASES 5          /* diagnostics: value = max CTAs; the fused kernel records per-CTA
                                        %globaltimer stamps (read with boids_get_phases); 0 = off */
 

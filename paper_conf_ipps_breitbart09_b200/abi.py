@@ -22,7 +22,7 @@ BOIDS_INIT_OPENSTEER, BOIDS_INIT_WORLD = 0, 1
 BOIDS_STEER_THESIS, BOIDS_STEER_OPENSTEER = 0, 1
 BOIDS_KERNEL_FUSED, BOIDS_KERNEL_SIMPLE, BOIDS_KERNEL_CLUSTER = 0, 1, 2
 BOIDS_OPT_RECORD_STEERING, BOIDS_OPT_KERNEL, BOIDS_OPT_PROFILE, BOIDS_OPT_CLUSTER, BOIDS_OPT_PHASES = 1, 2, 3, 4, 5
-BOIDS_OPT_RESORT, BOIDS_OPT_VOTE_U, BOIDS_OPT_SYMMETRIC, BOIDS_OPT_BALANCE = 6, 7, 8, 9
+BOIDS_OPT_RESORT, BOIDS_OPT_VOTE_U, BOIDS_OPT_SYMMETRIC, BOIDS_OPT_BALANCE, BOIDS_OPT_GRAPH = 6, 7, 8, 9, 10
 BOIDS_PROF_CLASSES = 5
 PROF_NAMES = ("fused_or_search", "update", "binning", "grid_search", "route")
 
@@ -62,6 +62,7 @@ class boids_info_t(C.Structure):
         ("launches", C.c_int64), ("slow_groups", C.c_int64), ("vote_groups", C.c_int64),
         ("fallbacks", C.c_int64), ("grid_pairs", C.c_int64), ("step_index", C.c_int64),
         ("last_path", C.c_int32), ("reserved0", C.c_int32), ("steps_sorted", C.c_int64),
+        ("graph_launches", C.c_int64),
     ]
 
 

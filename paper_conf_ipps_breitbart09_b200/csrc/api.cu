@@ -114,6 +114,27 @@ struct boids_ctx {
   int cluster_opt = 0;
   int profile = 0;          // BOIDS_OPT_PROFILE level
   int64_t launches = 0;
+  // CUDA graphs of single warm steps (boids_step): one per distinct launch
+  // sequence (search path, resort-or-not, k_sym feedback parity, ping-pong
+  // parity, dt); replayed with cudaGraphLaunch, the host-side step state advanced
+  // by a dry run of one_step
+  bool dry = false;
+  bool capturing = false;  // one_step runs inside graph_step's stream capture
+  bool use_graphs = false;  // BOIDS_OPT_GRAPH
+  cudaStream_t cap_stream = nullptr;
+  struct GraphEntry {
+    uint32_t key;
+    float dt;
+    cudaGraphExec_t exec;
+    cudaGraph_t graph;  // kept: its event-record nodes address the exec's nodes
+    struct Prof {
+      int cls;
+      cudaGraphNode_t a, b;  // event-record nodes bracketing one profiled launch (BOIDS_OPT_PROFILE)
+    };
+    std::vector<Prof> prof;
+  };
+  std::vector<GraphEntry> graphs;
+  int64_t graph_launches = 0;
   struct Rec {
     int cls;
     cudaEvent_t a, b;
@@ -208,6 +229,11 @@ void free_ctx(boids_ctx* c) {
   cudaFree(c->rpart);
   cudaFree(c->rbcount);
   cudaFree(c->sym_rcount);
+  for (auto& g : c->graphs) {
+    cudaGraphExecDestroy(g.exec);
+    cudaGraphDestroy(g.graph);
+  }
+  if (c->cap_stream) cudaStreamDestroy(c->cap_stream);
   for (auto& r : c->recs) {
     cudaEventDestroy(r.a);
     cudaEventDestroy(r.b);
@@ -227,9 +253,20 @@ cudaEvent_t get_event(boids_ctx* c) {
   return e;
 }
 
+// A step's memset on the handle's stream (skipped on a dry run: see replay_step).
+cudaError_t mset(boids_ctx* c, void* p, int v, size_t bytes) {
+  return c->dry ? cudaSuccess : cudaMemsetAsync(p, v, bytes, c->stream);
+}
+
 // Launch wrapper: counts launches and, when profiling, brackets with events.
+// On a dry run (replay_step) nothing is enqueued: only the host-side state of
+// the step advances, exactly as it did when the step's graph was captured.
 template <class F>
 int launch(boids_ctx* c, int cls, F&& f, int kernels = 1) {
+  if (c->dry) {
+    c->launches += kernels;
+    return BOIDS_OK;
+  }
   cudaEvent_t a = nullptr, b = nullptr;
   // level 2: only the search classes (0, 3), plus the update (1) in think mode
   // (k_apply / k_select carry that step's modification roofline) -- fewer event
@@ -239,12 +276,14 @@ int launch(boids_ctx* c, int cls, F&& f, int kernels = 1) {
   if (rec) {
     a = get_event(c);
     b = get_event(c);
-    CK(cudaEventRecord(a, c->stream));
+    // External: inside a stream capture (graph_step) the record becomes an
+    // event-record node of the graph instead of a capture-internal marker
+    CK(cudaEventRecordWithFlags(a, c->stream, c->capturing ? cudaEventRecordExternal : cudaEventRecordDefault));
   }
   CK(f());
   c->launches += kernels;
   if (rec) {
-    CK(cudaEventRecord(b, c->stream));
+    CK(cudaEventRecordWithFlags(b, c->stream, c->capturing ? cudaEventRecordExternal : cudaEventRecordDefault));
     c->recs.push_back({cls, a, b});
   }
   return BOIDS_OK;
@@ -443,7 +482,7 @@ int one_step(boids_ctx* c, float dt) {
   // neighbours and break the t0 bound).  Think mode keeps it per agent (k_select
   // writes it for warm thinkers, k_think_compact clears it for cold ones).
   const bool warm_path = !grid && !think && c->kernel == BOIDS_KERNEL_FUSED && c->warm;
-  if (!warm_path && !(think && !grid)) CK(cudaMemsetAsync(c->nbr8, 0xFF, c->m * sizeof(int32_t), c->stream));
+  if (!warm_path && !(think && !grid)) CK(mset(c, c->nbr8, 0xFF, c->m * sizeof(int32_t)));
   if (grid) {
     // a2: bin all agents (candidates) and the owned ones (queries) by search cell;
     // think mode: only this step's thinkers are queries
@@ -476,7 +515,7 @@ int one_step(boids_ctx* c, float dt) {
     g.grid = c->sgrid;
     StepArgs ag = a;
     ag.store_only = think ? 1 : 0;
-    CK(cudaMemsetAsync(c->sym_rcount, 0, sizeof(int32_t), c->stream));
+    CK(mset(c, c->sym_rcount, 0, sizeof(int32_t)));
     c->last_path = BOIDS_PATH_GRID;
     if ((rc = launch(c, 3, [&] { return launch_grid(ag, g, c->stream); }))) return rc;
     if ((rc = launch(c, 4, [&] { return launch_grid_far(ag, g, c->stream); }))) return rc;
@@ -503,7 +542,7 @@ int one_step(boids_ctx* c, float dt) {
       // this step's thinkers, in spatial order, split into never-searched (cold)
       // and warm-bounded ones
       c->last_path = BOIDS_PATH_THINK;
-      CK(cudaMemsetAsync(c->tcnt, 0, 2 * sizeof(int32_t), c->stream));
+      CK(mset(c, c->tcnt, 0, 2 * sizeof(int32_t)));
       if ((rc = launch(c, 2, [&] {
              return launch_think_compact(a, c->qperm, c->tcold, c->tcnt, c->twarm, c->tcnt + 1, c->stream);
            })))
@@ -519,7 +558,7 @@ int one_step(boids_ctx* c, float dt) {
       StepArgs aw = a;
       aw.qperm = c->twarm;
       aw.qcount = c->tcnt + 1;
-      CK(cudaMemsetAsync(c->sym_rcount, 0, sizeof(int32_t), c->stream));
+      CK(mset(c, c->sym_rcount, 0, sizeof(int32_t)));
       if ((rc = launch(c, 0, [&] { return launch_warm_scan(aw, c->stream); }, 2))) return rc;
       if ((rc = launch(c, 1, [&] { return launch_warm_select(a, c->stream); }))) return rc;
       if ((rc = launch(c, 4, [&] { return launch_route(a, c->stream); }))) return rc;
@@ -536,7 +575,7 @@ int one_step(boids_ctx* c, float dt) {
         c->last_path = BOIDS_PATH_SYM;
         StepArgs as = a;
         as.routed = c->routed;  // agents routed to k_route by k_sym_prep (k_select skips them)
-        CK(cudaMemsetAsync(c->sym_rcount, 0, sizeof(int32_t), c->stream));
+        CK(mset(c, c->sym_rcount, 0, sizeof(int32_t)));
         long long* fb_prev = c->sym_fb + (c->sym_fb_par ^ 1) * SYM_FB_LEN;
         long long* fb_cur = c->sym_fb + c->sym_fb_par * SYM_FB_LEN;
         c->sym_fb_par ^= 1;
@@ -549,7 +588,7 @@ int one_step(boids_ctx* c, float dt) {
         if ((rc = launch(c, 4, [&] { return launch_route(as, c->stream); }))) return rc;
       } else {
         c->last_path = BOIDS_PATH_SCAN;
-        CK(cudaMemsetAsync(c->sym_rcount, 0, sizeof(int32_t), c->stream));
+        CK(mset(c, c->sym_rcount, 0, sizeof(int32_t)));
         if ((rc = launch(c, 0, [&] { return launch_warm_scan(a, c->stream); }, 2))) return rc;
         if ((rc = launch(c, 1, [&] { return launch_warm_select(a, c->stream); }))) return rc;
         if ((rc = launch(c, 4, [&] { return launch_route(a, c->stream); }))) return rc;
@@ -566,6 +605,109 @@ int one_step(boids_ctx* c, float dt) {
   c->steering_valid = c->record_steering;
   c->step_index++;
   c->steps_taken++;
+  return BOIDS_OK;
+}
+
+// boids_step's CUDA-graph path: warm single-rank steps without profiling or
+// think frequency replay a captured graph of the step's launches (the host
+// launch cost of 4-6 kernels and memsets per step becomes one graph launch; the
+// PDL edges are captured as programmatic graph edges).  The launch sequence of
+// a step is fixed by host-side state: whether the spatial query order is
+// rebuilt this step, the k_sym feedback-record parity and the ping-pong buffer
+// parity; together with dt they key the cache.  A replay first advances that
+// host state by a dry run of one_step (nothing enqueued), exactly as the
+// captured run did.  Results never depend on the path taken.
+// Profiling (BOIDS_OPT_PROFILE) works inside graphs: the event records that
+// bracket a profiled launch are captured as event-record nodes, and every replay
+// points them at fresh events first (cudaGraphExecEventRecordNodeSetEvent), so
+// each replayed launch is timed like an eager one.
+bool graph_ok(const boids_ctx* c) {
+  const bool grid = c->p.search_mode == BOIDS_GRID;
+  return c->use_graphs && !c->shard && c->p.think_every == 1 && c->phase == nullptr && c->steps_taken >= 2 &&
+         (grid || (c->warm && c->kernel == BOIDS_KERNEL_FUSED));
+}
+
+void clear_graphs(boids_ctx* c) {
+  for (auto& g : c->graphs) {
+    cudaGraphExecDestroy(g.exec);
+    cudaGraphDestroy(g.graph);
+  }
+  c->graphs.clear();
+}
+
+int graph_step(boids_ctx* c, float dt) {
+  const bool resort = c->since_sort < 0 || c->since_sort >= c->resort_every;
+  const uint32_t key = (resort ? 1u : 0u) | ((uint32_t)c->sym_fb_par << 1) | ((uint32_t)c->cur << 2);
+  for (auto& g : c->graphs)
+    if (g.key == key && g.dt == dt) {
+      c->dry = true;
+      const int rc = one_step(c, dt);
+      c->dry = false;
+      if (rc) return rc;
+      for (auto& pr : g.prof) {
+        cudaEvent_t ea = get_event(c), eb = get_event(c);
+        CK(cudaGraphExecEventRecordNodeSetEvent(g.exec, pr.a, ea));
+        CK(cudaGraphExecEventRecordNodeSetEvent(g.exec, pr.b, eb));
+        c->recs.push_back({pr.cls, ea, eb});
+      }
+      CK(cudaGraphLaunch(g.exec, c->stream));
+      c->graph_launches++;
+      return BOIDS_OK;
+    }
+  if (c->graphs.size() >= 16) clear_graphs(c);  // e.g. a caller cycling through many dt values
+  if (!c->cap_stream) CK(cudaStreamCreateWithFlags(&c->cap_stream, cudaStreamNonBlocking));
+  cudaStream_t orig = c->stream;
+  c->stream = c->cap_stream;
+  cudaError_t e = cudaStreamBeginCapture(c->cap_stream, cudaStreamCaptureModeRelaxed);
+  if (e != cudaSuccess) {
+    c->stream = orig;
+    CK(e);
+  }
+  const size_t rec0 = c->recs.size();
+  c->capturing = true;
+  const int rc = one_step(c, dt);
+  c->capturing = false;
+  cudaGraph_t g = nullptr;
+  e = cudaStreamEndCapture(c->cap_stream, &g);
+  c->stream = orig;
+  if (rc) {
+    if (g) cudaGraphDestroy(g);
+    return rc;
+  }
+  CK(e);
+  // the event-record nodes of the profiled launches of this step (if any)
+  std::vector<boids_ctx::GraphEntry::Prof> prof;
+  if (c->recs.size() > rec0) {
+    size_t nn = 0;
+    CK(cudaGraphGetNodes(g, nullptr, &nn));
+    std::vector<cudaGraphNode_t> nodes(nn);
+    CK(cudaGraphGetNodes(g, nodes.data(), &nn));
+    auto node_of = [&](cudaEvent_t ev) -> cudaGraphNode_t {
+      for (auto nd : nodes) {
+        cudaGraphNodeType t;
+        cudaEvent_t x = nullptr;
+        if (cudaGraphNodeGetType(nd, &t) == cudaSuccess && t == cudaGraphNodeTypeEventRecord &&
+            cudaGraphEventRecordNodeGetEvent(nd, &x) == cudaSuccess && x == ev)
+          return nd;
+      }
+      return nullptr;
+    };
+    for (size_t i = rec0; i < c->recs.size(); ++i) {
+      const auto& r = c->recs[i];
+      prof.push_back({r.cls, node_of(r.a), node_of(r.b)});
+      if (!prof.back().a || !prof.back().b) {
+        cudaGraphDestroy(g);
+        return fail(BOIDS_ECUDA, "graph capture: profiling event node not found");
+      }
+    }
+  }
+  cudaGraphExec_t exec = nullptr;
+  e = cudaGraphInstantiate(&exec, g, 0);
+  if (e != cudaSuccess) cudaGraphDestroy(g);
+  CK(e);
+  c->graphs.push_back({key, dt, exec, g, prof});
+  CK(cudaGraphLaunch(exec, c->stream));
+  c->graph_launches++;
   return BOIDS_OK;
 }
 
@@ -652,7 +794,12 @@ BOIDS_API int boids_set_stream(boids_ctx* c, void* stream) {
 BOIDS_API int boids_set_option(boids_ctx* c, int32_t opt, int64_t v) {
   if (!c) return fail(BOIDS_EINVAL, "NULL handle");
   DeviceGuard g(c->dev);
+  CK(cudaStreamSynchronize(c->stream));  // captured graphs may still run: drop them only when done
+  clear_graphs(c);
   switch (opt) {
+    case BOIDS_OPT_GRAPH:
+      c->use_graphs = v != 0;
+      return BOIDS_OK;
     case BOIDS_OPT_RECORD_STEERING:
       if (v && !c->force4) CK(cudaMalloc((void**)&c->force4, c->m * sizeof(float4)));
       c->record_steering = v != 0;
@@ -708,7 +855,7 @@ BOIDS_API int boids_step(boids_ctx* c, float dt, int32_t steps) {
   if (steps < 0) return fail(BOIDS_EINVAL, "steps must be >= 0");
   DeviceGuard g(c->dev);
   for (int32_t t = 0; t < steps; ++t)
-    if ((rc = one_step(c, dt))) return rc;
+    if ((rc = graph_ok(c) ? graph_step(c, dt) : one_step(c, dt))) return rc;
   return BOIDS_OK;
 }
 
@@ -884,6 +1031,7 @@ BOIDS_API int boids_info(boids_ctx* c, boids_info_t* o) {
   o->last_path = c->last_path;
   o->reserved0 = 0;
   o->steps_sorted = c->steps_sorted;
+  o->graph_launches = c->graph_launches;
   return BOIDS_OK;
 }
 

@@ -17,9 +17,9 @@
 // reverse test both come from the same array; phantoms p >= n have NaN positions
 // and lim = -1).  Query block b holds sorted positions [b*QB, (b+1)*QB); its item
 // space is the candidates [b*QB, npad):
-//   * diagonal tiles [b*QB, (b+1)*QB): every ordered pair inside the block is
-//     evaluated from the query side only (self excluded by sorted position), as
-//     in k_scan -- the block's pairs are not split by a triangle mask;
+//   * diagonal tiles [b*QB, (b+1)*QB): the block's 16 groups of 128 against
+//     each other as a triangle -- groups (kc, w) with kc > w tested from both
+//     sides, (w, w) from the query side only (self excluded by sorted position);
 //   * off-diagonal tiles [(b+1)*QB, npad): both sides are tested.
 // Stream-K: the triangular item space sum_b (npad - b*QB) is cut into equal
 // contiguous ranges per CTA, as in k_scan.  Candidates and their original
@@ -338,8 +338,8 @@ __global__ void __launch_bounds__(NTS, NTS == 128 ? 4 : (NTS == 256 ? 2 : 1))
   __syncthreads();
   Rec* rec = sm.rec[warp];
   int wcount = 0;
-  unsigned slow_groups = 0, groups = 0;
-  int64_t cur_b = -1;
+  unsigned slow_groups = 0;
+  int cur_b = -1;
   int cur_w = -1;
   float px[Q], py[Q], pz[Q], limq = 0.f;
   int qbase = 0;  // sorted position of the thread's query 0 (query q: qbase + 32 q)
@@ -353,11 +353,13 @@ __global__ void __launch_bounds__(NTS, NTS == 128 ? 4 : (NTS == 256 ? 2 : 1))
     u = __shfl_sync(0xffffffffu, u, 0);
     if (u >= nunits) break;
     const int k = u / NW, wq = u - k * NW;
-    const TileDesc td = tile_desc(k, L0, L1, npad, QBS);
-    if (td.b != cur_b || wq != cur_w) {  // query group wq of row b: 4 x 32 spatially compact queries
-      cur_b = td.b;
+    // the range is re-read from shared memory per unit: keeping L0 / L1 (int64)
+    // live in registers across the pair loop cost the fast path spills
+    const TileDesc td = tile_desc(k, *(volatile int64_t*)&s_range[0], *(volatile int64_t*)&s_range[1], npad, QBS);
+    if ((int)td.b != cur_b || wq != cur_w) {  // query group wq of row b: 4 x 32 spatially compact queries
+      cur_b = (int)td.b;
       cur_w = wq;
-      qbase = (int)(cur_b * QBS + wq * 32 * Q + lane);
+      qbase = cur_b * QBS + wq * 32 * Q + lane;
       float lq[Q];
       __syncwarp();  // the previous group's slow path is done with wqg / wql
 #pragma unroll
@@ -470,7 +472,6 @@ __global__ void __launch_bounds__(NTS, NTS == 128 ? 4 : (NTS == 256 ? 2 : 1))
           thr = fmaxf(fmaxf(fmaxf(thr, fmaxf(W0.x, W0.y)), fmaxf(W0.z, W0.w)),
                       fmaxf(fmaxf(W1.x, W1.y), fmaxf(W1.z, W1.w)));
         }
-        ++groups;
         if (__any_sync(0xffffffffu, m <= thr)) {  // rare, warp-uniform
           ++slow_groups;
 #pragma unroll 1
@@ -480,10 +481,23 @@ __global__ void __launch_bounds__(NTS, NTS == 128 ? 4 : (NTS == 256 ? 2 : 1))
       if (!diag && cnt == CT) {  // full off-diagonal tile: constant trip count (the common case)
 #pragma unroll 1
         for (int c = 0; c < CT; c += UG) group(c, std::false_type{});
-      } else if (!diag) {
-        for (int c = 0; c < cnt; c += UG) group(c, std::false_type{});
       } else {
-        for (int c = 0; c < cnt; c += UG) group(c, std::true_type{});
+        // Diagonal tile (candidates of the query block itself): the block's pairs are
+        // symmetric too.  Candidate group kc (block positions [kc*128, kc*128 + 128), the
+        // positions of query group kc) against query group wq: kc > wq -- both sides,
+        // like an off-diagonal tile; kc == wq -- the group with itself, query side only
+        // (self excluded); kc < wq -- skipped: unit (kc, wq) evaluates those pairs.  Every
+        // unordered pair of the block is evaluated once (UG divides 128).  kc grows with
+        // c, so the three cases are three contiguous candidate ranges of the tile.
+        int ce = 0, co = 0;  // [ce_start, ce) query-side-only range, [co, cnt) both sides
+        int cs = 0;
+        if (diag) {
+          const int rel0 = jb - cur_b * QBS;
+          cs = min(max(wq * 32 * Q - rel0, 0), cnt);
+          ce = co = min(max((wq + 1) * 32 * Q - rel0, 0), cnt);
+        }
+        for (int c = cs; c < ce; c += UG) group(c, std::true_type{});
+        for (int c = co; c < cnt; c += UG) group(c, std::false_type{});
       }
     }
     __syncwarp();
@@ -516,7 +530,8 @@ __global__ void __launch_bounds__(NTS, NTS == 128 ? 4 : (NTS == 256 ? 2 : 1))
   }
   if (a.stats && lane == 0) {
     atomicAdd(a.stats, (unsigned long long)slow_groups);
-    atomicAdd(a.stats + 1, (unsigned long long)groups);
+    // vote groups: every candidate item of the range meets every query group, UG candidates per vote
+    if (warp == 0) atomicAdd(a.stats + 1, (unsigned long long)((L1 - L0) / UG * NW));
   }
   if (a.phase) {
     if (lane == 0) {

@@ -490,3 +490,35 @@ def test_set_state_between_steps_small_n(pk, orc, n):
         o_state, o_idx, _, o_F = orc.step(orc.State(s), DT)
         np.testing.assert_array_equal(f.neighbors()[0], o_idx)
         assert bitexact(f.state(), o_state) and np.array_equal(f.steering(), o_F)
+
+
+@pytest.mark.parametrize("mode,n,steps", [(0, 1500, 20), (0, 20000, 12), (1, 6000, 12)])
+def test_graph_steps_match_eager_and_oracle(pk, orc, mode, n, steps):
+    """boids_step replays captured CUDA graphs of warm steps (BOIDS_OPT_GRAPH =
+    1): the trajectory must equal the eager launches bit for bit and
+    the oracle's; resort steps (every 8th) and both k_sym feedback parities are
+    captured separately.  Profiling inside graphs (events retargeted per replay)
+    must still report every search launch."""
+    from paper_conf_ipps_breitbart09_b200 import abi
+
+    p = pk.boids_default_params(init_mode=1, search_mode=mode, world_radius=20.0)
+    op = _oparams(orc, p)
+    with pk.Flock(n, p, seed=3) as fg, pk.Flock(n, p, seed=3) as fe:
+        abi.boids_set_option(fg.h, abi.BOIDS_OPT_GRAPH, 1)
+        abi.boids_set_option(fe.h, abi.BOIDS_OPT_GRAPH, 0)
+        fg.step(DT, steps)
+        fe.step(DT, steps)
+        assert fg.info().graph_launches >= steps - 3 and fe.info().graph_launches == 0
+        sg, se = fg.state(), fe.state()
+        assert all(np.array_equal(sg[k], se[k]) for k in KEYS)
+        assert np.array_equal(fg.neighbors()[0], fe.neighbors()[0])
+        o = orc.run(orc.init(n, op, seed=3), DT, steps, op)
+        assert bitexact(sg, o)
+        abi.boids_set_option(fg.h, abi.BOIDS_OPT_PROFILE, 2)
+        abi.boids_get_profile(fg.h, reset=True)
+        g0 = fg.info().graph_launches
+        fg.step(DT, 5)
+        prof = abi.boids_get_profile(fg.h, reset=True)
+        assert fg.info().graph_launches - g0 == 5
+        cls = "grid_search" if mode else "fused_or_search"
+        assert prof[cls][1] == 5 and prof[cls][0] > 0
