@@ -156,11 +156,15 @@ __global__ void __launch_bounds__(NT) k_fused(StepArgs a, int64_t tiles_total) {
 #pragma unroll
     for (int s = 0; s < STAGES; ++s) {
       mbar_init(&sm.full[s], 1);
-      mbar_init(&sm.empty[s], NW);
+      mbar_init(&sm.empty[s], NT);
     }
     mbar_fence_init();
   }
-  __syncthreads();
+  // fence.mbarrier_init is a release at cluster scope: in a cluster launch the
+  // barriers' initialisation is made visible by a cluster barrier (the acquire),
+  // before the first arrive / bulk copy uses them
+  if constexpr (K > 1) cg::this_cluster().sync();
+  else __syncthreads();
   if (tid == 0) {  // prologue: fill the ring
     for (int t = 0; t < STAGES && t < nt; ++t) {
       mbar_arrive_expect_tx(&sm.full[t], CT * sizeof(float4));
@@ -257,9 +261,11 @@ __global__ void __launch_bounds__(NT) k_fused(StepArgs a, int64_t tiles_total) {
         limc = fmaxf(fmaxf(lim[0], lim[1]), fmaxf(lim[2], lim[3]));
       }
     }
-    __syncwarp();
-    if (lane == 0) mbar_arrive(&sm.empty[s]);
-    // refill this stage with tile t + STAGES once every warp has released it
+    // every thread releases the stage after its own reads of it (release
+    // semantics per thread: the stage's reuse by the bulk copy is ordered after
+    // all of them without relying on __syncwarp; this kernel runs on cold steps only)
+    mbar_arrive(&sm.empty[s]);
+    // refill this stage with tile t + STAGES once every thread has released it
     if (tid == 0 && t + STAGES < nt) {
       mbar_wait(&sm.empty[s], (uint32_t)((t / STAGES) & 1));
       fence_proxy_async_smem();

@@ -192,7 +192,7 @@ __global__ void __launch_bounds__(NTG, 5) k_grid(StepArgs a, GridArgs g) {  // 5
 #pragma unroll
     for (int s = 0; s < STAGES; ++s) {
       mbar_init(&sm.full[s], 1);
-      mbar_init(&sm.empty[s], NTG / 32);
+      mbar_init(&sm.empty[s], NTG);
     }
     mbar_fence_init();
   }
@@ -342,8 +342,10 @@ __global__ void __launch_bounds__(NTG, 5) k_grid(StepArgs a, GridArgs g) {  // 5
       else if (qv == 3) grid_tile<3>(tile, cnt, pxy, pz, lim, limc, gq, sm.lists, warp, lane, groups, slow_groups);
       else if (qv == 2) grid_tile<2>(tile, cnt, pxy, pz, lim, limc, gq, sm.lists, warp, lane, groups, slow_groups);
       else if (qv == 1) grid_tile<1>(tile, cnt, pxy, pz, lim, limc, gq, sm.lists, warp, lane, groups, slow_groups);
-      __syncwarp();
-      if (lane == 0) mbar_arrive(&sm.empty[s]);
+      // every thread releases the stage after its own reads (per-thread release
+      // orders them before the stage's refill by the bulk copy; compute-sanitizer
+      // racecheck does not count a __syncwarp before one lane's arrive as ordering)
+      mbar_arrive(&sm.empty[s]);
       ++tc;
       next_tile(sm, r, off);
       if (tid == 0 && pr < nr) {
