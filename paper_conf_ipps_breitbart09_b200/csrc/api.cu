@@ -85,6 +85,7 @@ struct boids_ctx {
   unsigned long long* phase = nullptr;  // diagnostics (BOIDS_OPT_PHASES): per-CTA timestamps
   // grid mode (BOIDS_GRID): search grid and its binning buffers
   BinGrid sgrid{};
+  BinGrid qgrid{};  // blocks of sgrid: the queries' binning and the grid search's work items
   int2* gcellrank = nullptr;
   int32_t *gcnt = nullptr, *gstart = nullptr, *gqstart = nullptr, *counter = nullptr;
   int4* gitems = nullptr;      // grid search work items (k_bin_scan)
@@ -352,6 +353,7 @@ int create_impl(int64_t n, const boids_params* p, uint64_t seed, int32_t rank, i
   }
   if (p->search_mode == BOIDS_GRID) {
     c->sgrid = make_search_grid(*p);
+    c->qgrid = make_query_grid(c->sgrid);
     const int C = c->sgrid.cells;
     if ((rc = alloc((void**)&c->gcellrank, slots * sizeof(int2))) ||
         (rc = alloc((void**)&c->gcnt, C * sizeof(int32_t))) ||
@@ -486,26 +488,26 @@ int one_step(boids_ctx* c, float dt) {
   if (grid) {
     // a2: bin all agents (candidates) and the owned ones (queries) by search cell;
     // think mode: only this step's thinkers are queries
-    const bool one = (!c->shard || c->world == 1) && !think;
+    // candidates: every agent by fine search cell (spos, gstart); queries: the
+    // owned agents (this step's thinkers in think mode) by block of cells
+    // (qperm, gqstart) and the work items over the blocks
     const int64_t slots = c->shard ? (int64_t)c->world * c->m : c->m;
     const int chunk = grid_chunk();
     if ((rc = launch(c, 2, [&] {
            cudaError_t e = launch_bin(a.full, c->m, a.sdiv, 0, slots, c->sgrid, c->gcellrank, c->gcnt, c->gstart,
-                                      c->spos, one ? c->qperm : nullptr, 0, c->stream, nullptr,
-                                      one ? c->gitems : nullptr, one ? c->gnitems : nullptr, chunk,
-                                      one ? c->counter : nullptr, 1, 0, c->growbuf);
-           if (e == cudaSuccess && !one)
-             e = launch_bin(a.full, c->m, a.sdiv, c->lo, c->nloc, c->sgrid, c->gcellrank, c->gcnt, c->gqstart,
+                                      c->spos, nullptr, 0, c->stream, nullptr, nullptr, nullptr, chunk, nullptr, 1,
+                                      0, c->growbuf);
+           if (e == cudaSuccess)
+             e = launch_bin(a.full, c->m, a.sdiv, c->lo, c->nloc, c->qgrid, c->gcellrank, c->gcnt, c->gqstart,
                             nullptr, c->qperm, (int)c->lo, c->stream, nullptr, c->gitems, c->gnitems, chunk,
-                            c->counter,
-                            c->p.think_every, c->step_index, c->growbuf);
+                            c->counter, c->p.think_every, c->step_index, c->growbuf);
            return e;
-         }, one ? 3 : 6)))
+         }, 6)))
       return rc;
     GridArgs g;
     g.spos = c->spos;
     g.cstart = c->gstart;
-    g.qstart = one ? c->gstart : c->gqstart;
+    g.qstart = c->gqstart;
     g.qperm = c->qperm;
     g.items = c->gitems;
     g.nitems = c->gnitems;
@@ -513,6 +515,7 @@ int one_step(boids_ctx* c, float dt) {
     g.fcount = c->sym_rcount;
     g.counter = c->counter;
     g.grid = c->sgrid;
+    g.qgrid = c->qgrid;
     StepArgs ag = a;
     ag.store_only = think ? 1 : 0;
     CK(mset(c, c->sym_rcount, 0, sizeof(int32_t)));

@@ -21,7 +21,18 @@ __device__ __forceinline__ int cell_coord(float v, const BinGrid& g, int d) {
   return c < 0 ? 0 : (c >= g.dim[d] ? g.dim[d] - 1 : c);
 }
 
+__device__ __forceinline__ int fine_coord(float v, const BinGrid& g, int d) {
+  float t = (v - g.lo[d]) * g.inv_h;
+  int c = (int)floorf(t);
+  return c < 0 ? 0 : (c >= g.fdim ? g.fdim - 1 : c);
+}
+
 __device__ __forceinline__ int cell_of(float4 p, const BinGrid& g) {
+  if (g.block > 0) {  // block of the fine cell (exactly the fine cell's own coordinates / block)
+    const int bx = fine_coord(p.x, g, 0) / g.block, by = fine_coord(p.y, g, 1) / g.block,
+              bz = fine_coord(p.z, g, 2) / g.block;
+    return (bz * g.dim[1] + by) * g.dim[0] + bx;
+  }
   int ix = cell_coord(p.x, g, 0), iy = cell_coord(p.y, g, 1), iz = cell_coord(p.z, g, 2);
   if (g.morton) return (int)(spread3(ix) | (spread3(iy) << 1) | (spread3(iz) << 2));
   return (iz * g.dim[1] + iy) * g.dim[0] + ix;

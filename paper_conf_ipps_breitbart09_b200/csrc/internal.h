@@ -64,6 +64,10 @@ struct BinGrid {
   int cells;
   int morton;  // 1: cell id = Morton code (dim must be a power of two), 0: row-major
   int reach;   // search grid: cells per axis an agent closer than r can be away (h * reach >= r)
+  int block;   // > 0: a grid of BLOCKS of block^3 cells of the fine grid (lo, h, fdim): the block of a
+               // position is its fine cell coordinate / block (so it agrees with the fine cell exactly);
+               // dim[] then counts blocks per axis
+  int fdim;    // fine cells per axis (block > 0)
 };
 
 struct StepArgs {
@@ -127,7 +131,8 @@ struct GridArgs {
   int* counter;           // work-queue counter (reset by the binning scan)
   int* flist;             // queries routed to k_grid_far (limit beyond the adjacent cells)
   int* fcount;            // their number (zeroed before k_grid)
-  BinGrid grid;
+  BinGrid grid;           // the fine search grid of the candidates (cstart)
+  BinGrid qgrid;          // its blocks: the queries' binning (qstart, items; item.z = block index)
 };
 
 // Does global agent g think at step t (think frequency k)?
@@ -191,6 +196,7 @@ cudaError_t launch_bin(const float4* full, int64_t m, const SliceDiv& sd, int64_
                        int* rowbuf = nullptr);  // [2 * rows] scratch: large grids scan on many CTAs
 BinGrid make_locality_grid(int64_t n, const boids_params& p);
 BinGrid make_search_grid(const boids_params& p);
+BinGrid make_query_grid(const BinGrid& search);  // blocks of the search grid: the grid search's work items
 cudaError_t launch_fill_nan(float4* p, int64_t count, cudaStream_t s);
 cudaError_t launch_apply(const StepArgs& a, cudaStream_t s);
 cudaError_t launch_pack_draw(const float4* local, int64_t m, const float4* up4, const float4* side4, int64_t k,

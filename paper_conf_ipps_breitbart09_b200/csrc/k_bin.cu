@@ -300,25 +300,28 @@ cudaError_t launch_bin(const float4* full, int64_t m, const SliceDiv& sd, int64_
   const int rows = g.cells / g.dim[0];
   // think mode: items hold only this step's thinkers (1/k of the agents); longer
   // runs stream more candidates per query but amortise each item's fixed cost
-  const int span = think_k > 1 ? THINK_SPAN : MAX_SPAN;
+  const int span = g.block > 0 ? (think_k > 1 ? 4 : 2) : (think_k > 1 ? THINK_SPAN : MAX_SPAN);
   const size_t shm = (size_t)(g.cells + g.cells / 32 + 1 + (items ? rows + rows / 32 + 1 : 0)) * sizeof(int);
-  if (shm > 48 * 1024) {
+  const int D = g.dim[0];
+  // large grids scan on many CTAs (one warp per row); small ones in one CTA's shared memory
+  const bool many = rowbuf && g.cells > 16384 && D <= RW_MAXD && g.cells % D == 0;
+  if (!many && shm > 48 * 1024) {
     cudaError_t e = cudaFuncSetAttribute(k_bin_scan, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)shm);
     if (e != cudaSuccess) return e;
   }
-  if (count <= 0) {  // still publish an empty binning (starts, items, counter)
+  if (count <= 0 && !many) {  // still publish an empty binning (starts, items, counter)
     k_bin_scan<<<1, SCAN_T, shm, s>>>(cnt, start, g.cells, items, nitems, chunk, counter, g.dim[0], span);
     return cudaGetLastError();
   }
   BOIDS_PREFER_SMEM(k_bin_count);
   BOIDS_PREFER_SMEM(k_bin_scatter);
   BOIDS_PREFER_SMEM(k_bin_scan);
-  k_bin_count<<<blocks, 256, 0, s>>>(full, m, sd, j0, count, g, cellrank, cnt, spos == nullptr,
-                                     spos == nullptr ? think_k : 1, think_t);
+  if (count > 0)
+    k_bin_count<<<blocks, 256, 0, s>>>(full, m, sd, j0, count, g, cellrank, cnt, spos == nullptr,
+                                       spos == nullptr ? think_k : 1, think_t);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return e;
-  const int D = g.dim[0];
-  if (rowbuf && g.cells > 16384 && D <= RW_MAXD && g.cells % D == 0) {  // large grid: many CTAs
+  if (many) {  // large grid: many CTAs
     const unsigned rb = (unsigned)((rows + RW_WARPS - 1) / RW_WARPS);
     int* rowsum = rowbuf;
     int* rowit = items ? rowbuf + rows : nullptr;
@@ -337,7 +340,7 @@ cudaError_t launch_bin(const float4* full, int64_t m, const SliceDiv& sd, int64_
     k_bin_scan<<<1, SCAN_T, shm, s>>>(cnt, start, g.cells, items, nitems, chunk, counter, g.dim[0], span);
     if ((e = cudaGetLastError()) != cudaSuccess) return e;
   }
-  k_bin_scatter<<<blocks, 256, 0, s>>>(full, m, sd, j0, count, cellrank, start, spos, perm, perm_base);
+  if (count > 0) k_bin_scatter<<<blocks, 256, 0, s>>>(full, m, sd, j0, count, cellrank, start, spos, perm, perm_base);
   if (launches) *launches += 3;
   return cudaGetLastError();
 }
@@ -345,22 +348,23 @@ cudaError_t launch_bin(const float4* full, int64_t m, const SliceDiv& sd, int64_
 // Search grid of BOIDS_GRID: row-major over the world box [-B, B]^3, B = max(world,
 // init radius) * 1.02; agents outside are clamped into boundary cells (clamping
 // is monotone and 1-Lipschitz on cell coordinates, so it never separates a pair
-// by more cells than the distance allows).  Cells are SMALLER than r: h =
-// r (1 + 2^-10) / 3, so an agent closer than r lies within `reach` = 3 cells per
+// by more cells than the distance allows).  Cells are much SMALLER than r: h =
+// r (1 + 2^-10) / 6, so an agent closer than r lies within `reach` = 6 cells per
 // axis (the 2^-10 margin is far above the fp32 rounding of the cell coordinate
 // and of d2), and the warm bound of k_grid prunes the stencil to the cells its
-// queries can reach (usually 1 per axis: 27 small cells instead of 27 cells of
-// size r).  The table is capped at MAXD cells per axis (single-CTA scan in
-// shared memory): larger worlds get larger cells and a smaller reach (>= 1).
-constexpr int MAXD = 34;
+// queries can reach (at C5's density 1 per axis: a warm limit of ~0.9 against
+// cells of 1.5).  The table is capped at MAXD cells per axis: larger worlds get
+// coarser cells and a smaller reach (>= 1).
+constexpr int MAXD = 128;
+constexpr int SEARCH_REACH = 6;
 BinGrid make_search_grid(const boids_params& p) {
   BinGrid g{};
   const float B = fmaxf(p.world_radius, p.init_radius) * 1.02f;
   const float hr = p.search_radius * (1.0f + 1.0f / 1024.0f);  // >= r with margin
-  int reach = 3;
-  float h = hr / 3.f;
+  int reach = SEARCH_REACH;
+  float h = hr / (float)reach;
   int dim = (int)ceilf(2.f * B / h);
-  while (dim > MAXD && reach > 1) {  // coarser cells: reach 2, then 1 (cells >= r)
+  while (dim > MAXD && reach > 1) {  // coarser cells, down to cells >= r (reach 1)
     --reach;
     h = hr / (float)reach;
     dim = (int)ceilf(2.f * B / h);
@@ -379,6 +383,24 @@ BinGrid make_search_grid(const boids_params& p) {
   g.cells = dim * dim * dim;
   g.morton = 0;
   g.reach = reach;
+  g.fdim = dim;
+  return g;
+}
+
+// The grid search's query blocks: QBLOCK^3 cells of the search grid.  A work
+// item of k_grid is (a run along x of) one block's queries, so its stencil is a
+// compact box -- (QBLOCK + 2R)^3 cells around QBLOCK^3 -- instead of the long thin
+// one of a run of cells along x (C5: ~1500 instead of ~4200 candidates per
+// query); the queries are binned by block (cell_of on a block grid divides the
+// fine cell coordinates, so a query's block always contains its fine cell).
+constexpr int QBLOCK = 4;
+BinGrid make_query_grid(const BinGrid& sg) {
+  BinGrid g = sg;
+  g.block = QBLOCK;
+  g.fdim = sg.dim[0];
+  const int nb = (sg.dim[0] + QBLOCK - 1) / QBLOCK;
+  for (int d = 0; d < 3; ++d) g.dim[d] = nb;
+  g.cells = nb * nb * nb;
   return g;
 }
 

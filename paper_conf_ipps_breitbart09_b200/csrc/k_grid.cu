@@ -42,6 +42,7 @@ constexpr int CT = 256;         // candidates per tile (<= 4 KB bulk copy)
 constexpr int STAGES = 3;
 constexpr int U = 4;
 constexpr int FAR_MAX = 16;  // queries per item routed to k_grid_far
+constexpr int MAXROWS = 256;  // stencil rows of an item: (QBLOCK + 2 reach)^2 <= (4 + 12)^2
 // Query slot of (warp, q, lane).  Round-robin over the warps (BOIDS_GRID_RR=1):
 // an item with fewer than QBG queries still keeps every warp working, at the
 // cost of computing the padded slots; blocked (0): a warp's 4 x 32 queries are
@@ -63,8 +64,9 @@ struct __align__(16) GridSmem {
   key_t lists[7 * QBG];  // [7][QBG]
   uint64_t full[STAGES];
   uint64_t empty[STAGES];
-  int2 range[49];        // stencil row ranges [lo, hi) in the sorted candidate array ((2R+1)^2 <= 49)
+  int2 range[MAXROWS];   // stencil row ranges [lo, hi) in the sorted candidate array (empty ones too)
   int nrange, item, cell, span, qs0, qn;
+  unsigned long long cand;  // candidates of the item's stencil (grid_pairs accounting)
   int maxlim;            // largest query limit of the item (float bits; limits are >= 0)
   int maxnear;           // ... over the queries that need only the adjacent cells
   int nfar;              // queries that need more (routed to k_grid_far when few)
@@ -72,11 +74,11 @@ struct __align__(16) GridSmem {
 
 // A bound for a query whose warm bound reaches past the adjacent cells (a cold
 // step, an agent that wrapped to the diametric opposite point, or whose
-// neighbours did): the 7th smallest d2 to the other agents of its own cell,
-// which the binning of THIS step put together (current positions).  Real,
-// distinct agents, so an upper bound on the 7th key like t0; +inf with fewer
-// than 7.  It usually brings the query back within the adjacent cells, so it
-// is searched in its item instead of by k_grid_far.
+// neighbours did): the 7th smallest d2 to the other agents of the 3 x 3 x 3
+// cells around its own, which the binning of THIS step put together (current
+// positions).  Real, distinct agents, so an upper bound on the 7th key like t0;
+// +inf with fewer than 7.  It usually brings the query back within the adjacent
+// cells, so it is searched in its item instead of by k_grid_far.
 __device__ float cell_bound(const GridArgs& g, float4 me, int gi) {
   auto coord = [&](float v, int d) {
     const int c = (int)floorf((v - g.grid.lo[d]) * g.grid.inv_h);
@@ -86,52 +88,80 @@ __device__ float cell_bound(const GridArgs& g, float4 me, int gi) {
 #pragma unroll
   for (int k = 0; k < 7; ++k) b[k] = __int_as_float(0x7f800000);
   if (!(me.x == me.x && me.y == me.y && me.z == me.z)) return b[6];
-  const int cell = (coord(me.z, 2) * g.grid.dim[1] + coord(me.y, 1)) * g.grid.dim[0] + coord(me.x, 0);
-  const int lo = __ldg(g.cstart + cell), hi = __ldg(g.cstart + cell + 1);
-  constexpr int G = 16;  // loads in flight
-  for (int k0 = lo; k0 < hi; k0 += G) {
-    float4 c[G];
+  const int D = g.grid.dim[0];
+  const int cx = coord(me.x, 0), cy = coord(me.y, 1), cz = coord(me.z, 2);
+  const int x0 = max(cx - 1, 0), x1 = min(cx + 1, D - 1);
+  for (int z = max(cz - 1, 0); z <= min(cz + 1, D - 1); ++z)
+    for (int y = max(cy - 1, 0); y <= min(cy + 1, D - 1); ++y) {
+      const int row = (z * D + y) * D;
+      const int lo = __ldg(g.cstart + row + x0), hi = __ldg(g.cstart + row + x1 + 1);
+      constexpr int G = 8;  // loads in flight
+      for (int k0 = lo; k0 < hi; k0 += G) {
+        float4 c[G];
 #pragma unroll
-    for (int k = 0; k < G; ++k)
-      c[k] = k0 + k < hi ? __ldg(g.spos + k0 + k) : make_float4(__int_as_float(0x7fc00000), 0.f, 0.f, 0.f);
+        for (int k = 0; k < G; ++k)
+          c[k] = k0 + k < hi ? __ldg(g.spos + k0 + k) : make_float4(__int_as_float(0x7fc00000), 0.f, 0.f, 0.f);
 #pragma unroll
-    for (int k = 0; k < G; ++k) {
-      if (__float_as_int(c[k].w) == gi) continue;
-      float d = dist2(me.x, me.y, me.z, c[k]);
-      if (!(d == d)) continue;
+        for (int k = 0; k < G; ++k) {
+          if (__float_as_int(c[k].w) == gi) continue;
+          float d = dist2(me.x, me.y, me.z, c[k]);
+          if (!(d == d)) continue;
 #pragma unroll
-      for (int t = 0; t < 7; ++t) {  // keep the 7 smallest, ascending
-        const float l = fminf(b[t], d);
-        d = fmaxf(b[t], d);
-        b[t] = l;
+          for (int t = 0; t < 7; ++t) {  // keep the 7 smallest, ascending
+            const float l = fminf(b[t], d);
+            d = fmaxf(b[t], d);
+            b[t] = l;
+          }
+        }
       }
     }
-  }
   return b[6];
 }
 
-__device__ __forceinline__ int tile_count(const GridSmem& sm, int r, int off) {
-  return min(CT, sm.range[r].y - (sm.range[r].x + off));
-}
-
-// Advance a (range, offset) tile iterator.
-__device__ __forceinline__ void next_tile(const GridSmem& sm, int& r, int& off) {
-  off += CT;
-  if (sm.range[r].x + off >= sm.range[r].y) {
-    ++r;
-    off = 0;
+// Tiles concatenate consecutive stencil rows: a tile takes up to CT candidates
+// from ranges r, r+1, ... (one bulk copy per piece, into consecutive ring
+// slots, all completing on the stage's full barrier), so the short rows of a
+// compact stencil (~40 candidates each at C5) still fill whole tiles.
+// walk(): the tile at (r, off) -> its candidate count; (r, off) advanced past it.
+__device__ __forceinline__ int walk(const GridSmem& sm, int& r, int& off) {
+  int cnt = 0;
+  while (r < sm.nrange && cnt < CT) {
+    const int len = sm.range[r].y - sm.range[r].x;
+    const int take = min(len - off, CT - cnt);
+    cnt += take;
+    off += take;
+    if (off >= len) {
+      ++r;
+      off = 0;
+    }
   }
+  return cnt;
 }
 
-__device__ __forceinline__ void issue(GridSmem& sm, const GridArgs& g, uint32_t tc, int r, int off) {
+__device__ __forceinline__ void issue(GridSmem& sm, const GridArgs& g, uint32_t tc, int& r, int& off) {
   const int s = (int)(tc % STAGES);
   if (tc >= STAGES) {
     mbar_wait(&sm.empty[s], ((tc - STAGES) / STAGES) & 1u);
     fence_proxy_async_smem();
   }
-  const int cnt = tile_count(sm, r, off);
+  int r2 = r, off2 = off;
+  const int cnt = walk(sm, r2, off2);
   mbar_arrive_expect_tx(&sm.full[s], cnt * (uint32_t)sizeof(float4));
-  tma_load_1d(sm.ring[s], g.spos + sm.range[r].x + off, cnt * (uint32_t)sizeof(float4), &sm.full[s]);
+  int done = 0;
+  while (done < cnt) {
+    const int len = sm.range[r].y - sm.range[r].x;
+    const int take = min(len - off, cnt - done);
+    if (take > 0)
+      tma_load_1d(sm.ring[s] + done, g.spos + sm.range[r].x + off, take * (uint32_t)sizeof(float4), &sm.full[s]);
+    done += take;
+    off += take;
+    if (off >= len) {
+      ++r;
+      off = 0;
+    }
+  }
+  r = r2;
+  off = off2;
 }
 
 // One tile of candidates against this thread's first QV queries (the rest of
@@ -170,13 +200,43 @@ __device__ __forceinline__ void grid_tile(const float4* tile, int cnt, const flo
     ++groups;
     if (__any_sync(0xffffffffu, m <= limc)) {
       ++slow_groups;
+      // Every lane collects its passing (query, candidate) pairs as bits, then
+      // the warp inserts them lane-parallel: each round every lane with bits
+      // left inserts its lowest one, so the warp runs max-per-lane rounds of the
+      // insertion instead of one per distinct (q, u) any lane holds.  The order
+      // of insertions never matters (exact (d2, index) key; a pair above the
+      // tightened limit cannot be among the final 7).
+      unsigned bits = 0;
 #pragma unroll
       for (int u = 0; u < U; ++u) {
         const int j = __float_as_int(cc[u].w);  // original index
 #pragma unroll
         for (int q = 0; q < QV; ++q)
-          if (d[q][u] <= lim[q] && j != gq[q])
-            lim[q] = fminf(lim[q], insert_smem7(&lists[qslot(warp, q, lane)], QBG, make_key(d[q][u], j)));
+          if (d[q][u] <= lim[q] && j != gq[q]) bits |= 1u << (q * U + u);
+      }
+      while (__any_sync(0xffffffffu, bits != 0)) {
+        if (bits) {
+          const int b = __ffs(bits) - 1;
+          bits &= bits - 1;
+          float dd = 0.f, lq = 0.f;
+          int j = 0, qq = 0;
+#pragma unroll
+          for (int q = 0; q < QV; ++q)
+#pragma unroll
+            for (int u = 0; u < U; ++u)
+              if (b == q * U + u) {
+                dd = d[q][u];
+                j = __float_as_int(cc[u].w);
+                lq = lim[q];
+                qq = q;
+              }
+          if (dd <= lq) {  // the limit may have tightened since the bit was set
+            const float nl = insert_smem7(&lists[qslot(warp, qq, lane)], QBG, make_key(dd, j));
+#pragma unroll
+            for (int q = 0; q < QV; ++q)
+              if (q == qq) lim[q] = fminf(lim[q], nl);
+          }
+        }
       }
       limc = lim[0];
 #pragma unroll
@@ -285,34 +345,48 @@ __global__ void __launch_bounds__(NTG, 5) k_grid(StepArgs a, GridArgs g) {  // 5
       }
     }
     __syncthreads();
-    if (tid == 0) {
-      // stencil reach of this item: agents within sqrt(maxlim) are at most
-      // floor(sqrt(maxlim) / h) + 1 cells away per axis (margin 2^-10 >> fp32 rounding)
+    {
+      // Stencil of this item: its block run (QBLOCK^3 cells each, `span` + 1
+      // blocks along x) grown by R cells per side, where agents within
+      // sqrt(maxlim) are at most floor(sqrt(maxlim) / h) + 1 cells away per axis
+      // (margin 2^-10 >> fp32 rounding).  One range of the cell-sorted candidate
+      // array per row (y, z) of the box, computed by one thread each.
       const float ml = __int_as_float(sm.maxlim);
       const int Rg = g.grid.reach;
       const float cells = sqrtf(ml) * g.grid.inv_h * (1.0f + 1.0f / 1024.0f);
       const int R = cells >= (float)Rg ? Rg : min(Rg, 1 + (int)cells);
-      const int cell = sm.cell;
-      const int cx = cell % D, cy = (cell / D) % D, cz = cell / (D * D);
-      const int x0 = max(cx - R, 0), x1 = min(cx + sm.span + R, D - 1);
-      int nr = 0;
-      for (int z = max(cz - R, 0); z <= min(cz + R, D - 1); ++z)
-        for (int y = max(cy - R, 0); y <= min(cy + R, D - 1); ++y) {
-          const int row = (z * D + y) * D;
-          const int lo_r = g.cstart[row + x0], hi_r = g.cstart[row + x1 + 1];
-          if (hi_r > lo_r) sm.range[nr++] = make_int2(lo_r, hi_r);
-        }
-      sm.nrange = nr;
-      if (a.stats) {
-        long long cand = 0;
-        for (int r = 0; r < nr; ++r) cand += sm.range[r].y - sm.range[r].x;
-        atomicAdd(a.stats + 3, (unsigned long long)(cand * sm.qn));
+      const int NB = g.qgrid.dim[0], B = g.qgrid.block;
+      const int blk = sm.cell;
+      const int bx = blk % NB, by = (blk / NB) % NB, bz = blk / (NB * NB);
+      const int x0 = max(bx * B - R, 0), x1 = min((bx + sm.span + 1) * B - 1 + R, D - 1);
+      const int y0 = max(by * B - R, 0), y1 = min(by * B + B - 1 + R, D - 1);
+      const int z0 = max(bz * B - R, 0), z1 = min(bz * B + B - 1 + R, D - 1);
+      const int ny = y1 - y0 + 1, nrows = ny * (z1 - z0 + 1);
+      if (tid == 0) sm.cand = 0;
+      __syncthreads();
+      unsigned long long cand = 0;
+      for (int t = tid; t < nrows; t += NTG) {
+        const int row = ((z0 + t / ny) * D + (y0 + t % ny)) * D;
+        const int lo_r = __ldg(g.cstart + row + x0), hi_r = __ldg(g.cstart + row + x1 + 1);
+        sm.range[t] = make_int2(lo_r, hi_r);
+        cand += (unsigned long long)(hi_r - lo_r);
       }
-      // producer: first tiles of the item
-      int r = 0, off = 0;
-      for (int t = 0; t < STAGES && r < nr; ++t) {
-        issue(sm, g, tc + t, r, off);
-        next_tile(sm, r, off);
+      if (a.stats) {
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) cand += __shfl_xor_sync(0xffffffffu, cand, o);
+        if (lane == 0) atomicAdd(&sm.cand, cand);
+      }
+      if (tid == 0) sm.nrange = nrows;
+      __syncthreads();
+      if (tid == 0) {
+        if (a.stats) atomicAdd(a.stats + 3, sm.cand * (unsigned long long)sm.qn);
+        // producer: first tiles of the item
+        int r = 0, off = 0;
+        for (int t = 0; t < STAGES; ++t) {
+          while (r < nrows && sm.range[r].y == sm.range[r].x) ++r;
+          if (r >= nrows) break;
+          issue(sm, g, tc + t, r, off);
+        }
       }
     }
     __syncthreads();
@@ -328,13 +402,20 @@ __global__ void __launch_bounds__(NTG, 5) k_grid(StepArgs a, GridArgs g) {  // 5
     // consumers: walk the same tile sequence as the producer
     int pr = 0, poff = 0;  // producer iterator (thread 0): STAGES tiles ahead
     if (tid == 0)
-      for (int t = 0; t < STAGES && pr < nr; ++t) next_tile(sm, pr, poff);
+      for (int t = 0; t < STAGES; ++t) {  // mirror of the producer's first issues
+        while (pr < nr && sm.range[pr].y == sm.range[pr].x) ++pr;
+        if (pr >= nr) break;
+        walk(sm, pr, poff);
+      }
     int r = 0, off = 0;
-    while (r < nr) {
+    for (;;) {
+      // skip empty rows (a tile never starts on one unless nothing is left)
+      while (r < nr && sm.range[r].y == sm.range[r].x) ++r;
+      if (r >= nr) break;
       const int s = (int)(tc % STAGES);
       mbar_wait(&sm.full[s], (tc / STAGES) & 1u);
       const float4* tile = sm.ring[s];
-      const int cnt = tile_count(sm, r, off);
+      const int cnt = walk(sm, r, off);
       // warps without queries in this item only keep the ring protocol; a warp
       // computes only its query groups that hold queries (the item's last warp
       // is usually partial: the padded groups cost work and loosen the vote)
@@ -347,10 +428,9 @@ __global__ void __launch_bounds__(NTG, 5) k_grid(StepArgs a, GridArgs g) {  // 5
       // racecheck does not count a __syncwarp before one lane's arrive as ordering)
       mbar_arrive(&sm.empty[s]);
       ++tc;
-      next_tile(sm, r, off);
-      if (tid == 0 && pr < nr) {
-        issue(sm, g, tc + STAGES - 1, pr, poff);
-        next_tile(sm, pr, poff);
+      if (tid == 0) {
+        while (pr < nr && sm.range[pr].y == sm.range[pr].x) ++pr;
+        if (pr < nr) issue(sm, g, tc + STAGES - 1, pr, poff);
       }
     }
     // lists are final: finish this thread's agents
@@ -379,7 +459,7 @@ __global__ void __launch_bounds__(NTG, 5) k_grid(StepArgs a, GridArgs g) {  // 5
 constexpr int FT = 128;
 __global__ void __launch_bounds__(FT) k_grid_far(StepArgs a, GridArgs g) {
   __shared__ key_t wl[FT / 32][7];
-  __shared__ int2 rng[49];
+  __shared__ int2 rng[(2 * 6 + 1) * (2 * 6 + 1)];  // (2 reach + 1)^2 rows, reach <= 6
   __shared__ int nrng;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int nf = *g.fcount;
