@@ -172,6 +172,45 @@ BOIDS_API int boids_create(int64_t n, const boids_params* p, uint64_t seed, boid
 BOIDS_API int boids_create_shard(int64_t n, const boids_params* p, uint64_t seed, int32_t rank,
                        int32_t world, boids_ctx** out);
 
+/* ---- Spatial decomposition (future work of the thesis) ----
+ * A spatial shard of a grid-mode flock (search_mode BOIDS_GRID, think_every 1):
+ * rank `rank` of `world` OWNS the agents whose search-grid cell layer z lies in
+ * its slab [zb[rank], zb[rank+1]) (boundaries balance the initial agent counts,
+ * boids_spatial_bounds) and holds, besides them, only its HALO -- the agents
+ * within `reach` cell layers of the slab, i.e. within the search radius of any
+ * owned agent.  Indices stay global: the handle addresses all n agents (arrays
+ * of boids_get_state / get_neighbors have n rows; rows of agents not owned are
+ * meaningless, see boids_spatial_owned).  Every rank creates its handle from
+ * the same (n, params, seed).  A step is
+ *   boids_step_spatial(h, dt)           owned agents: search + steer + modify,
+ *                                       then pack the outgoing records;
+ *   boids_spatial_outbox(h, ...)        record counts per destination rank;
+ *   (caller moves the records: destination d's halo records of every rank into
+ *    d's halo inbox, migrant records likewise -- NCCL all-to-all, or copies);
+ *   boids_spatial_unpack(h, nh, nm)     apply the received records.
+ * Records are float4 arrays: halo = 2 float4 (x, y, z, index bits | forward,
+ * speed); migrant = 8 float4 (the whole per-agent state incl. neighbour lists).
+ * Outbox of destination d: halo_out + d * cap_halo * 2 float4, mig_out + d *
+ * cap_mig * 8 float4.  The results are those of the single-GPU step (identical
+ * neighbour lists and states for every agent, each computed by its owner). */
+BOIDS_API int boids_create_spatial(int64_t n, const boids_params* p, uint64_t seed, int32_t rank, int32_t world,
+                                   boids_ctx** out);
+BOIDS_API int boids_step_spatial(boids_ctx* ctx, float dt);
+/* Synchronises.  halo_counts / mig_counts: world int32 each (records for each
+ * destination; 0 for this rank).  BOIDS_ENOMEM if an outbox overflowed. */
+BOIDS_API int boids_spatial_outbox(boids_ctx* ctx, int32_t* halo_counts, int32_t* mig_counts, void** halo_out,
+                                   void** mig_out, int64_t* cap_halo, int64_t* cap_mig);
+/* Device inboxes (records are placed at their start, contiguous) and capacities in records. */
+BOIDS_API int boids_spatial_inbox(boids_ctx* ctx, void** halo_in, void** mig_in, int64_t* cap_halo_in,
+                                  int64_t* cap_mig_in);
+/* Apply n_halo halo and n_mig migrant records from the inboxes (asynchronous).
+ * BOIDS_EINVAL if a count exceeds its inbox capacity. */
+BOIDS_API int boids_spatial_unpack(boids_ctx* ctx, int64_t n_halo, int64_t n_mig);
+/* own[n]: 1 for the agents this rank owns now.  Synchronises. */
+BOIDS_API int boids_spatial_owned(boids_ctx* ctx, uint8_t* own);
+/* zb[world + 1]: slab boundaries in search-cell layers; *reach: halo width in layers. */
+BOIDS_API int boids_spatial_bounds(boids_ctx* ctx, int32_t* zb, int32_t* reach);
+
 /* Enqueue all later work on `cuda_stream` (a cudaStream_t; NULL = legacy default). */
 BOIDS_API int boids_set_stream(boids_ctx* ctx, void* cuda_stream);
 

@@ -34,7 +34,10 @@ EXPORTS = (
     "boids_sync", "boids_info", "boids_get_profile", "boids_get_phases", "boids_destroy", "boids_last_error",
     "boids_get_think_state", "boids_set_think_state", "boids_readback_begin", "boids_readback_wait",
     "boids_get_accel", "boids_set_accel", "boids_bench_update",
+    "boids_create_spatial", "boids_step_spatial", "boids_spatial_outbox", "boids_spatial_inbox",
+    "boids_spatial_unpack", "boids_spatial_owned", "boids_spatial_bounds",
 )
+SPATIAL_HALO_F4, SPATIAL_MIG_F4 = 2, 8  # float4 per halo / migrant record (include/boids.h)
 # boids_info_t.last_path
 BOIDS_PATH_FUSED, BOIDS_PATH_SCAN, BOIDS_PATH_SYM, BOIDS_PATH_GRID, BOIDS_PATH_SIMPLE, BOIDS_PATH_THINK = range(6)
 
@@ -105,6 +108,13 @@ def load(path: str = LIB_PATH):
         "boids_get_think_state": (C.c_int, [vp, C.POINTER(i64), fp]),
         "boids_set_think_state": (C.c_int, [vp, i64, fp]),
         "boids_bench_update": (C.c_int, [vp, f32, i32, C.POINTER(C.c_double)]),
+        "boids_create_spatial": (C.c_int, [i64, P, C.c_uint64, i32, i32, C.POINTER(vp)]),
+        "boids_step_spatial": (C.c_int, [vp, f32]),
+        "boids_spatial_outbox": (C.c_int, [vp, ip, ip, C.POINTER(vp), C.POINTER(vp), C.POINTER(i64), C.POINTER(i64)]),
+        "boids_spatial_inbox": (C.c_int, [vp, C.POINTER(vp), C.POINTER(vp), C.POINTER(i64), C.POINTER(i64)]),
+        "boids_spatial_unpack": (C.c_int, [vp, i64, i64]),
+        "boids_spatial_owned": (C.c_int, [vp, C.POINTER(C.c_uint8)]),
+        "boids_spatial_bounds": (C.c_int, [vp, ip, ip]),
         "boids_destroy": (None, [vp]),
         "boids_last_error": (C.c_char_p, []),
     }
@@ -285,6 +295,50 @@ def boids_bench_update(h: int, dt: float, reps: int = 1) -> float:
     ms = C.c_double()
     _check(load().boids_bench_update(h, dt, reps, C.byref(ms)))
     return ms.value
+
+
+def boids_create_spatial(n: int, params=None, seed: int = 1, rank: int = 0, world: int = 1) -> int:
+    h = C.c_void_p()
+    _check(load().boids_create_spatial(n, C.byref(params or boids_default_params()), C.c_uint64(seed), rank, world,
+                                       C.byref(h)))
+    return h.value
+
+
+def boids_step_spatial(h: int, dt: float):
+    _check(load().boids_step_spatial(h, C.c_float(dt)))
+
+
+def boids_spatial_outbox(h: int, world: int):
+    """(halo_counts (world,), mig_counts (world,), halo_out ptr, mig_out ptr, cap_halo, cap_mig)."""
+    hc = np.zeros(world, np.int32)
+    mc = np.zeros(world, np.int32)
+    ho, mo, ch, cm = C.c_void_p(), C.c_void_p(), C.c_int64(), C.c_int64()
+    _check(load().boids_spatial_outbox(h, _iptr(hc), _iptr(mc), C.byref(ho), C.byref(mo), C.byref(ch), C.byref(cm)))
+    return hc, mc, ho.value, mo.value, ch.value, cm.value
+
+
+def boids_spatial_inbox(h: int):
+    """(halo_in ptr, mig_in ptr, cap_halo_in, cap_mig_in)."""
+    hi, mi, ch, cm = C.c_void_p(), C.c_void_p(), C.c_int64(), C.c_int64()
+    _check(load().boids_spatial_inbox(h, C.byref(hi), C.byref(mi), C.byref(ch), C.byref(cm)))
+    return hi.value, mi.value, ch.value, cm.value
+
+
+def boids_spatial_unpack(h: int, n_halo: int, n_mig: int):
+    _check(load().boids_spatial_unpack(h, n_halo, n_mig))
+
+
+def boids_spatial_owned(h: int) -> np.ndarray:
+    own = np.zeros(_count(h), np.uint8)
+    _check(load().boids_spatial_owned(h, own.ctypes.data_as(C.POINTER(C.c_uint8))))
+    return own.astype(bool)
+
+
+def boids_spatial_bounds(h: int, world: int):
+    zb = np.zeros(world + 1, np.int32)
+    r = np.zeros(1, np.int32)
+    _check(load().boids_spatial_bounds(h, _iptr(zb), _iptr(r)))
+    return zb, int(r[0])
 
 
 def boids_destroy(h: int):

@@ -119,6 +119,17 @@ struct boids_ctx {
   // sequence (search path, resort-or-not, k_sym feedback parity, ping-pong
   // parity, dt); replayed with cudaGraphLaunch, the host-side step state advanced
   // by a dry run of one_step
+  // spatial shard (boids_create_spatial; k_spatial.cu): this rank owns the agents whose
+  // search-cell layer z is in [zb[rank], zb[rank+1]), holds them and its halo layers
+  bool spatial = false;
+  int sp_reach = 0;                        // halo width in cell layers (cells >= r)
+  int* zb = nullptr;                       // device slab boundaries [world + 1]
+  std::vector<int> zb_host;
+  unsigned char* own = nullptr;            // [n] 1 = owned
+  float4 *halo_out = nullptr, *mig_out = nullptr, *halo_in = nullptr, *mig_in = nullptr;
+  int64_t cap_h = 0, cap_m = 0, cap_in_h = 0, cap_in_m = 0;
+  int* sp_counts = nullptr;                // [2 world]: halo records per destination, then migrants
+  int* sp_overflow = nullptr;
   bool dry = false;
   bool capturing = false;  // one_step runs inside graph_step's stream capture
   bool use_graphs = false;  // BOIDS_OPT_GRAPH
@@ -220,6 +231,14 @@ void free_ctx(boids_ctx* c) {
   cudaFree(c->twarm);
   cudaFree(c->tcnt);
   cudaFree(c->ocheck);
+  cudaFree(c->zb);
+  cudaFree(c->own);
+  cudaFree(c->halo_out);
+  cudaFree(c->mig_out);
+  cudaFree(c->halo_in);
+  cudaFree(c->mig_in);
+  cudaFree(c->sp_counts);
+  cudaFree(c->sp_overflow);
   cudaFree(c->ubench);
   cudaFree(c->phase);
   cudaFree(c->sym_sp);
@@ -500,7 +519,7 @@ int one_step(boids_ctx* c, float dt) {
            if (e == cudaSuccess)
              e = launch_bin(a.full, c->m, a.sdiv, c->lo, c->nloc, c->qgrid, c->gcellrank, c->gcnt, c->gqstart,
                             nullptr, c->qperm, (int)c->lo, c->stream, nullptr, c->gitems, c->gnitems, chunk,
-                            c->counter, c->p.think_every, c->step_index, c->growbuf);
+                            c->counter, c->p.think_every, c->step_index, c->growbuf, c->spatial ? c->own : nullptr);
            return e;
          }, 6)))
       return rc;
@@ -604,6 +623,15 @@ int one_step(boids_ctx* c, float dt) {
     }
   }
   if (!c->shard) c->cur ^= 1;
+  if (c->spatial) {  // the new positions decide migrants and halo copies (k_spatial.cu)
+    CK(mset(c, c->sp_counts, 0, 2 * c->world * sizeof(int)));
+    if ((rc = launch(c, 2, [&] {
+           return launch_spatial_pack(c->buf[c->cur], c->m, c->n, c->own, c->up4, c->side4, c->nbr, c->cnt, c->nbr8,
+                                      c->acc4, c->sgrid, c->zb, c->world, c->rank, c->sp_reach, c->halo_out, c->cap_h,
+                                      c->mig_out, c->cap_m, c->sp_counts, c->sp_overflow, c->stream);
+         })))
+      return rc;
+  }
   c->warm = true;
   c->steering_valid = c->record_steering;
   c->step_index++;
@@ -626,7 +654,7 @@ int one_step(boids_ctx* c, float dt) {
 // each replayed launch is timed like an eager one.
 bool graph_ok(const boids_ctx* c) {
   const bool grid = c->p.search_mode == BOIDS_GRID;
-  return c->use_graphs && !c->shard && c->p.think_every == 1 && c->phase == nullptr && c->steps_taken >= 2 &&
+  return c->use_graphs && !c->shard && !c->spatial && c->p.think_every == 1 && c->phase == nullptr && c->steps_taken >= 2 &&
          (grid || (c->warm && c->kernel == BOIDS_KERNEL_FUSED));
 }
 
@@ -788,6 +816,154 @@ BOIDS_API int boids_create_shard(int64_t n, const boids_params* p, uint64_t seed
   return create_impl(n, p, seed, rank, world, true, out);
 }
 
+BOIDS_API int boids_create_spatial(int64_t n, const boids_params* p, uint64_t seed, int32_t rank, int32_t world,
+                                   boids_ctx** out) {
+  if (!out) return fail(BOIDS_EINVAL, "out is NULL");
+  *out = nullptr;
+  if (!p) return fail(BOIDS_EINVAL, "params is NULL");
+  if (p->search_mode != BOIDS_GRID) return fail(BOIDS_EINVAL, "spatial shards need search_mode = BOIDS_GRID");
+  if (p->think_every != 1) return fail(BOIDS_EINVAL, "spatial shards need think_every = 1");
+  if (world < 1 || world > 256 || rank < 0 || rank >= world) return fail(BOIDS_EINVAL, "bad rank/world");
+  boids_ctx* c = nullptr;
+  int rc = create_impl(n, p, seed, 0, 1, false, &c);
+  if (rc) return rc;
+  c->spatial = true;
+  c->rank = rank;
+  c->world = world;
+  c->sp_reach = c->sgrid.reach;
+  const int L = c->sgrid.dim[2];
+  auto bad = [&](cudaError_t e) -> int {
+    (void)cudaGetLastError();
+    free_ctx(c);
+    return fail(e == cudaErrorMemoryAllocation ? BOIDS_ENOMEM : BOIDS_ECUDA,
+                std::string("create_spatial: ") + cudaGetErrorString(e));
+  };
+  // slab boundaries: equal shares of the initial agents over the cell layers z
+  // (every rank holds all n initial agents and computes the same boundaries)
+  int* hist = nullptr;
+  cudaError_t e = cudaMalloc((void**)&hist, L * sizeof(int));
+  if (e == cudaSuccess) e = cudaMemsetAsync(hist, 0, L * sizeof(int), c->stream);
+  if (e == cudaSuccess) e = launch_zhist(c->buf[c->cur], n, c->sgrid, hist, c->stream);
+  std::vector<int> h(L, 0);
+  if (e == cudaSuccess) e = cudaMemcpyAsync(h.data(), hist, L * sizeof(int), cudaMemcpyDeviceToHost, c->stream);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(c->stream);
+  cudaFree(hist);
+  if (e != cudaSuccess) return bad(e);
+  c->zb_host.assign(world + 1, L);
+  c->zb_host[0] = 0;
+  int64_t cum = 0;
+  int g = 1;
+  for (int z = 0; z < L && g < world; ++z) {
+    cum += h[z];
+    while (g < world && cum * world >= (int64_t)g * n) c->zb_host[g++] = z + 1;
+  }
+  for (int k = 1; k <= world; ++k) c->zb_host[k] = std::max(c->zb_host[k], c->zb_host[k - 1]);
+  // outbox capacities: the largest halo band of the initial distribution, doubled
+  int64_t band = 0;
+  for (int d = 0; d < world; ++d) {
+    int64_t b = 0;
+    for (int z = std::max(0, c->zb_host[d] - c->sp_reach); z < c->zb_host[d]; ++z) b += h[z];
+    for (int z = c->zb_host[d + 1]; z < std::min(L, c->zb_host[d + 1] + c->sp_reach); ++z) b += h[z];
+    band = std::max(band, b);
+  }
+  c->cap_h = std::max<int64_t>(4096, 2 * band);
+  c->cap_m = std::max<int64_t>(4096, n / 16);
+  c->cap_in_h = c->cap_h * std::max(1, world - 1);
+  c->cap_in_m = c->cap_m * std::max(1, world - 1);
+  const size_t hf = spatial_halo_f4() * sizeof(float4), mf = spatial_mig_f4() * sizeof(float4);
+  if ((e = cudaMalloc((void**)&c->zb, (world + 1) * sizeof(int))) != cudaSuccess ||
+      (e = cudaMalloc((void**)&c->own, std::max<int64_t>(1, n))) != cudaSuccess ||
+      (e = cudaMalloc((void**)&c->halo_out, (size_t)world * c->cap_h * hf)) != cudaSuccess ||
+      (e = cudaMalloc((void**)&c->mig_out, (size_t)world * c->cap_m * mf)) != cudaSuccess ||
+      (e = cudaMalloc((void**)&c->halo_in, (size_t)c->cap_in_h * hf)) != cudaSuccess ||
+      (e = cudaMalloc((void**)&c->mig_in, (size_t)c->cap_in_m * mf)) != cudaSuccess ||
+      (e = cudaMalloc((void**)&c->sp_counts, 2 * world * sizeof(int))) != cudaSuccess ||
+      (e = cudaMalloc((void**)&c->sp_overflow, sizeof(int))) != cudaSuccess)
+    return bad(e);
+  if ((e = cudaMemcpyAsync(c->zb, c->zb_host.data(), (world + 1) * sizeof(int), cudaMemcpyHostToDevice,
+                           c->stream)) != cudaSuccess ||
+      (e = cudaMemsetAsync(c->sp_counts, 0, 2 * world * sizeof(int), c->stream)) != cudaSuccess ||
+      (e = cudaMemsetAsync(c->sp_overflow, 0, sizeof(int), c->stream)) != cudaSuccess ||
+      (e = launch_spatial_init(c->buf[c->cur], c->m, n, c->own, c->sgrid, c->zb, world, rank, c->sp_reach,
+                               c->stream)) != cudaSuccess ||
+      (e = cudaStreamSynchronize(c->stream)) != cudaSuccess)
+    return bad(e);
+  *out = c;
+  return BOIDS_OK;
+}
+
+BOIDS_API int boids_step_spatial(boids_ctx* c, float dt) {
+  if (!c) return fail(BOIDS_EINVAL, "NULL handle");
+  if (!c->spatial) return fail(BOIDS_EINVAL, "not a spatial handle");
+  int rc = check_dt(dt);
+  if (rc) return rc;
+  DeviceGuard g(c->dev);
+  return one_step(c, dt);
+}
+
+BOIDS_API int boids_spatial_outbox(boids_ctx* c, int32_t* halo_counts, int32_t* mig_counts, void** halo_out,
+                                   void** mig_out, int64_t* cap_halo, int64_t* cap_mig) {
+  if (!c) return fail(BOIDS_EINVAL, "NULL handle");
+  if (!c->spatial) return fail(BOIDS_EINVAL, "not a spatial handle");
+  DeviceGuard g(c->dev);
+  std::vector<int> cnt(2 * c->world);
+  int ovf = 0;
+  CK(cudaMemcpyAsync(cnt.data(), c->sp_counts, cnt.size() * sizeof(int), cudaMemcpyDeviceToHost, c->stream));
+  CK(cudaMemcpyAsync(&ovf, c->sp_overflow, sizeof(int), cudaMemcpyDeviceToHost, c->stream));
+  CK(cudaStreamSynchronize(c->stream));
+  if (ovf) return fail(BOIDS_ENOMEM, "spatial outbox overflow (more halo/migrant records than capacity)");
+  for (int d = 0; d < c->world; ++d) {
+    if (halo_counts) halo_counts[d] = cnt[d];
+    if (mig_counts) mig_counts[d] = cnt[c->world + d];
+  }
+  if (halo_out) *halo_out = c->halo_out;
+  if (mig_out) *mig_out = c->mig_out;
+  if (cap_halo) *cap_halo = c->cap_h;
+  if (cap_mig) *cap_mig = c->cap_m;
+  return BOIDS_OK;
+}
+
+BOIDS_API int boids_spatial_inbox(boids_ctx* c, void** halo_in, void** mig_in, int64_t* cap_halo_in,
+                                  int64_t* cap_mig_in) {
+  if (!c) return fail(BOIDS_EINVAL, "NULL handle");
+  if (!c->spatial) return fail(BOIDS_EINVAL, "not a spatial handle");
+  if (halo_in) *halo_in = c->halo_in;
+  if (mig_in) *mig_in = c->mig_in;
+  if (cap_halo_in) *cap_halo_in = c->cap_in_h;
+  if (cap_mig_in) *cap_mig_in = c->cap_in_m;
+  return BOIDS_OK;
+}
+
+BOIDS_API int boids_spatial_unpack(boids_ctx* c, int64_t n_halo, int64_t n_mig) {
+  if (!c) return fail(BOIDS_EINVAL, "NULL handle");
+  if (!c->spatial) return fail(BOIDS_EINVAL, "not a spatial handle");
+  if (n_halo < 0 || n_mig < 0 || n_halo > c->cap_in_h || n_mig > c->cap_in_m)
+    return fail(BOIDS_EINVAL, "record counts outside the inbox capacities");
+  DeviceGuard g(c->dev);
+  CK(launch_spatial_unpack(c->halo_in, n_halo, c->mig_in, n_mig, c->buf[c->cur], c->m, c->own, c->up4, c->side4,
+                           c->nbr, c->cnt, c->nbr8, c->acc4, c->stream));
+  c->launches += (n_halo > 0) + (n_mig > 0);
+  return BOIDS_OK;
+}
+
+BOIDS_API int boids_spatial_owned(boids_ctx* c, uint8_t* own) {
+  if (!c || !own) return fail(BOIDS_EINVAL, "NULL argument");
+  if (!c->spatial) return fail(BOIDS_EINVAL, "not a spatial handle");
+  DeviceGuard g(c->dev);
+  CK(cudaMemcpyAsync(own, c->own, c->n, cudaMemcpyDeviceToHost, c->stream));
+  CK(cudaStreamSynchronize(c->stream));
+  return BOIDS_OK;
+}
+
+BOIDS_API int boids_spatial_bounds(boids_ctx* c, int32_t* zb, int32_t* reach) {
+  if (!c) return fail(BOIDS_EINVAL, "NULL handle");
+  if (!c->spatial) return fail(BOIDS_EINVAL, "not a spatial handle");
+  if (zb)
+    for (int k = 0; k <= c->world; ++k) zb[k] = c->zb_host[k];
+  if (reach) *reach = c->sp_reach;
+  return BOIDS_OK;
+}
+
 BOIDS_API int boids_set_stream(boids_ctx* c, void* stream) {
   if (!c) return fail(BOIDS_EINVAL, "NULL handle");
   c->stream = (cudaStream_t)stream;
@@ -853,6 +1029,7 @@ BOIDS_API int boids_set_option(boids_ctx* c, int32_t opt, int64_t v) {
 BOIDS_API int boids_step(boids_ctx* c, float dt, int32_t steps) {
   if (!c) return fail(BOIDS_EINVAL, "NULL handle");
   if (c->shard) return fail(BOIDS_EINVAL, "shard handle: use boids_step_shard after the all-gather");
+  if (c->spatial) return fail(BOIDS_EINVAL, "spatial handle: use boids_step_spatial + the record exchange");
   int rc = check_dt(dt);
   if (rc) return rc;
   if (steps < 0) return fail(BOIDS_EINVAL, "steps must be >= 0");
@@ -942,6 +1119,11 @@ BOIDS_API int boids_set_state(boids_ctx* c, const float* pos3, const float* fwd3
   CK(cudaMemcpyAsync(st + 12 * k, speed, k * sizeof(float), cudaMemcpyHostToDevice, c->stream));
   CK(launch_state_in(st, side3 != nullptr, k, c->local(), c->m, c->up4, c->side4, c->stream));
   c->launches++;
+  if (c->spatial) {  // all n uploaded: own / halo / cleared again from the new positions
+    CK(launch_spatial_init(c->local(), c->m, c->n, c->own, c->sgrid, c->zb, c->world, c->rank, c->sp_reach,
+                           c->stream));
+    c->launches++;
+  }
   // The previous neighbour lists are KEPT: the warm bound they seed (the 7th
   // smallest current distance to 7-8 distinct existing agents) is an upper bound
   // on the 7th neighbour distance for ANY positions, so the next step stays exact;

@@ -193,7 +193,8 @@ cudaError_t launch_bin(const float4* full, int64_t m, const SliceDiv& sd, int64_
                        int2* cellrank, int* cnt, int* start, float4* spos, int* perm, int perm_base,
                        cudaStream_t s, int* launches, int4* items = nullptr, int* nitems = nullptr, int chunk = 1,
                        int* counter = nullptr, int think_k = 1, int64_t think_t = 0,
-                       int* rowbuf = nullptr);  // [2 * rows] scratch: large grids scan on many CTAs
+                       int* rowbuf = nullptr,  // [2 * rows] scratch: large grids scan on many CTAs
+                       const unsigned char* own = nullptr);  // spatial shards: bin only agents with own[k]
 BinGrid make_locality_grid(int64_t n, const boids_params& p);
 BinGrid make_search_grid(const boids_params& p);
 BinGrid make_query_grid(const BinGrid& search);  // blocks of the search grid: the grid search's work items
@@ -229,5 +230,19 @@ cudaError_t launch_sym_scan(const StepArgs& a, float4* sp, int* sidx, const long
                             long long* splits, cudaStream_t s);
 cudaError_t launch_route(const StepArgs& a, cudaStream_t s);
 int fused_auto_cluster(int64_t n_pad_total, int64_t nloc, int sm_count);
+// spatial shards (k_spatial.cu)
+int spatial_halo_f4();
+int spatial_mig_f4();
+cudaError_t launch_zhist(const float4* cur, int64_t n, const BinGrid& g, int* hist, cudaStream_t s);
+cudaError_t launch_spatial_init(float4* cur, int64_t m, int64_t n, unsigned char* own, const BinGrid& g,
+                                const int* zb, int world, int rank, int reach, cudaStream_t s);
+cudaError_t launch_spatial_pack(float4* cur, int64_t m, int64_t n, unsigned char* own, const float4* up4,
+                                const float4* side4, const int32_t* nbr, const int32_t* cnt, const int32_t* nbr8,
+                                const float4* acc4, const BinGrid& g, const int* zb, int world, int rank, int reach,
+                                float4* halo_out, int64_t cap_h, float4* mig_out, int64_t cap_m, int* counts,
+                                int* overflow, cudaStream_t s);
+cudaError_t launch_spatial_unpack(const float4* halo_in, int64_t nh, const float4* mig_in, int64_t nm, float4* cur,
+                                  int64_t m, unsigned char* own, float4* up4, float4* side4, int32_t* nbr,
+                                  int32_t* cnt, int32_t* nbr8, float4* acc4, cudaStream_t s);
 
 }  // namespace boids

@@ -25,10 +25,11 @@ namespace boids {
 // pad every slice -- are skipped (candidate binning).
 __global__ void k_bin_count(const float4* __restrict__ full, int64_t m, SliceDiv sd, int64_t j0, int64_t count,
                             BinGrid g, int2* __restrict__ cellrank, int* __restrict__ cnt, int keep_nan,
-                            int think_k, int64_t think_t) {
+                            int think_k, int64_t think_t, const unsigned char* __restrict__ own) {
   int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (k >= count) return;
-  if (!thinks(j0 + k, think_t, think_k)) {  // think mode: only this step's thinkers are queries
+  // think mode: only this step's thinkers are queries; spatial shards: only the owned agents
+  if (!thinks(j0 + k, think_t, think_k) || (own && !own[k])) {
     cellrank[k] = make_int2(-1, 0);
     return;
   }
@@ -295,7 +296,7 @@ __global__ void k_bin_scatter(const float4* __restrict__ full, int64_t m, SliceD
 cudaError_t launch_bin(const float4* full, int64_t m, const SliceDiv& sd, int64_t j0, int64_t count, const BinGrid& g,
                        int2* cellrank, int* cnt, int* start, float4* spos, int* perm, int perm_base,
                        cudaStream_t s, int* launches, int4* items, int* nitems, int chunk, int* counter,
-                       int think_k, int64_t think_t, int* rowbuf) {
+                       int think_k, int64_t think_t, int* rowbuf, const unsigned char* own) {
   const unsigned blocks = (unsigned)((count + 255) / 256);
   const int rows = g.cells / g.dim[0];
   // think mode: items hold only this step's thinkers (1/k of the agents); longer
@@ -317,8 +318,8 @@ cudaError_t launch_bin(const float4* full, int64_t m, const SliceDiv& sd, int64_
   BOIDS_PREFER_SMEM(k_bin_scatter);
   BOIDS_PREFER_SMEM(k_bin_scan);
   if (count > 0)
-    k_bin_count<<<blocks, 256, 0, s>>>(full, m, sd, j0, count, g, cellrank, cnt, spos == nullptr,
-                                       spos == nullptr ? think_k : 1, think_t);
+    k_bin_count<<<blocks, 256, 0, s>>>(full, m, sd, j0, count, g, cellrank, cnt, spos == nullptr && !own,
+                                       spos == nullptr ? think_k : 1, think_t, own);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return e;
   if (many) {  // large grid: many CTAs

@@ -24,13 +24,17 @@ __device__ __forceinline__ float warm_bound(const StepArgs& a, int64_t qi, float
 #pragma unroll
   for (int k = 0; k < 8; ++k) p[k] = __ldg(pos_of(a.full, a.m, a.sdiv, nb[k] < 0 ? 0 : nb[k]));
   float m1 = 0.f, m2 = 0.f;  // largest and second largest
+  bool absent = false;        // a previous neighbour whose position this handle does not hold
 #pragma unroll
   for (int k = 0; k < 8; ++k) {
     const float d = (k < 7 || nb[7] >= 0) ? dist2(me.x, me.y, me.z, p[k]) : 0.f;  // no 8th: ignore
+    absent |= !(d == d);
     m2 = fmaxf(m2, fminf(m1, d));
     m1 = fmaxf(m1, d);
   }
-  if (c < 7) return __int_as_float(0x7f800000);
+  // a spatial shard holds only its own agents and its halo (NaN elsewhere): a
+  // bound over fewer than the 7-8 real agents would not be one
+  if (c < 7 || absent) return __int_as_float(0x7f800000);
   return nb[7] >= 0 ? m2 : m1;
 }
 
