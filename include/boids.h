@@ -105,7 +105,8 @@ typedef struct boids_info_t {
   int64_t vote_groups; /* ... out of this many (diagnostics; boids_info synchronises) */
   int64_t fallbacks;   /* warm path, cumulative: agents searched whole (k_route) after a hit-buffer
                           overflow or, on k_sym steps, because their previous neighbours all
-                          left the radius (a wrap) */
+                          left the radius (a wrap); grid mode: queries whose bound reached past the
+                          adjacent cells, searched alone by k_grid_far */
   int64_t grid_pairs;  /* grid mode, cumulative: (query, candidate) pairs evaluated over the
                           27-cell stencils -- the grid search's algorithmic work */
   int64_t step_index;  /* steps taken by this handle (the t of the think schedule) */

@@ -86,6 +86,8 @@ struct boids_ctx {
   // grid mode (BOIDS_GRID): search grid and its binning buffers
   BinGrid sgrid{};
   BinGrid qgrid{};  // blocks of sgrid: the queries' binning and the grid search's work items
+  // the grids the binning and the search use: sgrid / qgrid, or a spatial shard's slab of them
+  BinGrid bgrid{}, bqgrid{};
   int2* gcellrank = nullptr;
   int32_t *gcnt = nullptr, *gstart = nullptr, *gqstart = nullptr, *counter = nullptr;
   int4* gitems = nullptr;      // grid search work items (k_bin_scan)
@@ -129,6 +131,10 @@ struct boids_ctx {
   float4 *halo_out = nullptr, *mig_out = nullptr, *halo_in = nullptr, *mig_in = nullptr;
   int64_t cap_h = 0, cap_m = 0, cap_in_h = 0, cap_in_m = 0;
   int* sp_counts = nullptr;                // [2 world]: halo records per destination, then migrants
+  int* kept = nullptr;                     // [n] non-owned entries kept as halo locally (cleared next pack)
+  int* nkept = nullptr;                    // their number (device)
+  int64_t kept_bound = 0;                  // host upper bound of *nkept
+  int64_t last_nh = 0;                     // halo records applied by the last unpack (cleared next pack)
   int* sp_overflow = nullptr;
   bool dry = false;
   bool capturing = false;  // one_step runs inside graph_step's stream capture
@@ -239,6 +245,8 @@ void free_ctx(boids_ctx* c) {
   cudaFree(c->mig_in);
   cudaFree(c->sp_counts);
   cudaFree(c->sp_overflow);
+  cudaFree(c->kept);
+  cudaFree(c->nkept);
   cudaFree(c->ubench);
   cudaFree(c->phase);
   cudaFree(c->sym_sp);
@@ -373,17 +381,20 @@ int create_impl(int64_t n, const boids_params* p, uint64_t seed, int32_t rank, i
   if (p->search_mode == BOIDS_GRID) {
     c->sgrid = make_search_grid(*p);
     c->qgrid = make_query_grid(c->sgrid);
+    c->bgrid = c->sgrid;
+    c->bqgrid = c->qgrid;
     const int C = c->sgrid.cells;
     if ((rc = alloc((void**)&c->gcellrank, slots * sizeof(int2))) ||
         (rc = alloc((void**)&c->gcnt, C * sizeof(int32_t))) ||
         (rc = alloc((void**)&c->gstart, (C + 1) * sizeof(int32_t))) ||
         (rc = alloc((void**)&c->gqstart, (C + 1) * sizeof(int32_t))) ||
-        (rc = alloc((void**)&c->gitems, (size_t)(C + m / grid_chunk() + 2) * sizeof(int4))) ||
+        (rc = alloc((void**)&c->gitems, (size_t)(C + m / 128 + 2) * sizeof(int4))) ||
         (rc = alloc((void**)&c->gnitems, sizeof(int32_t))) ||
         (rc = alloc((void**)&c->growbuf, (size_t)2 * (C / c->sgrid.dim[0] + 1) * sizeof(int32_t))) ||
         (rc = alloc((void**)&c->counter, sizeof(int32_t))) ||
         (rc = alloc((void**)&c->sym_rlist, m * sizeof(int32_t))) ||
         (rc = alloc((void**)&c->sym_rcount, sizeof(int32_t))) ||
+        (rc = alloc((void**)&c->qlim, m * sizeof(float))) ||
         (rc = alloc((void**)&c->spos, (size_t)n * sizeof(float4)))) {
       free_ctx(c);
       return rc;
@@ -511,13 +522,14 @@ int one_step(boids_ctx* c, float dt) {
     // owned agents (this step's thinkers in think mode) by block of cells
     // (qperm, gqstart) and the work items over the blocks
     const int64_t slots = c->shard ? (int64_t)c->world * c->m : c->m;
-    const int chunk = grid_chunk();
+    // owned queries: a spatial shard owns about n / world of its n slots
+    const int chunk = grid_chunk(c->spatial ? c->nloc / c->world : c->nloc / (think ? c->p.think_every : 1));
     if ((rc = launch(c, 2, [&] {
-           cudaError_t e = launch_bin(a.full, c->m, a.sdiv, 0, slots, c->sgrid, c->gcellrank, c->gcnt, c->gstart,
+           cudaError_t e = launch_bin(a.full, c->m, a.sdiv, 0, slots, c->bgrid, c->gcellrank, c->gcnt, c->gstart,
                                       c->spos, nullptr, 0, c->stream, nullptr, nullptr, nullptr, chunk, nullptr, 1,
                                       0, c->growbuf);
            if (e == cudaSuccess)
-             e = launch_bin(a.full, c->m, a.sdiv, c->lo, c->nloc, c->qgrid, c->gcellrank, c->gcnt, c->gqstart,
+             e = launch_bin(a.full, c->m, a.sdiv, c->lo, c->nloc, c->bqgrid, c->gcellrank, c->gcnt, c->gqstart,
                             nullptr, c->qperm, (int)c->lo, c->stream, nullptr, c->gitems, c->gnitems, chunk,
                             c->counter, c->p.think_every, c->step_index, c->growbuf, c->spatial ? c->own : nullptr);
            return e;
@@ -532,9 +544,10 @@ int one_step(boids_ctx* c, float dt) {
     g.nitems = c->gnitems;
     g.flist = c->sym_rlist;  // (the brute-force routing list; unused in grid mode otherwise)
     g.fcount = c->sym_rcount;
+    g.flim = c->qlim;
     g.counter = c->counter;
-    g.grid = c->sgrid;
-    g.qgrid = c->qgrid;
+    g.grid = c->bgrid;
+    g.qgrid = c->bqgrid;
     StepArgs ag = a;
     ag.store_only = think ? 1 : 0;
     CK(mset(c, c->sym_rcount, 0, sizeof(int32_t)));
@@ -626,11 +639,14 @@ int one_step(boids_ctx* c, float dt) {
   if (c->spatial) {  // the new positions decide migrants and halo copies (k_spatial.cu)
     CK(mset(c, c->sp_counts, 0, 2 * c->world * sizeof(int)));
     if ((rc = launch(c, 2, [&] {
-           return launch_spatial_pack(c->buf[c->cur], c->m, c->n, c->own, c->up4, c->side4, c->nbr, c->cnt, c->nbr8,
+           return launch_spatial_pack(c->buf[c->cur], c->buf[c->cur ^ 1], c->m, c->n, c->own, c->up4, c->side4, c->nbr, c->cnt, c->nbr8,
                                       c->acc4, c->sgrid, c->zb, c->world, c->rank, c->sp_reach, c->halo_out, c->cap_h,
-                                      c->mig_out, c->cap_m, c->sp_counts, c->sp_overflow, c->stream);
+                                      c->mig_out, c->cap_m, c->sp_counts, c->sp_overflow, c->halo_in, c->last_nh,
+                                      c->kept, c->nkept, c->kept_bound, c->stream);
          })))
       return rc;
+    c->kept_bound = c->n;  // refined by boids_spatial_outbox (it reads the count)
+    c->last_nh = 0;
   }
   c->warm = true;
   c->steering_valid = c->record_steering;
@@ -866,6 +882,11 @@ BOIDS_API int boids_create_spatial(int64_t n, const boids_params* p, uint64_t se
     for (int z = c->zb_host[d + 1]; z < std::min(L, c->zb_host[d + 1] + c->sp_reach); ++z) b += h[z];
     band = std::max(band, b);
   }
+  // binning and search over this rank's layers only (its slab and halo): the
+  // cell tables and their scans shrink with the slab
+  c->bgrid = make_slab_grid(c->sgrid, std::max(0, c->zb_host[rank] - c->sp_reach),
+                            std::min(L, c->zb_host[rank + 1] + c->sp_reach));
+  c->bqgrid = make_query_grid(c->bgrid);
   c->cap_h = std::max<int64_t>(4096, 2 * band);
   c->cap_m = std::max<int64_t>(4096, n / 16);
   c->cap_in_h = c->cap_h * std::max(1, world - 1);
@@ -878,16 +899,20 @@ BOIDS_API int boids_create_spatial(int64_t n, const boids_params* p, uint64_t se
       (e = cudaMalloc((void**)&c->halo_in, (size_t)c->cap_in_h * hf)) != cudaSuccess ||
       (e = cudaMalloc((void**)&c->mig_in, (size_t)c->cap_in_m * mf)) != cudaSuccess ||
       (e = cudaMalloc((void**)&c->sp_counts, 2 * world * sizeof(int))) != cudaSuccess ||
-      (e = cudaMalloc((void**)&c->sp_overflow, sizeof(int))) != cudaSuccess)
+      (e = cudaMalloc((void**)&c->sp_overflow, sizeof(int))) != cudaSuccess ||
+      (e = cudaMalloc((void**)&c->kept, std::max<int64_t>(1, n) * sizeof(int))) != cudaSuccess ||
+      (e = cudaMalloc((void**)&c->nkept, sizeof(int))) != cudaSuccess)
     return bad(e);
   if ((e = cudaMemcpyAsync(c->zb, c->zb_host.data(), (world + 1) * sizeof(int), cudaMemcpyHostToDevice,
                            c->stream)) != cudaSuccess ||
       (e = cudaMemsetAsync(c->sp_counts, 0, 2 * world * sizeof(int), c->stream)) != cudaSuccess ||
       (e = cudaMemsetAsync(c->sp_overflow, 0, sizeof(int), c->stream)) != cudaSuccess ||
-      (e = launch_spatial_init(c->buf[c->cur], c->m, n, c->own, c->sgrid, c->zb, world, rank, c->sp_reach,
-                               c->stream)) != cudaSuccess ||
+      (e = launch_spatial_init(c->buf[c->cur], c->buf[c->cur ^ 1], c->m, n, c->own, c->sgrid, c->zb, world, rank,
+                               c->sp_reach, c->kept, c->nkept, c->stream)) != cudaSuccess ||
       (e = cudaStreamSynchronize(c->stream)) != cudaSuccess)
     return bad(e);
+  c->kept_bound = n;
+  c->last_nh = 0;
   *out = c;
   return BOIDS_OK;
 }
@@ -910,7 +935,10 @@ BOIDS_API int boids_spatial_outbox(boids_ctx* c, int32_t* halo_counts, int32_t* 
   int ovf = 0;
   CK(cudaMemcpyAsync(cnt.data(), c->sp_counts, cnt.size() * sizeof(int), cudaMemcpyDeviceToHost, c->stream));
   CK(cudaMemcpyAsync(&ovf, c->sp_overflow, sizeof(int), cudaMemcpyDeviceToHost, c->stream));
+  int nk = 0;
+  CK(cudaMemcpyAsync(&nk, c->nkept, sizeof(int), cudaMemcpyDeviceToHost, c->stream));
   CK(cudaStreamSynchronize(c->stream));
+  c->kept_bound = nk;
   if (ovf) return fail(BOIDS_ENOMEM, "spatial outbox overflow (more halo/migrant records than capacity)");
   for (int d = 0; d < c->world; ++d) {
     if (halo_counts) halo_counts[d] = cnt[d];
@@ -942,6 +970,7 @@ BOIDS_API int boids_spatial_unpack(boids_ctx* c, int64_t n_halo, int64_t n_mig) 
   DeviceGuard g(c->dev);
   CK(launch_spatial_unpack(c->halo_in, n_halo, c->mig_in, n_mig, c->buf[c->cur], c->m, c->own, c->up4, c->side4,
                            c->nbr, c->cnt, c->nbr8, c->acc4, c->stream));
+  c->last_nh = n_halo;  // these entries are cleared by the next pack (the inbox keeps their records)
   c->launches += (n_halo > 0) + (n_mig > 0);
   return BOIDS_OK;
 }
@@ -1120,8 +1149,10 @@ BOIDS_API int boids_set_state(boids_ctx* c, const float* pos3, const float* fwd3
   CK(launch_state_in(st, side3 != nullptr, k, c->local(), c->m, c->up4, c->side4, c->stream));
   c->launches++;
   if (c->spatial) {  // all n uploaded: own / halo / cleared again from the new positions
-    CK(launch_spatial_init(c->local(), c->m, c->n, c->own, c->sgrid, c->zb, c->world, c->rank, c->sp_reach,
-                           c->stream));
+    CK(launch_spatial_init(c->local(), c->buf[c->cur ^ 1], c->m, c->n, c->own, c->sgrid, c->zb, c->world, c->rank,
+                           c->sp_reach, c->kept, c->nkept, c->stream));
+    c->kept_bound = c->n;
+    c->last_nh = 0;
     c->launches++;
   }
   // The previous neighbour lists are KEPT: the warm bound they seed (the 7th

@@ -24,7 +24,7 @@ __device__ __forceinline__ int cell_coord(float v, const BinGrid& g, int d) {
 __device__ __forceinline__ int fine_coord(float v, const BinGrid& g, int d) {
   float t = (v - g.lo[d]) * g.inv_h;
   int c = (int)floorf(t);
-  return c < 0 ? 0 : (c >= g.fdim ? g.fdim - 1 : c);
+  return c < 0 ? 0 : (c >= g.fdim[d] ? g.fdim[d] - 1 : c);
 }
 
 __device__ __forceinline__ int cell_of(float4 p, const BinGrid& g) {

@@ -67,7 +67,7 @@ struct BinGrid {
   int block;   // > 0: a grid of BLOCKS of block^3 cells of the fine grid (lo, h, fdim): the block of a
                // position is its fine cell coordinate / block (so it agrees with the fine cell exactly);
                // dim[] then counts blocks per axis
-  int fdim;    // fine cells per axis (block > 0)
+  int fdim[3];  // fine cells per axis (block > 0)
 };
 
 struct StepArgs {
@@ -131,6 +131,7 @@ struct GridArgs {
   int* counter;           // work-queue counter (reset by the binning scan)
   int* flist;             // queries routed to k_grid_far (limit beyond the adjacent cells)
   int* fcount;            // their number (zeroed before k_grid)
+  float* flim;            // their search limits (inclusive d2 bound: min of r2, warm bound, cell bound)
   BinGrid grid;           // the fine search grid of the candidates (cstart)
   BinGrid qgrid;          // its blocks: the queries' binning (qstart, items; item.z = block index)
 };
@@ -198,6 +199,7 @@ cudaError_t launch_bin(const float4* full, int64_t m, const SliceDiv& sd, int64_
 BinGrid make_locality_grid(int64_t n, const boids_params& p);
 BinGrid make_search_grid(const boids_params& p);
 BinGrid make_query_grid(const BinGrid& search);  // blocks of the search grid: the grid search's work items
+BinGrid make_slab_grid(const BinGrid& search, int z0, int z1);  // layers [z0, z1) of a search grid
 cudaError_t launch_fill_nan(float4* p, int64_t count, cudaStream_t s);
 cudaError_t launch_apply(const StepArgs& a, cudaStream_t s);
 cudaError_t launch_pack_draw(const float4* local, int64_t m, const float4* up4, const float4* side4, int64_t k,
@@ -216,7 +218,7 @@ cudaError_t launch_fused(const StepArgs& a, int cluster, cudaStream_t s);
 cudaError_t launch_warm_scan(const StepArgs& a, cudaStream_t s);
 cudaError_t launch_grid(const StepArgs& a, const GridArgs& g, cudaStream_t s);
 cudaError_t launch_grid_far(const StepArgs& a, const GridArgs& g, cudaStream_t s);
-int grid_chunk();
+int grid_chunk(int64_t nq);  // queries per grid work item for nq queries
 // pdl: launch k_select1 as a programmatic dependent of the scan.  Measured: a
 // gain after k_scan (C1 30 -> 25 us/step), a loss after k_sym (C3 97 -> 121).
 cudaError_t launch_warm_select(const StepArgs& a, cudaStream_t s, bool pdl = true);
@@ -234,13 +236,15 @@ int fused_auto_cluster(int64_t n_pad_total, int64_t nloc, int sm_count);
 int spatial_halo_f4();
 int spatial_mig_f4();
 cudaError_t launch_zhist(const float4* cur, int64_t n, const BinGrid& g, int* hist, cudaStream_t s);
-cudaError_t launch_spatial_init(float4* cur, int64_t m, int64_t n, unsigned char* own, const BinGrid& g,
-                                const int* zb, int world, int rank, int reach, cudaStream_t s);
-cudaError_t launch_spatial_pack(float4* cur, int64_t m, int64_t n, unsigned char* own, const float4* up4,
+cudaError_t launch_spatial_init(float4* cur, float4* other, int64_t m, int64_t n, unsigned char* own,
+                                const BinGrid& g, const int* zb, int world, int rank, int reach, int* kept,
+                                int* nkept, cudaStream_t s);
+cudaError_t launch_spatial_pack(float4* cur, float4* prev, int64_t m, int64_t n, unsigned char* own, const float4* up4,
                                 const float4* side4, const int32_t* nbr, const int32_t* cnt, const int32_t* nbr8,
                                 const float4* acc4, const BinGrid& g, const int* zb, int world, int rank, int reach,
                                 float4* halo_out, int64_t cap_h, float4* mig_out, int64_t cap_m, int* counts,
-                                int* overflow, cudaStream_t s);
+                                int* overflow, const float4* halo_in, int64_t nh_prev, int* kept, int* nkept,
+                                int64_t nkept_cap, cudaStream_t s);
 cudaError_t launch_spatial_unpack(const float4* halo_in, int64_t nh, const float4* mig_in, int64_t nm, float4* cur,
                                   int64_t m, unsigned char* own, float4* up4, float4* side4, int32_t* nbr,
                                   int32_t* cnt, int32_t* nbr8, float4* acc4, cudaStream_t s);

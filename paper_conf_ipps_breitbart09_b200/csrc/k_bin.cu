@@ -15,6 +15,8 @@
 // (sorted query blocks and candidate stream -> spatially coherent warps, far
 // fewer insertion-path entries; every pair is still evaluated) and the
 // search grid of BOIDS_GRID (cells >= r, see k_grid.cu).
+#include <algorithm>
+
 #include "cells.cuh"
 
 namespace boids {
@@ -384,7 +386,7 @@ BinGrid make_search_grid(const boids_params& p) {
   g.cells = dim * dim * dim;
   g.morton = 0;
   g.reach = reach;
-  g.fdim = dim;
+  for (int d = 0; d < 3; ++d) g.fdim[d] = dim;
   return g;
 }
 
@@ -398,10 +400,23 @@ constexpr int QBLOCK = 4;
 BinGrid make_query_grid(const BinGrid& sg) {
   BinGrid g = sg;
   g.block = QBLOCK;
-  g.fdim = sg.dim[0];
-  const int nb = (sg.dim[0] + QBLOCK - 1) / QBLOCK;
-  for (int d = 0; d < 3; ++d) g.dim[d] = nb;
-  g.cells = nb * nb * nb;
+  for (int d = 0; d < 3; ++d) {
+    g.fdim[d] = sg.dim[d];
+    g.dim[d] = (sg.dim[d] + QBLOCK - 1) / QBLOCK;
+  }
+  g.cells = g.dim[0] * g.dim[1] * g.dim[2];
+  return g;
+}
+
+// A spatial shard's own part of the search grid: the cell layers z in [z0, z1)
+// (its slab plus its halo layers) with the x and y extent of the whole grid.
+// The cells are those of the full grid, so nothing but the table shrinks.
+BinGrid make_slab_grid(const BinGrid& sg, int z0, int z1) {
+  BinGrid g = sg;
+  g.lo[2] = sg.lo[2] + (float)z0 * sg.h;
+  g.dim[2] = std::max(1, z1 - z0);
+  g.fdim[2] = g.dim[2];
+  g.cells = g.dim[0] * g.dim[1] * g.dim[2];
   return g;
 }
 

@@ -29,6 +29,8 @@
 // list's own 7th key) is final at the end of the item, and the CTA finishes the
 // agents (steering + modification) itself: search, steering and modification
 // in one kernel, no merge.
+#include <algorithm>
+
 #include "step_common.cuh"
 #include "tma.cuh"
 
@@ -43,20 +45,15 @@ constexpr int STAGES = 3;
 constexpr int U = 4;
 constexpr int FAR_MAX = 16;  // queries per item routed to k_grid_far
 constexpr int MAXROWS = 256;  // stencil rows of an item: (QBLOCK + 2 reach)^2 <= (4 + 12)^2
-// Query slot of (warp, q, lane).  Round-robin over the warps (BOIDS_GRID_RR=1):
-// an item with fewer than QBG queries still keeps every warp working, at the
-// cost of computing the padded slots; blocked (0): a warp's 4 x 32 queries are
-// consecutive and warps past the item's queries only keep the ring protocol
-// (measured: round-robin C5 4.13 vs blocked 3.25 ms/step -- the padded slots cost
-// more than the idle warps).
-#ifndef BOIDS_GRID_RR
-#define BOIDS_GRID_RR 0
-#endif
-__device__ __forceinline__ int qslot(int warp, int q, int lane) {
-  return BOIDS_GRID_RR ? q * NTG + warp * 32 + lane : warp * 32 * Q + q * 32 + lane;
-}
-__device__ __forceinline__ bool warp_has_queries(int warp, int qn) {
-  return BOIDS_GRID_RR ? warp * 32 < qn : warp * 32 * Q < qn;
+// Query slot of (warp, q, lane).  Blocked (full items): a warp's 4 x 32 queries
+// are consecutive and warps past the item's queries only keep the ring protocol
+// (measured on full C5 items: round-robin 4.13 vs blocked 3.25 ms/step -- the
+// padded slots cost more than the idle warps).  Round-robin over the warps
+// (small items, <= RR_MAX queries: a spatial shard's or a sparse region's): q
+// group q of warp w holds slots q*NTG + 32w + lane, so every warp works.
+constexpr int RR_MAX = 2 * NTG;
+__device__ __forceinline__ int qslot(int warp, int q, int lane, bool rr) {
+  return rr ? q * NTG + warp * 32 + lane : warp * 32 * Q + q * 32 + lane;
 }
 
 struct __align__(16) GridSmem {
@@ -88,12 +85,12 @@ __device__ float cell_bound(const GridArgs& g, float4 me, int gi) {
 #pragma unroll
   for (int k = 0; k < 7; ++k) b[k] = __int_as_float(0x7f800000);
   if (!(me.x == me.x && me.y == me.y && me.z == me.z)) return b[6];
-  const int D = g.grid.dim[0];
+  const int Dx = g.grid.dim[0], Dy = g.grid.dim[1], Dz = g.grid.dim[2];
   const int cx = coord(me.x, 0), cy = coord(me.y, 1), cz = coord(me.z, 2);
-  const int x0 = max(cx - 1, 0), x1 = min(cx + 1, D - 1);
-  for (int z = max(cz - 1, 0); z <= min(cz + 1, D - 1); ++z)
-    for (int y = max(cy - 1, 0); y <= min(cy + 1, D - 1); ++y) {
-      const int row = (z * D + y) * D;
+  const int x0 = max(cx - 1, 0), x1 = min(cx + 1, Dx - 1);
+  for (int z = max(cz - 1, 0); z <= min(cz + 1, Dz - 1); ++z)
+    for (int y = max(cy - 1, 0); y <= min(cy + 1, Dy - 1); ++y) {
+      const int row = (z * Dy + y) * Dx;
       const int lo = __ldg(g.cstart + row + x0), hi = __ldg(g.cstart + row + x1 + 1);
       constexpr int G = 8;  // loads in flight
       for (int k0 = lo; k0 < hi; k0 += G) {
@@ -169,7 +166,7 @@ __device__ __forceinline__ void issue(GridSmem& sm, const GridArgs& g, uint32_t 
 template <int QV>
 __device__ __forceinline__ void grid_tile(const float4* tile, int cnt, const float2 (&pxy)[Q], const float (&pz)[Q],
                                           float (&lim)[Q], float& limc, const int (&gq)[Q], key_t* lists, int warp,
-                                          int lane, unsigned& groups, unsigned& slow_groups) {
+                                          int lane, bool rr, unsigned& groups, unsigned& slow_groups) {
   for (int c = 0; c < cnt; c += U) {
     float4 cc[U];
     if (c + U <= cnt) {
@@ -231,7 +228,7 @@ __device__ __forceinline__ void grid_tile(const float4* tile, int cnt, const flo
                 qq = q;
               }
           if (dd <= lq) {  // the limit may have tightened since the bit was set
-            const float nl = insert_smem7(&lists[qslot(warp, qq, lane)], QBG, make_key(dd, j));
+            const float nl = insert_smem7(&lists[qslot(warp, qq, lane, rr)], QBG, make_key(dd, j));
 #pragma unroll
             for (int q = 0; q < QV; ++q)
               if (q == qq) lim[q] = fminf(lim[q], nl);
@@ -281,6 +278,7 @@ __global__ void __launch_bounds__(NTG, 5) k_grid(StepArgs a, GridArgs g) {  // 5
     __syncthreads();
     if (sm.item >= n_items) break;
     const int qs0 = sm.qs0, qn = sm.qn;
+    const bool rr = qn <= RR_MAX;  // small item: query slots round-robin over the warps
 
     // queries: 4 per thread, with their limits (the warm bound)
     float2 pxy[Q];
@@ -289,7 +287,7 @@ __global__ void __launch_bounds__(NTG, 5) k_grid(StepArgs a, GridArgs g) {  // 5
     int64_t qloc[Q];
 #pragma unroll
     for (int q = 0; q < Q; ++q) {
-      const int slot = qslot(warp, q, lane);
+      const int slot = qslot(warp, q, lane, rr);
       const int64_t qi = slot < qn ? (int64_t)__ldg(g.qperm + qs0 + slot) : a.nloc;
       qloc[q] = qi;
       gq[q] = (int)(a.lo + qi);
@@ -336,7 +334,10 @@ __global__ void __launch_bounds__(NTG, 5) k_grid(StepArgs a, GridArgs g) {  // 5
 #pragma unroll
         for (int q = 0; q < Q; ++q)
           if (far[q]) {
-            g.flist[atomicAdd(g.fcount, 1)] = (int)qloc[q];
+            const int fs = atomicAdd(g.fcount, 1);
+            g.flist[fs] = (int)qloc[q];
+            g.flim[fs] = lim[q];  // its bound (warm bound, cell bound): k_grid_far's reach
+            if (a.stats) atomicAdd(a.stats + 2, 1ull);  // boids_info.fallbacks: queries searched by k_grid_far
             qloc[q] = a.nloc;  // not finished here
             pxy[q] = make_float2(__int_as_float(0x7fc00000), 0.f);
             lim[q] = -1.f;
@@ -355,18 +356,19 @@ __global__ void __launch_bounds__(NTG, 5) k_grid(StepArgs a, GridArgs g) {  // 5
       const int Rg = g.grid.reach;
       const float cells = sqrtf(ml) * g.grid.inv_h * (1.0f + 1.0f / 1024.0f);
       const int R = cells >= (float)Rg ? Rg : min(Rg, 1 + (int)cells);
-      const int NB = g.qgrid.dim[0], B = g.qgrid.block;
+      const int NBx = g.qgrid.dim[0], NBy = g.qgrid.dim[1], B = g.qgrid.block;
+      const int Dy = g.grid.dim[1], Dz = g.grid.dim[2];
       const int blk = sm.cell;
-      const int bx = blk % NB, by = (blk / NB) % NB, bz = blk / (NB * NB);
+      const int bx = blk % NBx, by = (blk / NBx) % NBy, bz = blk / (NBx * NBy);
       const int x0 = max(bx * B - R, 0), x1 = min((bx + sm.span + 1) * B - 1 + R, D - 1);
-      const int y0 = max(by * B - R, 0), y1 = min(by * B + B - 1 + R, D - 1);
-      const int z0 = max(bz * B - R, 0), z1 = min(bz * B + B - 1 + R, D - 1);
+      const int y0 = max(by * B - R, 0), y1 = min(by * B + B - 1 + R, Dy - 1);
+      const int z0 = max(bz * B - R, 0), z1 = min(bz * B + B - 1 + R, Dz - 1);
       const int ny = y1 - y0 + 1, nrows = ny * (z1 - z0 + 1);
       if (tid == 0) sm.cand = 0;
       __syncthreads();
       unsigned long long cand = 0;
       for (int t = tid; t < nrows; t += NTG) {
-        const int row = ((z0 + t / ny) * D + (y0 + t % ny)) * D;
+        const int row = ((z0 + t / ny) * Dy + (y0 + t % ny)) * D;
         const int lo_r = __ldg(g.cstart + row + x0), hi_r = __ldg(g.cstart + row + x1 + 1);
         sm.range[t] = make_int2(lo_r, hi_r);
         cand += (unsigned long long)(hi_r - lo_r);
@@ -392,7 +394,7 @@ __global__ void __launch_bounds__(NTG, 5) k_grid(StepArgs a, GridArgs g) {  // 5
     __syncthreads();
     const int nr = sm.nrange;
     // query groups of 32 slots this warp holds queries in (blocked slots)
-    const int qv = BOIDS_GRID_RR ? (warp * 32 < qn ? Q : 0) : max(0, min(Q, (qn - warp * 32 * Q + 31) / 32));
+    const int qv = rr ? max(0, min(Q, (qn - warp * 32 + NTG - 1) / NTG)) : max(0, min(Q, (qn - warp * 32 * Q + 31) / 32));
     float limc = 0.f;
 #pragma unroll
     for (int q = 0; q < Q; ++q)
@@ -419,10 +421,10 @@ __global__ void __launch_bounds__(NTG, 5) k_grid(StepArgs a, GridArgs g) {  // 5
       // warps without queries in this item only keep the ring protocol; a warp
       // computes only its query groups that hold queries (the item's last warp
       // is usually partial: the padded groups cost work and loosen the vote)
-      if (qv == 4) grid_tile<4>(tile, cnt, pxy, pz, lim, limc, gq, sm.lists, warp, lane, groups, slow_groups);
-      else if (qv == 3) grid_tile<3>(tile, cnt, pxy, pz, lim, limc, gq, sm.lists, warp, lane, groups, slow_groups);
-      else if (qv == 2) grid_tile<2>(tile, cnt, pxy, pz, lim, limc, gq, sm.lists, warp, lane, groups, slow_groups);
-      else if (qv == 1) grid_tile<1>(tile, cnt, pxy, pz, lim, limc, gq, sm.lists, warp, lane, groups, slow_groups);
+      if (qv == 4) grid_tile<4>(tile, cnt, pxy, pz, lim, limc, gq, sm.lists, warp, lane, rr, groups, slow_groups);
+      else if (qv == 3) grid_tile<3>(tile, cnt, pxy, pz, lim, limc, gq, sm.lists, warp, lane, rr, groups, slow_groups);
+      else if (qv == 2) grid_tile<2>(tile, cnt, pxy, pz, lim, limc, gq, sm.lists, warp, lane, rr, groups, slow_groups);
+      else if (qv == 1) grid_tile<1>(tile, cnt, pxy, pz, lim, limc, gq, sm.lists, warp, lane, rr, groups, slow_groups);
       // every thread releases the stage after its own reads (per-thread release
       // orders them before the stage's refill by the bulk copy; compute-sanitizer
       // racecheck does not count a __syncwarp before one lane's arrive as ordering)
@@ -437,7 +439,7 @@ __global__ void __launch_bounds__(NTG, 5) k_grid(StepArgs a, GridArgs g) {  // 5
     __syncwarp();
 #pragma unroll
     for (int q = 0; q < Q; ++q) {
-      const int slot = qslot(warp, q, lane);
+      const int slot = qslot(warp, q, lane, rr);
       if (slot < qn && qloc[q] < a.nloc) {
         key_t A[7];
 #pragma unroll
@@ -470,8 +472,7 @@ __global__ void __launch_bounds__(FT) k_grid_far(StepArgs a, GridArgs g) {
     const int qi = g.flist[f];
     const float4 me = __ldg(pos_of(a.full, a.m, a.sdiv, a.lo + qi));
     const int gi = (int)(a.lo + qi);
-    const float lim = fminf(fminf(r2_in, a.warm ? warm_bound(a, qi, me) : __int_as_float(0x7f800000)),
-                            cell_bound(g, me, gi));
+    const float lim = fminf(r2_in, g.flim[f]);  // computed once by k_grid when it routed the query
     if (tid == 0) {
       const int Rg = g.grid.reach;
       const float cells = sqrtf(lim) * g.grid.inv_h * (1.0f + 1.0f / 1024.0f);
@@ -482,11 +483,12 @@ __global__ void __launch_bounds__(FT) k_grid_far(StepArgs a, GridArgs g) {
         return c < 0 ? 0 : (c >= g.grid.dim[d] ? g.grid.dim[d] - 1 : c);
       };
       const int cx = coord(c4.x, 0), cy = coord(c4.y, 1), cz = coord(c4.z, 2);
+      const int Dy = g.grid.dim[1], Dz = g.grid.dim[2];
       const int x0 = max(cx - R, 0), x1 = min(cx + R, D - 1);
       int nr = 0;
-      for (int z = max(cz - R, 0); z <= min(cz + R, D - 1); ++z)
-        for (int y = max(cy - R, 0); y <= min(cy + R, D - 1); ++y) {
-          const int row = (z * D + y) * D;
+      for (int z = max(cz - R, 0); z <= min(cz + R, Dz - 1); ++z)
+        for (int y = max(cy - R, 0); y <= min(cy + R, Dy - 1); ++y) {
+          const int row = (z * Dy + y) * D;
           const int lo_r = g.cstart[row + x0], hi_r = g.cstart[row + x1 + 1];
           if (hi_r > lo_r) rng[nr++] = make_int2(lo_r, hi_r);
         }
@@ -556,6 +558,17 @@ cudaError_t launch_grid(const StepArgs& a, const GridArgs& g, cudaStream_t s) {
   return cudaGetLastError();
 }
 
-int grid_chunk() { return QBG; }
+// Queries per work item: QBG (512) for large query sets; fewer when the queries
+// would make fewer than ~3 items per persistent CTA (a spatial shard's ~n/G
+// owned agents), so every SM still gets several items (a block's queries are
+// then split over items that share its stencil: the same pairs, more items).
+int grid_chunk(int64_t nq) {
+  int dev = 0, sms = 148, r = 5;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const int64_t ctas = (int64_t)sms * r;
+  int64_t c = (nq / (3 * ctas) + 31) / 32 * 32;
+  return (int)std::max<int64_t>(128, std::min<int64_t>(QBG, c));
+}
 
 }  // namespace boids

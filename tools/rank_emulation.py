@@ -1,7 +1,7 @@
 """Per-rank step times of the G-rank sharded step, emulated on ONE GPU (the pool
 gives one GPU per call), and the G-GPU step time they project.
 
-    python tools/rank_emulation.py --workload c5 --ranks 1 2 4 8 [--steps 5 --warmup 3]
+    python tools/rank_emulation.py --workload c5 --ranks 1 2 4 8 [--steps 5 --warmup 3] [--spatial]
 
 For each G: G shard handles (boids_create_shard, ranks 0..G-1) live in this
 process; every step the NCCL all-gather is replaced by device copies of every
@@ -16,6 +16,12 @@ direction plus a fixed 15 us of NCCL latency (an assumption, stated in the
 output: no multi-GPU box was available to measure it).  The 1-GPU reference
 is the single-rank handle's own step (boids_create, k_sym / k_grid), so the
 projected scaling is against the best 1-GPU path, not against a 1-rank shard.
+
+--spatial (grid workloads): spatial shards instead (boids_create_spatial, slab
+ownership + halo layers; spatial.py).  Rank time = its boids_step_spatial +
+boids_spatial_unpack of the records it received; the exchange is estimated
+from the records actually sent (halo 32 B, migrant 128 B) at the same link rate
+plus latency, point to point (a rank receives from its slab neighbours).
 """
 from __future__ import annotations
 
@@ -94,12 +100,62 @@ def emulate(cfg, params, G, steps, warmup, flush):
             abi.boids_destroy(h)
 
 
+def emulate_spatial(cfg, params, G, steps, warmup, flush):
+    from paper_conf_ipps_breitbart09_b200.spatial import _views, inbox_layout
+
+    dev = torch.device("cuda", 0)
+    hs = [abi.boids_create_spatial(cfg.n, params, 1, r, G) for r in range(G)]
+    try:
+        stream = torch.cuda.current_stream().cuda_stream
+        for h in hs:
+            abi.boids_set_stream(h, stream)
+        per_rank = np.zeros((steps, G))
+        recv_bytes = np.zeros((steps, G))
+        for k in range(warmup + steps):
+            ts = []
+            for r, h in enumerate(hs):
+                flush.fill_(float(k * G + r))
+                a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                a.record()
+                abi.boids_step_spatial(h, float(W.DT))
+                b.record()
+                ts.append((a, b))
+            vs = [_views(h, G, dev) for h in hs]
+            hc = np.stack([v["hc"] for v in vs])
+            mc = np.stack([v["mc"] for v in vs])
+            hoff, htot = inbox_layout(hc)
+            moff, mtot = inbox_layout(mc)
+            for d, vd in enumerate(vs):
+                for s_, vs_ in enumerate(vs):
+                    if hc[s_, d]:
+                        vd["hin"][hoff[s_, d]:hoff[s_, d] + hc[s_, d]].copy_(vs_["hout"][d, :hc[s_, d]])
+                    if mc[s_, d]:
+                        vd["min"][moff[s_, d]:moff[s_, d] + mc[s_, d]].copy_(vs_["mout"][d, :mc[s_, d]])
+            us = []
+            for d, h in enumerate(hs):
+                a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                a.record()
+                abi.boids_spatial_unpack(h, int(htot[d]), int(mtot[d]))
+                b.record()
+                us.append((a, b))
+            torch.cuda.synchronize()
+            if k >= warmup:
+                for r in range(G):
+                    per_rank[k - warmup, r] = ts[r][0].elapsed_time(ts[r][1]) + us[r][0].elapsed_time(us[r][1])
+                    recv_bytes[k - warmup, r] = htot[r] * 32 + mtot[r] * 128
+        return per_rank.mean(0), recv_bytes.mean(0)
+    finally:
+        for h in hs:
+            abi.boids_destroy(h)
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--workload", default="c5", choices=sorted(W.CONFIGS))
     ap.add_argument("--ranks", type=int, nargs="+", default=[1, 2, 4, 8])
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--spatial", action="store_true", help="spatial shards (grid workloads) instead of index shards")
     args = ap.parse_args()
     cfg = W.CONFIGS[args.workload]
     torch.cuda.set_device(0)
@@ -109,7 +165,18 @@ def main():
     out = {"workload": cfg.name, "n": cfg.n, "one_gpu_ms": t1, "one_gpu_path": path1,
            "assumptions": f"all-gather = (G-1)/G x 32 B x n at {NVLINK_GBS} GB/s + {NCCL_LAT_US} us",
            "ranks": {}}
+    out["mode"] = "spatial shards" if args.spatial else "index shards"
     for G in args.ranks:
+        if args.spatial:
+            per_rank, rb = emulate_spatial(cfg, params, G, args.steps, args.warmup, flush)
+            recv, path = float(rb.max()), abi.BOIDS_PATH_GRID
+            ag_ms = 0.0 if G == 1 else (recv / (NVLINK_GBS * 1e9) * 1e3 + NCCL_LAT_US * 1e-3)
+            proj = float(per_rank.max()) + ag_ms
+            out["ranks"][G] = {"rank_ms_max": float(per_rank.max()), "rank_ms_min": float(per_rank.min()),
+                               "rank_path": path, "exchange_recv_bytes_max": int(recv), "exchange_ms_est": ag_ms,
+                               "projected_step_ms": proj, "projected_speedup_vs_1gpu": t1 / proj}
+            print(json.dumps({G: out["ranks"][G]}), flush=True)
+            continue
         per_rank, slice_bytes, path = emulate(cfg, params, G, args.steps, args.warmup, flush)
         recv = (G - 1) * slice_bytes
         ag_ms = 0.0 if G == 1 else (recv / (NVLINK_GBS * 1e9) * 1e3 + NCCL_LAT_US * 1e-3)
