@@ -13,10 +13,15 @@ a6 modification; a2 binning in grid mode), through the C ABI of libboids.so.
              before every timed step (the state of every config fits in L2).
 * e2e        the same metric through the public C ABI with HOST buffers: every
              step boids_set_state (H2D) + step + boids_get_state (D2H), wall clock.
-* roofline   the dominant kernel (the fused search kernel): algorithmic FP32
-             lane-ops per launch (8 per candidate pair) / its mean
-             launch duration (library-side CUDA events on the same stream),
+* roofline   the search kernel of the path the library reports it ran
+             (boids_info.last_path: k_sym_prep + k_sym, k_bound + k_scan, k_grid):
+             algorithmic FP32 lane-ops per launch (8 per evaluated pair,
+             DESIGN.md sec 5) / its mean launch duration (library-side CUDA
+             events on the handle's stream; inside the timed region, or with
+             --kernel-timing pass in a profiled pass of K steps right after it),
              against the FP32 SIMT peak 148 SMs x 128 lanes x sm_max_mhz.
+* update_roofline / update_standalone / binning_roofline  the update and
+             binning kernels against the measured HBM copy bandwidth.
 * cpu_baseline  the CPU oracle (oracle/, single thread) on a bounded sample of
              the same workload: full O(n) search + steer + modify for each sampled
              agent, extrapolated per agent-step (rank 0, N=1 only).
@@ -412,9 +417,10 @@ def main():
     b_ms, b_n = prof1["binning"]
     binning_roofline = None
     if b_n and grid:
-        # per agent: read pos4 (16) + write cell/rank (8) + read cell/rank (8) + read pos4 (16) + write the
-        # sorted record (16) + query permutation (4) + cell counts/starts (~2 x 4 per agent amortised)
-        per_agent = 76
+        # two binnings per step: candidates by cell -- read pos4 (16), write + read
+        # cell/rank (16), read pos4 (16), write the sorted record (16) -- and the owned queries by block --
+        # read pos4 (16), write + read cell/rank (16), write the permutation (4); counts amortised
+        per_agent = 100
         steps_binned = args.steps
         bb = per_agent * float(cfg.n) * steps_binned / (b_ms / 1e3) / 1e9
         binning_roofline = {"bound": "hbm", "kernel": "k_bin_count + scan + scatter (counting sort by cell)",
