@@ -363,7 +363,8 @@ def main():
                     abi.BOIDS_PATH_SCAN: "k_bound + k_scan (warm-step ordered-pair search)",
                     abi.BOIDS_PATH_THINK: "k_bound + k_scan over this step's thinkers (k_fused for never-searched ones)",
                     abi.BOIDS_PATH_FUSED: "k_fused (cold-step cluster kernel)",
-                    abi.BOIDS_PATH_SIMPLE: "k_search_simple (tiled search, thesis structure)"}
+                    abi.BOIDS_PATH_SIMPLE: "k_search_simple (tiled search, thesis structure)",
+                    abi.BOIDS_PATH_SMALL: "k_small (whole warm step in one kernel: search + merge + steer + modify)"}
     roofline = {"bound": "alu",
                 "kernel": kernel_names.get(path, f"path {path}"), "path": path,
                 "achieved": achieved, "peak": peak, "unit": "TFLOP/s", "frac": achieved / peak,

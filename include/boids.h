@@ -124,6 +124,7 @@ typedef struct boids_info_t {
 #define BOIDS_PATH_GRID 3    /* grid mode: binning + k_grid (+ k_grid_far) */
 #define BOIDS_PATH_SIMPLE 4  /* BOIDS_KERNEL_SIMPLE: k_search_simple + k_update */
 #define BOIDS_PATH_THINK 5   /* brute force, think mode: thinkers on k_bound + k_scan (cold ones k_fused) */
+#define BOIDS_PATH_SMALL 6   /* warm step of a small single-rank flock: k_small (ordered pairs n x n, one kernel) */
 
 #define BOIDS_KERNEL_FUSED 0   /* default: cold steps run the fused cluster kernel (search + merge +
                                   steer + modify); warm steps (previous lists known) run the
@@ -156,6 +157,10 @@ typedef struct boids_info_t {
                                        B200: the graph saves host enqueue time but a step of 4-6 dependent
                                        kernels behind a cold L2 runs 5-6 us slower as a graph, C1-C3).
                                        Results are identical either way. */
+#define BOIDS_OPT_SMALL 11          /* 1 (default): warm brute-force steps of a single-rank handle with
+                                       n < 8192 run as one kernel (k_small: P threads per query scan all
+                                       agents, merge their top-8 lists, steer and modify); 0: the
+                                       k_bound + k_scan + k_select1 + k_route chain.  Results identical. */
 #define BOIDS_OPT_PHASES 5          /* diagnostics: value = max CTAs; the fused kernel records per-CTA
                                        %globaltimer stamps (read with boids_get_phases); 0 = off */
 

@@ -23,6 +23,7 @@ BOIDS_STEER_THESIS, BOIDS_STEER_OPENSTEER = 0, 1
 BOIDS_KERNEL_FUSED, BOIDS_KERNEL_SIMPLE, BOIDS_KERNEL_CLUSTER = 0, 1, 2
 BOIDS_OPT_RECORD_STEERING, BOIDS_OPT_KERNEL, BOIDS_OPT_PROFILE, BOIDS_OPT_CLUSTER, BOIDS_OPT_PHASES = 1, 2, 3, 4, 5
 BOIDS_OPT_RESORT, BOIDS_OPT_VOTE_U, BOIDS_OPT_SYMMETRIC, BOIDS_OPT_BALANCE, BOIDS_OPT_GRAPH = 6, 7, 8, 9, 10
+BOIDS_OPT_SMALL = 11
 BOIDS_PROF_CLASSES = 5
 PROF_NAMES = ("fused_or_search", "update", "binning", "grid_search", "route")
 
@@ -39,7 +40,8 @@ EXPORTS = (
 )
 SPATIAL_HALO_F4, SPATIAL_MIG_F4 = 2, 8  # float4 per halo / migrant record (include/boids.h)
 # boids_info_t.last_path
-BOIDS_PATH_FUSED, BOIDS_PATH_SCAN, BOIDS_PATH_SYM, BOIDS_PATH_GRID, BOIDS_PATH_SIMPLE, BOIDS_PATH_THINK = range(6)
+BOIDS_PATH_FUSED, BOIDS_PATH_SCAN, BOIDS_PATH_SYM, BOIDS_PATH_GRID, BOIDS_PATH_SIMPLE, BOIDS_PATH_THINK, \
+    BOIDS_PATH_SMALL = range(7)
 
 
 class BoidsError(RuntimeError):

@@ -80,6 +80,7 @@ struct boids_ctx {
   unsigned long long* rpart = nullptr;    // k_route partial lists [m][16][8]
   int32_t* rbcount = nullptr;             // k_route parts done per routed agent [m]
   bool symmetric = true;                  // BOIDS_OPT_SYMMETRIC
+  bool use_small = true;                  // BOIDS_OPT_SMALL
   bool balance = true;                    // BOIDS_OPT_BALANCE: k_sym split from the last launch's CTA times
   int32_t* pcnt = nullptr;
   unsigned long long* phase = nullptr;  // diagnostics (BOIDS_OPT_PHASES): per-CTA timestamps
@@ -560,10 +561,16 @@ int one_step(boids_ctx* c, float dt) {
     if ((rc = launch(c, 0, [&] { return launch_search_simple(a, c->stream); }))) return rc;
     if ((rc = launch(c, 1, [&] { return launch_update(a, c->stream); }))) return rc;
   } else {
+    // small flocks: the whole warm step in one kernel (k_small.cu), no spatial order needed
+    const bool small = warm_path && !think && !c->shard && c->use_small && c->nloc < small_max();
+    if (small) {
+      c->last_path = BOIDS_PATH_SMALL;
+      if ((rc = launch(c, 0, [&] { return launch_small(a, c->stream); }))) return rc;
+    }
     // a2: spatial (Morton) order of the owned queries, so the 128 queries of a
     // warp are spatially coherent.  It is only a permutation of the work (results
     // never depend on it), so it is refreshed every resort_every steps.
-    if (c->since_sort < 0 || c->since_sort >= c->resort_every) {
+    if (!small && (c->since_sort < 0 || c->since_sort >= c->resort_every)) {
       if ((rc = launch(c, 2, [&] {
              return launch_bin(a.full, c->m, a.sdiv, c->lo, c->nloc, c->loc_grid, c->cellrank, c->bcnt, c->bstart,
                                nullptr, c->qperm, (int)c->lo, c->stream, nullptr);
@@ -572,8 +579,10 @@ int one_step(boids_ctx* c, float dt) {
       c->since_sort = 0;
       c->steps_sorted++;
     }
-    c->since_sort++;
-    if (think) {
+    if (!small) c->since_sort++;
+    if (small) {
+      // done above
+    } else if (think) {
       // this step's thinkers, in spatial order, split into never-searched (cold)
       // and warm-bounded ones
       c->last_path = BOIDS_PATH_THINK;
@@ -1007,6 +1016,9 @@ BOIDS_API int boids_set_option(boids_ctx* c, int32_t opt, int64_t v) {
   switch (opt) {
     case BOIDS_OPT_GRAPH:
       c->use_graphs = v != 0;
+      return BOIDS_OK;
+    case BOIDS_OPT_SMALL:
+      c->use_small = v != 0;
       return BOIDS_OK;
     case BOIDS_OPT_RECORD_STEERING:
       if (v && !c->force4) CK(cudaMalloc((void**)&c->force4, c->m * sizeof(float4)));

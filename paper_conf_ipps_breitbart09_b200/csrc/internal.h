@@ -218,7 +218,10 @@ cudaError_t launch_fused(const StepArgs& a, int cluster, cudaStream_t s);
 cudaError_t launch_warm_scan(const StepArgs& a, cudaStream_t s);
 cudaError_t launch_grid(const StepArgs& a, const GridArgs& g, cudaStream_t s);
 cudaError_t launch_grid_far(const StepArgs& a, const GridArgs& g, cudaStream_t s);
-int grid_chunk(int64_t nq);  // queries per grid work item for nq queries
+int grid_chunk(int64_t nq);
+// k_small.cu: the whole warm brute-force step in one kernel for single-rank handles with n < small_max()
+int small_max();
+cudaError_t launch_small(const StepArgs& a, cudaStream_t s);  // queries per grid work item for nq queries
 // pdl: launch k_select1 as a programmatic dependent of the scan.  Measured: a
 // gain after k_scan (C1 30 -> 25 us/step), a loss after k_sym (C3 97 -> 121).
 cudaError_t launch_warm_select(const StepArgs& a, cudaStream_t s, bool pdl = true);

@@ -522,3 +522,26 @@ def test_graph_steps_match_eager_and_oracle(pk, orc, mode, n, steps):
         assert fg.info().graph_launches - g0 == 5
         cls = "grid_search" if mode else "fused_or_search"
         assert prof[cls][1] == 5 and prof[cls][0] > 0
+
+
+@pytest.mark.parametrize("small", [1, 0])
+@pytest.mark.parametrize("n,steps", [(1, 3), (2, 3), (7, 4), (100, 5), (1024, 12), (3000, 6), (8191, 4)])
+def test_small_step_kernel(pk, orc, n, steps, small):
+    """Warm steps of small single-rank flocks run as one kernel (k_small,
+    BOIDS_OPT_SMALL = 1, the default below 8192 agents) or as the k_bound +
+    k_scan + k_select1 + k_route chain (0): both bit-identical to the oracle's
+    trajectory, lists included (ragged sizes, 16 and 8 threads per query)."""
+    from paper_conf_ipps_breitbart09_b200 import abi
+
+    p = pk.boids_default_params(init_mode=1, world_radius=max(4.0, 20.0 * (n / 8192) ** (1 / 3)))
+    op = _oparams(orc, p)
+    with pk.Flock(n, p, seed=5) as f:
+        abi.boids_set_option(f.h, abi.BOIDS_OPT_SMALL, small)
+        o = orc.init(n, op, seed=5)
+        for t in range(steps):
+            o, o_idx, _, _ = orc.step(o, DT, op)
+            f.step(DT, 1)
+            np.testing.assert_array_equal(f.neighbors()[0], o_idx, err_msg=f"step {t}")
+            assert bitexact(f.state(), o), f"step {t}"
+        want = abi.BOIDS_PATH_SMALL if small else abi.BOIDS_PATH_SCAN
+        assert f.info().last_path == want
