@@ -178,6 +178,36 @@ BOIDS_API int boids_create(int64_t n, const boids_params* p, uint64_t seed, boid
 BOIDS_API int boids_create_shard(int64_t n, const boids_params* p, uint64_t seed, int32_t rank,
                        int32_t world, boids_ctx** out);
 
+/* ---- Sym-shards: the unordered-pair triangle of a brute-force flock split over
+ * index shards (boids_create_shard handles, search_mode BOIDS_BRUTE, think_every 1;
+ * the search is Listing 5.2's brute force, multiple devices are the thesis's future
+ * work).
+ * A single-GPU handle evaluates every unordered pair once (k_sym: d2 is bitwise
+ * symmetric); plain index shards evaluate n/G x n ordered pairs each.  Here the
+ * ranks share the n(n-1)/2 pairs of ONE global order instead.  A warm step (the
+ * first step of a handle runs boids_step_shard) is, after the usual all-gather of
+ * the [pos4 | fwd4] slices:
+ *   boids_symshard_prep(h)        this rank's agents' warm limits -> lim_send (m floats)
+ *   all-gather lim_send -> lim_full (world * m floats, rank g's slice at g * m)
+ *   boids_symshard_search(h)      the same deterministic global Morton order on every
+ *                                 rank, this rank's 1/world share of the triangle: hits
+ *                                 (u64 keys) for ANY agent j into hits[j * hits_cap ...],
+ *                                 counts hitcnt[j] (world * m slots, agent j at slot j)
+ *   all-to-all: block d of hits / hitcnt (slots [d*m, (d+1)*m)) to rank d, received
+ *                                 from rank s into recv / rcnt block s
+ *   boids_symshard_finish(h, dt)  this rank's agents: the hits of all world blocks ->
+ *                                 top-7, steering, modification into the send slice.
+ * hits_cap (16) bounds one agent's hits per rank segment; an agent with more in any
+ * segment is searched whole by its owner in finish (exact either way).
+ * Lists and states are those of the single-GPU step.  Asynchronous; EINVAL if the
+ * handle is not a warm brute-force shard handle. */
+BOIDS_API int boids_symshard_prep(boids_ctx* ctx);
+BOIDS_API int boids_symshard_search(boids_ctx* ctx);
+BOIDS_API int boids_symshard_finish(boids_ctx* ctx, float dt);
+/* Device buffers of the two exchanges (allocated on first use). */
+BOIDS_API int boids_symshard_buffers(boids_ctx* ctx, void** lim_send, void** lim_full, void** hits, void** hitcnt,
+                                     void** recv, void** rcnt, int32_t* hits_cap);
+
 /* ---- Spatial decomposition (future work of the thesis) ----
  * A spatial shard of a grid-mode flock (search_mode BOIDS_GRID, think_every 1):
  * rank `rank` of `world` OWNS the agents whose search-grid cell layer z lies in

@@ -37,6 +37,7 @@ EXPORTS = (
     "boids_get_accel", "boids_set_accel", "boids_bench_update",
     "boids_create_spatial", "boids_step_spatial", "boids_spatial_outbox", "boids_spatial_inbox",
     "boids_spatial_unpack", "boids_spatial_owned", "boids_spatial_bounds",
+    "boids_symshard_prep", "boids_symshard_search", "boids_symshard_finish", "boids_symshard_buffers",
 )
 SPATIAL_HALO_F4, SPATIAL_MIG_F4 = 2, 8  # float4 per halo / migrant record (include/boids.h)
 # boids_info_t.last_path
@@ -117,6 +118,10 @@ def load(path: str = LIB_PATH):
         "boids_spatial_unpack": (C.c_int, [vp, i64, i64]),
         "boids_spatial_owned": (C.c_int, [vp, C.POINTER(C.c_uint8)]),
         "boids_spatial_bounds": (C.c_int, [vp, ip, ip]),
+        "boids_symshard_prep": (C.c_int, [vp]),
+        "boids_symshard_search": (C.c_int, [vp]),
+        "boids_symshard_finish": (C.c_int, [vp, f32]),
+        "boids_symshard_buffers": (C.c_int, [vp] + [C.POINTER(vp)] * 6 + [ip]),
         "boids_destroy": (None, [vp]),
         "boids_last_error": (C.c_char_p, []),
     }
@@ -341,6 +346,29 @@ def boids_spatial_bounds(h: int, world: int):
     r = np.zeros(1, np.int32)
     _check(load().boids_spatial_bounds(h, _iptr(zb), _iptr(r)))
     return zb, int(r[0])
+
+
+def boids_symshard_prep(h: int):
+    _check(load().boids_symshard_prep(h))
+
+
+def boids_symshard_search(h: int):
+    _check(load().boids_symshard_search(h))
+
+
+def boids_symshard_finish(h: int, dt: float):
+    _check(load().boids_symshard_finish(h, C.c_float(dt)))
+
+
+def boids_symshard_buffers(h: int):
+    """dict of device pointers: lim_send, lim_full, hits, hitcnt, recv, rcnt; and hits_cap."""
+    ps = [C.c_void_p() for _ in range(6)]
+    cap = np.zeros(1, np.int32)
+    _check(load().boids_symshard_buffers(h, *[C.byref(x) for x in ps], _iptr(cap)))
+    names = ("lim_send", "lim_full", "hits", "hitcnt", "recv", "rcnt")
+    out = {k: v.value for k, v in zip(names, ps)}
+    out["hits_cap"] = int(cap[0])
+    return out
 
 
 def boids_destroy(h: int):

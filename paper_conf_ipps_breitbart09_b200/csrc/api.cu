@@ -137,6 +137,13 @@ struct boids_ctx {
   int64_t kept_bound = 0;                  // host upper bound of *nkept
   int64_t last_nh = 0;                     // halo records applied by the last unpack (cleared next pack)
   int* sp_overflow = nullptr;
+  // sym-shards (an index-sharded brute-force handle stepping its share of the global
+  // unordered-pair triangle; k_sym.cu "Sym-shards"): lazily allocated
+  float *ss_lim_send = nullptr, *ss_lim_full = nullptr;
+  unsigned long long *ss_hits = nullptr, *ss_recv = nullptr;
+  int32_t *ss_hitcnt = nullptr, *ss_rcnt = nullptr, *ss_gperm = nullptr, *ss_gbcnt = nullptr, *ss_gbstart = nullptr;
+  float4* ss_spos = nullptr;
+  int64_t ss_since_sort = -1;
   bool dry = false;
   bool capturing = false;  // one_step runs inside graph_step's stream capture
   bool use_graphs = false;  // BOIDS_OPT_GRAPH
@@ -238,6 +245,16 @@ void free_ctx(boids_ctx* c) {
   cudaFree(c->twarm);
   cudaFree(c->tcnt);
   cudaFree(c->ocheck);
+  cudaFree(c->ss_lim_send);
+  cudaFree(c->ss_lim_full);
+  cudaFree(c->ss_hits);
+  cudaFree(c->ss_recv);
+  cudaFree(c->ss_hitcnt);
+  cudaFree(c->ss_rcnt);
+  cudaFree(c->ss_gperm);
+  cudaFree(c->ss_gbcnt);
+  cudaFree(c->ss_gbstart);
+  cudaFree(c->ss_spos);
   cudaFree(c->zb);
   cudaFree(c->own);
   cudaFree(c->halo_out);
@@ -839,6 +856,134 @@ BOIDS_API int boids_create(int64_t n, const boids_params* p, uint64_t seed, boid
 BOIDS_API int boids_create_shard(int64_t n, const boids_params* p, uint64_t seed, int32_t rank,
                        int32_t world, boids_ctx** out) {
   return create_impl(n, p, seed, rank, world, true, out);
+}
+
+// ---- sym-shards: boids_symshard_prep / _search / _finish (include/boids.h) ----
+static int ss_check(boids_ctx* c) {
+  if (!c) return fail(BOIDS_EINVAL, "NULL handle");
+  if (!c->shard || c->p.search_mode != BOIDS_BRUTE || c->p.think_every != 1 || c->kernel != BOIDS_KERNEL_FUSED)
+    return fail(BOIDS_EINVAL, "sym-shards: a brute-force shard handle (think_every 1, default kernels)");
+  if (!c->warm) return fail(BOIDS_EINVAL, "sym-shards step warm handles: run the first step with boids_step_shard");
+  return BOIDS_OK;
+}
+
+static int ss_alloc(boids_ctx* c) {
+  if (c->ss_lim_send) return BOIDS_OK;
+  const int64_t slots = (int64_t)c->world * c->m;
+  const size_t hcap = (size_t)slots * SS_HITS * sizeof(unsigned long long);
+  cudaError_t e;
+  if ((e = cudaMalloc((void**)&c->ss_lim_send, c->m * sizeof(float))) != cudaSuccess ||
+      (e = cudaMalloc((void**)&c->ss_lim_full, slots * sizeof(float))) != cudaSuccess ||
+      (e = cudaMalloc((void**)&c->ss_hits, hcap)) != cudaSuccess ||
+      (e = cudaMalloc((void**)&c->ss_recv, hcap)) != cudaSuccess ||
+      (e = cudaMalloc((void**)&c->ss_hitcnt, slots * sizeof(int32_t))) != cudaSuccess ||
+      (e = cudaMalloc((void**)&c->ss_rcnt, slots * sizeof(int32_t))) != cudaSuccess ||
+      (e = cudaMalloc((void**)&c->ss_gperm, slots * sizeof(int32_t))) != cudaSuccess ||
+      (e = cudaMalloc((void**)&c->ss_gbcnt, c->loc_grid.cells * sizeof(int32_t))) != cudaSuccess ||
+      (e = cudaMalloc((void**)&c->ss_gbstart, (c->loc_grid.cells + 1) * sizeof(int32_t))) != cudaSuccess ||
+      (e = cudaMalloc((void**)&c->ss_spos, slots * sizeof(float4))) != cudaSuccess ||
+      (!c->sym_sp && (e = cudaMalloc((void**)&c->sym_sp, sym_capacity(slots) * sizeof(float4))) != cudaSuccess) ||
+      (!c->sym_idx && (e = cudaMalloc((void**)&c->sym_idx, sym_capacity(slots) * sizeof(int32_t))) != cudaSuccess) ||
+      (!c->sym_fb &&
+       (e = cudaMalloc((void**)&c->sym_fb, (2 * SYM_FB_LEN + SYM_FB_MAX_CTAS + 1) * sizeof(long long))) != cudaSuccess)) {
+    (void)cudaGetLastError();
+    return fail(BOIDS_ENOMEM, std::string("sym-shard buffers: ") + cudaGetErrorString(e));
+  }
+  CK(cudaMemsetAsync(c->ss_gbcnt, 0, c->loc_grid.cells * sizeof(int32_t), c->stream));
+  CK(cudaMemsetAsync(c->sym_fb, 0, 2 * SYM_FB_LEN * sizeof(long long), c->stream));
+  CK(cudaMemsetAsync(c->ss_lim_full, 0, slots * sizeof(float), c->stream));
+  return BOIDS_OK;
+}
+
+BOIDS_API int boids_symshard_prep(boids_ctx* c) {
+  int rc = ss_check(c);
+  if (rc) return rc;
+  DeviceGuard g(c->dev);
+  if ((rc = ss_alloc(c))) return rc;
+  StepArgs a = make_args(c, 0.f);
+  a.routed = c->routed;
+  // this rank's Morton query order (the window bound looks agents up in it)
+  if (c->since_sort < 0 || c->since_sort >= c->resort_every) {
+    if ((rc = launch(c, 2, [&] {
+           return launch_bin(a.full, c->m, a.sdiv, c->lo, c->nloc, c->loc_grid, c->cellrank, c->bcnt, c->bstart,
+                             nullptr, c->qperm, (int)c->lo, c->stream, nullptr);
+         }, 3)))
+      return rc;
+    c->since_sort = 0;
+    c->steps_sorted++;
+  }
+  c->since_sort++;
+  CK(cudaMemsetAsync(c->sym_rcount, 0, sizeof(int32_t), c->stream));
+  return launch(c, 0, [&] { return launch_ss_lim(a, c->ss_lim_send, c->stream); });
+}
+
+BOIDS_API int boids_symshard_search(boids_ctx* c) {
+  int rc = ss_check(c);
+  if (rc) return rc;
+  if (!c->ss_lim_send) return fail(BOIDS_EINVAL, "boids_symshard_prep first");
+  DeviceGuard g(c->dev);
+  StepArgs a = make_args(c, 0.f);
+  const int64_t slots = (int64_t)c->world * c->m;
+  // the global Morton order, identical on every rank (cells sorted by index)
+  if (c->ss_since_sort < 0 || c->ss_since_sort >= c->resort_every) {
+    if ((rc = launch(c, 2, [&] {
+           cudaError_t e = launch_bin(a.full, c->m, a.sdiv, 0, slots, c->loc_grid, c->cellrank, c->ss_gbcnt,
+                                      c->ss_gbstart, c->ss_spos, c->ss_gperm, 0, c->stream, nullptr);
+           if (e == cudaSuccess) e = launch_ss_cellsort(c->ss_gperm, c->ss_gbstart, c->loc_grid.cells, c->stream);
+           return e;
+         }, 4)))
+      return rc;
+    c->ss_since_sort = 0;
+  }
+  c->ss_since_sort++;
+  CK(cudaMemsetAsync(c->ss_hitcnt, 0, slots * sizeof(int32_t), c->stream));
+  StepArgs as = a;
+  as.hits = c->ss_hits;
+  as.hitcnt = c->ss_hitcnt;
+  as.hits_cap = SS_HITS;
+  long long* fb_prev = c->sym_fb + (c->sym_fb_par ^ 1) * SYM_FB_LEN;
+  long long* fb_cur = c->sym_fb + c->sym_fb_par * SYM_FB_LEN;
+  c->sym_fb_par ^= 1;
+  return launch(c, 0, [&] {
+    return launch_ss_search(as, c->ss_gperm, c->n, c->ss_lim_full, c->sym_sp, c->sym_idx, c->balance ? fb_prev : nullptr,
+                            fb_cur, c->sym_fb + 2 * SYM_FB_LEN, c->rank, c->world, c->stream);
+  }, 2);
+}
+
+BOIDS_API int boids_symshard_finish(boids_ctx* c, float dt) {
+  int rc = ss_check(c);
+  if (rc) return rc;
+  if ((rc = check_dt(dt))) return rc;
+  if (!c->ss_lim_send) return fail(BOIDS_EINVAL, "boids_symshard_prep first");
+  DeviceGuard g(c->dev);
+  StepArgs a = make_args(c, dt);
+  a.routed = c->routed;
+  a.hits_cap = SS_HITS;
+  if ((rc = launch(c, 1, [&] { return launch_ss_select(a, c->ss_recv, c->ss_rcnt, c->world, c->stream); }))) return rc;
+  if ((rc = launch(c, 4, [&] { return launch_route(a, c->stream); }))) return rc;
+  c->last_path = BOIDS_PATH_SYM;
+  c->warm = true;
+  c->steering_valid = c->record_steering;
+  c->step_index++;
+  c->steps_taken++;
+  return BOIDS_OK;
+}
+
+BOIDS_API int boids_symshard_buffers(boids_ctx* c, void** lim_send, void** lim_full, void** hits, void** hitcnt,
+                                     void** recv, void** rcnt, int32_t* hits_cap) {
+  if (!c) return fail(BOIDS_EINVAL, "NULL handle");
+  if (!c->shard || c->p.search_mode != BOIDS_BRUTE) return fail(BOIDS_EINVAL, "not a brute-force shard handle");
+  DeviceGuard g(c->dev);
+  int rc = ss_alloc(c);
+  if (rc) return rc;
+  if (lim_send) *lim_send = c->ss_lim_send;
+  if (lim_full) *lim_full = c->ss_lim_full;
+  if (hits) *hits = c->ss_hits;
+  if (hitcnt) *hitcnt = c->ss_hitcnt;
+  if (recv) *recv = c->ss_recv;
+  if (rcnt) *rcnt = c->ss_rcnt;
+  if (hits_cap) *hits_cap = SS_HITS;
+  return BOIDS_OK;
 }
 
 BOIDS_API int boids_create_spatial(int64_t n, const boids_params* p, uint64_t seed, int32_t rank, int32_t world,

@@ -10,6 +10,10 @@ namespace boids {
 
 constexpr int TILE = 256;  // slice granularity (agents); every slice m is a multiple
 constexpr int HITS = 48;   // warm path: hit-buffer slots per agent (more -> full re-search)
+// sym-shards: hit slots per agent per rank segment; the blocks cross ranks in an
+// all-to-all of fixed-size pieces, so the cap sets its payload (a segment holds a
+// 1/G share of an agent's ~8-12 hits; more in one segment -> full re-search)
+constexpr int SS_HITS = 16;
 constexpr int HITS_THINK = 128;  // ... in think mode (bounds from lists up to k steps old are looser)
 constexpr int PSLOTS = 16; // warm path: partial top-7 lists per unbounded agent
 
@@ -234,6 +238,14 @@ constexpr int SYM_FB_LEN = 2 + 3 * SYM_FB_MAX_CTAS;
 cudaError_t launch_sym_scan(const StepArgs& a, float4* sp, int* sidx, const long long* fb_prev, long long* fb_cur,
                             long long* splits, cudaStream_t s);
 cudaError_t launch_route(const StepArgs& a, cudaStream_t s);
+// sym-shards (k_sym.cu): the unordered-pair triangle split over index-sharded ranks
+cudaError_t launch_ss_lim(const StepArgs& a, float* lim_send, cudaStream_t s);
+cudaError_t launch_ss_cellsort(int* perm, const int* start, int cells, cudaStream_t s);
+cudaError_t launch_ss_search(const StepArgs& a, const int* gperm, int64_t nsorted, const float* lim_full, float4* sp,
+                             int* sidx, const long long* fb_prev, long long* fb_cur, long long* splits, int rank,
+                             int world, cudaStream_t s);
+cudaError_t launch_ss_select(const StepArgs& a, const unsigned long long* recv, const int* rcnt, int world,
+                             cudaStream_t s);
 int fused_auto_cluster(int64_t n_pad_total, int64_t nloc, int sm_count);
 // spatial shards (k_spatial.cu)
 int spatial_halo_f4();

@@ -187,13 +187,21 @@ __device__ __forceinline__ int64_t sym_split(int64_t i, int64_t grid, int64_t np
 // k_sym_prep's block 0 computes all G + 1 boundaries into `splits` (one
 // thread per boundary, binary search over a shared-memory prefix of the costs),
 // off k_sym's critical path: k_sym's CTAs then read their two boundaries.
-__device__ void compute_splits(const long long* __restrict__ fb, int G, int64_t total, int64_t npad, int64_t qb,
-                               int wd4, long long* __restrict__ splits) {
+// [lo, hi): the item sub-range this launch covers (the whole triangle on a single
+// GPU; a rank's share of it with sym-shards, k_ss_*); the record's "total" is
+// the whole triangle's length, its CTA ranges are absolute item positions, and it
+// is used only if its first and last CTA ranges start at lo and end at hi.
+__device__ void compute_splits(const long long* __restrict__ fb, int G, int64_t lo, int64_t hi, int64_t npad,
+                               int64_t qb, int wd4, long long* __restrict__ splits) {
   __shared__ double pre[SYM_FB_MAX_CTAS];
   __shared__ double wsum[32];
   __shared__ int ok;
+  const int64_t total = hi - lo;
+  const bool whole = lo == 0 && hi == sym_prefix(npad / qb, npad, qb);
   const int tid = threadIdx.x, nt = blockDim.x, lane = tid & 31, warp = tid >> 5;
-  if (tid == 0) ok = fb != nullptr && G <= SYM_FB_MAX_CTAS && fb[0] == G && fb[1] == total;
+  if (tid == 0)
+    ok = fb != nullptr && G <= SYM_FB_MAX_CTAS && fb[0] == G && fb[1] == sym_prefix(npad / qb, npad, qb) &&
+         fb[2] == lo && fb[3 * G] == hi;
   __syncthreads();
   if (ok) {  // inclusive prefix of the measured CTA costs (block scan over per-thread chunks)
     const int per = (G + nt - 1) / nt, j0 = min(G, tid * per), j1 = min(G, j0 + per);
@@ -222,23 +230,25 @@ __device__ void compute_splits(const long long* __restrict__ fb, int G, int64_t 
   for (int k = tid; k <= G; k += nt) {
     int64_t x;
     if (k == 0) {
-      x = 0;
+      x = lo;
     } else if (k == G) {
-      x = total;
+      x = hi;
     } else if (ok) {
       const double c = T * (double)k / (double)G;
-      int lo = 0, hi = G - 1;  // first j with pre[j] > c
-      while (lo < hi) {
-        const int mid = (lo + hi) >> 1;
-        if (pre[mid] > c) hi = mid; else lo = mid + 1;
+      int jl = 0, jh = G - 1;  // first j with pre[j] > c
+      while (jl < jh) {
+        const int mid = (jl + jh) >> 1;
+        if (pre[mid] > c) jh = mid; else jl = mid + 1;
       }
-      const double t = (double)fb[4 + 3 * lo], cum = pre[lo] - t;
-      const int64_t a0 = fb[2 + 3 * lo], a1 = fb[3 + 3 * lo];
+      const double t = (double)fb[4 + 3 * jl], cum = pre[jl] - t;
+      const int64_t a0 = fb[2 + 3 * jl], a1 = fb[3 + 3 * jl];
       x = t > 0.0 ? a0 + (int64_t)((c - cum) / t * (double)(a1 - a0)) : a0;
       x = x / UG * UG;
-      x = x < 0 ? 0 : (x > total ? total : x);
-    } else {
+      x = x < lo ? lo : (x > hi ? hi : x);
+    } else if (whole) {
       x = sym_split(k, G, npad, qb, wd4);
+    } else {  // a sub-range without a record: equal item shares
+      x = lo + (int64_t)((__int128)total * k / G) / UG * UG;
     }
     splits[k] = x;
   }
@@ -524,7 +534,7 @@ __global__ void __launch_bounds__(NTS, NTS == 128 ? 4 : (NTS == 256 ? 2 : 1))
       fb_cur[4 + 3 * blockIdx.x] = clock64() - s_cstart;
       if (blockIdx.x == 0) {
         fb_cur[0] = gridDim.x;
-        fb_cur[1] = total;
+        fb_cur[1] = total;  // the whole triangle's length (the record's CTA 0 range starts the covered sub-range)
       }
     }
   }
@@ -662,7 +672,7 @@ __global__ void __launch_bounds__(256) k_sym_prep(StepArgs a, float* __restrict_
   pdl_trigger();  // k_sym may be scheduled now; it waits for this grid before reading sp
   span_begin(a, SPAN_SLOT0 + 0);
   if (blockIdx.x == gridDim.x - 1)  // the last block (fewest real agents) also cuts k_sym's work
-    compute_splits(fb_prev, G, sym_prefix(npad / qb, npad, qb), npad, qb, wd4, splits);
+    compute_splits(fb_prev, G, 0, sym_prefix(npad / qb, npad, qb), npad, qb, wd4, splits);
   sym_prep_body(a, spf, cap, sidx, npad);
   span_end(a, SPAN_SLOT0 + 0);
 }
@@ -819,7 +829,172 @@ cudaError_t sym_with(const StepArgs& a, float4* sp, int* sidx, const long long* 
                     (const int*)sidx, npad, (const long long*)splits, fb_cur);
 }
 
+// ---------------------------------------------------------------------------
+// Sym-shards: the unordered-pair triangle of the whole flock split over the
+// ranks of an index-sharded (boids_create_shard) brute-force flock.
+//   prep    (k_ss_lim)      each rank: the warm limits of its own agents (as
+//                           k_sym_prep: t0, window bound, routing) -> its slice
+//   [all-gather of the limits]
+//   search  (k_ss_spbuild,  every rank: the same deterministic global Morton
+//            k_sym)         order (binning + a per-cell sort by index), the
+//                           agents as SoA with their limits, and k_sym over this
+//                           rank's share [T g / G, T (g + 1) / G) of the triangle:
+//                           hits for ANY agent into full-size buffers
+//   [all-to-all: the hits of rank h's agents to rank h]
+//   finish  (k_ss_select)   each rank: its agents' hits from all G segments ->
+//                           top-7, steering, modification (k_route as usual)
+// Every unordered pair is evaluated exactly once over all ranks (the ranks'
+// shares tile the triangle of ONE order), so the hit set of every agent is the
+// single-GPU one: identical lists.
+__global__ void __launch_bounds__(256) k_ss_lim(StepArgs a, float* __restrict__ lim_send) {
+  const int64_t i = (int64_t)blockIdx.x * 256 + threadIdx.x;
+  if (i >= a.m) return;
+  if (i >= a.nloc) {
+    lim_send[i] = -1.f;
+    return;
+  }
+  const float r2 = __fmul_rn(a.p.search_radius, a.p.search_radius);
+  const float r2_in = __uint_as_float(__float_as_uint(r2) - 1u);
+  const float4 me = __ldg(pos_of(a.full, a.m, a.sdiv, a.lo + i));
+  int c = 0;
+  const float t0 = sym_t0(a, i, me, c);
+  float lim = fminf(r2_in, t0);
+  if (t0 > r2_in) lim = fminf(lim, window_bound(a, (int)i, me));
+  if (c == 7 && lim > r2_in && a.rlist) {  // unbounded (a wrap): k_route searches it whole
+    a.rlist[atomicAdd(a.rcount, 1)] = (int)i;
+    a.routed[i] = 1;
+    if (a.stats) atomicAdd(a.stats + 2, 1ull);
+    lim = -1.f;
+  }
+  lim_send[i] = lim;
+}
+
+// The binning's order inside a cell follows its atomics: sort every cell's
+// entries by agent index, so every rank holds the same global order.
+__global__ void k_ss_cellsort(int* __restrict__ perm, const int* __restrict__ start, int cells) {
+  const int c = blockIdx.x * blockDim.x + threadIdx.x;
+  if (c >= cells) return;
+  const int lo = start[c], hi = start[c + 1];
+  for (int i = lo + 1; i < hi; ++i) {
+    const int v = perm[i];
+    int k = i - 1;
+    while (k >= lo && perm[k] > v) {
+      perm[k + 1] = perm[k];
+      --k;
+    }
+    perm[k + 1] = v;
+  }
+}
+
+// SoA of the globally sorted agents with their gathered limits (phantom slots
+// beyond n: NaN, limit -1); the last block also cuts this rank's item share.
+__global__ void __launch_bounds__(256) k_ss_spbuild(StepArgs a, const int* __restrict__ gperm, int64_t nsorted,
+                                                    const float* __restrict__ lim_full, float* __restrict__ spf,
+                                                    int64_t cap, int* __restrict__ sidx, int64_t npad, int64_t qb,
+                                                    int G, int64_t lo, int64_t hi, int wd4,
+                                                    const long long* __restrict__ fb_prev,
+                                                    long long* __restrict__ splits) {
+  pdl_trigger();
+  if (blockIdx.x == gridDim.x - 1) compute_splits(fb_prev, G, lo, hi, npad, qb, wd4, splits);
+  const int64_t p = (int64_t)blockIdx.x * 256 + threadIdx.x;
+  if (p >= npad) return;
+  if (p >= nsorted) {
+    const float nan = __int_as_float(0x7fc00000);
+    spf[p] = nan;
+    spf[cap + p] = nan;
+    spf[2 * cap + p] = nan;
+    spf[3 * cap + p] = -1.f;
+    sidx[p] = -1;
+    return;
+  }
+  const int j = __ldg(gperm + p);
+  const float4 q = __ldg(pos_of(a.full, a.m, a.sdiv, j));
+  spf[p] = q.x;
+  spf[cap + p] = q.y;
+  spf[2 * cap + p] = q.z;
+  spf[3 * cap + p] = __ldg(lim_full + j);  // agent j's limit, computed by its owner
+  sidx[p] = j;
+}
+
+// An owned agent's hits from the G ranks' segments -> exact top-7 (+ 8th),
+// steering, modification (k_select1's work over G hit buffers).
+__global__ void __launch_bounds__(128) k_ss_select(StepArgs a, const key_t* __restrict__ recv,
+                                                   const int* __restrict__ rcnt, int world) {
+  pdl_wait();
+  const int64_t qi = (int64_t)blockIdx.x * 128 + threadIdx.x;
+  if (qi >= a.nloc) return;
+  if (a.routed[qi]) {  // routed by k_ss_lim: finished by k_route
+    a.routed[qi] = 0;
+    a.nbr8[qi] = -1;
+    return;
+  }
+  bool over = false;
+  for (int sg = 0; sg < world; ++sg) over |= rcnt[(int64_t)sg * a.m + qi] > a.hits_cap;
+  if (over) {  // a rank's buffer for this agent overflowed: searched whole by k_route
+    if (a.stats) atomicAdd(a.stats + 2, 1ull);
+    a.rlist[atomicAdd(a.rcount, 1)] = (int)qi;
+    a.nbr8[qi] = -1;
+    return;
+  }
+  key_t L[8];
+#pragma unroll
+  for (int t = 0; t < 8; ++t) L[t] = KEY_EMPTY;
+  for (int sg = 0; sg < world; ++sg) {
+    const int c = rcnt[(int64_t)sg * a.m + qi];
+    const key_t* h = recv + ((int64_t)sg * a.m + qi) * a.hits_cap;
+    for (int k = 0; k < c; ++k) insert8(L, h[k]);
+  }
+  a.nbr8[qi] = L[7] == KEY_EMPTY ? -1 : key_idx(L[7]);
+  key_t A[7];
+#pragma unroll
+  for (int t = 0; t < 7; ++t) A[t] = L[t];
+  finish_agent(a, qi, A);
+}
+
 }  // namespace
+
+cudaError_t launch_ss_lim(const StepArgs& a, float* lim_send, cudaStream_t s) {
+  if (a.m <= 0) return cudaSuccess;
+  k_ss_lim<<<(unsigned)((a.m + 255) / 256), 256, 0, s>>>(a, lim_send);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_ss_cellsort(int* perm, const int* start, int cells, cudaStream_t s) {
+  k_ss_cellsort<<<(unsigned)((cells + 255) / 256), 256, 0, s>>>(perm, start, cells);
+  return cudaGetLastError();
+}
+
+// This rank's share of the global triangle over the nsorted sorted agents.
+cudaError_t launch_ss_search(const StepArgs& a, const int* gperm, int64_t nsorted, const float* lim_full, float4* sp,
+                             int* sidx, const long long* fb_prev, long long* fb_cur, long long* splits, int rank,
+                             int world, cudaStream_t s) {
+  constexpr int NT = 512;
+  constexpr int64_t QBS = NT * Q;
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const int64_t npad = (nsorted + QBS - 1) / QBS * QBS;
+  const int64_t nb = npad / QBS;
+  const int64_t T = nb * npad - QBS * (nb * (nb - 1) / 2);
+  const int64_t lo = (int64_t)((__int128)T * rank / world) / UG * UG;
+  const int64_t hi = rank + 1 == world ? T : (int64_t)((__int128)T * (rank + 1) / world) / UG * UG;
+  const int g = (int)std::max<int64_t>(1, std::min<int64_t>(std::min<int64_t>(sym_grid<NT>(sms), (hi - lo + CT - 1) / CT),
+                                                             SYM_FB_MAX_CTAS));
+  const int64_t cap = sym_capacity(nsorted);
+  float* spf = reinterpret_cast<float*>(sp);
+  k_ss_spbuild<<<(unsigned)((npad + 255) / 256), 256, 0, s>>>(a, gperm, nsorted, lim_full, spf, cap, sidx, npad, QBS,
+                                                              g, lo, hi, 6, fb_prev, splits);
+  if (cudaError_t e = cudaGetLastError()) return e;
+  if (hi <= lo) return cudaSuccess;
+  return launch_pdl(k_sym<NT>, dim3(g), dim3(NT), sizeof(SymSmem<NT>), s, a, (const float*)spf, cap,
+                    (const int*)sidx, npad, (const long long*)splits, fb_cur);
+}
+
+cudaError_t launch_ss_select(const StepArgs& a, const key_t* recv, const int* rcnt, int world, cudaStream_t s) {
+  if (a.nloc <= 0) return cudaSuccess;
+  BOIDS_PREFER_SMEM(k_ss_select);
+  return launch_pdl(k_ss_select, dim3((unsigned)((a.nloc + 127) / 128)), dim3(128), 0, s, a, recv, rcnt, world);
+}
 
 int64_t sym_capacity(int64_t nloc) { return (nloc + 2047) / 2048 * 2048; }
 

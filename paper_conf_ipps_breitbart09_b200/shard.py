@@ -69,11 +69,61 @@ def device_view(ptr: int, nbytes: int, device):
     return torch.as_tensor(_CudaArray(ptr, nbytes // 4), device=device)
 
 
+class _SymViews:
+    """Zero-copy float32 views of a handle's sym-shard exchange buffers (bits are moved, never read)."""
+
+    def __init__(self, h: int, world: int, m: int, device):
+        b = abi.boids_symshard_buffers(h)
+        cap = b["hits_cap"]
+        self.lim_send = device_view(b["lim_send"], m * 4, device)
+        self.lim_full = device_view(b["lim_full"], world * m * 4, device)
+        self.hits = device_view(b["hits"], world * m * cap * 8, device)  # u64 keys as 2 float32 each
+        self.hitcnt = device_view(b["hitcnt"], world * m * 4, device)
+        self.recv = device_view(b["recv"], world * m * cap * 8, device)
+        self.rcnt = device_view(b["rcnt"], world * m * 4, device)
+        self.block_keys = m * cap * 2  # float32 words per rank block
+        self.block_cnt = m
+
+
+def emulated_symshard_step(handles, views, dt: float, warm: bool):
+    """One step of G sym-shard handles on ONE device (tests, per-rank timing): both
+    exchanges (and the position all-gather) done by device copies."""
+    world = len(handles)
+    sends = views["pos"]
+    for r, (send, _, nf) in enumerate(sends):  # all-gather of the [pos4 | fwd4] slices
+        for (_, full, _) in sends:
+            full[r * nf:(r + 1) * nf].copy_(send)
+    if not warm:
+        for h in handles:
+            abi.boids_step_shard(h, dt)
+        return
+    sv = views["sym"]
+    m = sv[0].block_cnt
+    for h in handles:
+        abi.boids_symshard_prep(h)
+    for r, v in enumerate(sv):  # all-gather of the limits
+        for w in sv:
+            w.lim_full[r * m:(r + 1) * m].copy_(v.lim_send)
+    for h in handles:
+        abi.boids_symshard_search(h)
+    for d, vd in enumerate(sv):  # all-to-all of the hit blocks
+        for s_, vs in enumerate(sv):
+            k = vd.block_keys
+            vd.recv[s_ * k:(s_ + 1) * k].copy_(vs.hits[d * k:(d + 1) * k])
+            vd.rcnt[s_ * m:(s_ + 1) * m].copy_(vs.hitcnt[d * m:(d + 1) * m])
+    for h in handles:
+        abi.boids_symshard_finish(h, dt)
+
+
 class ShardedFlock:
-    """One rank of an index-sharded flock.  Call inside an initialised process group."""
+    """One rank of an index-sharded flock.  Call inside an initialised process group.
+
+    sym=True (brute force): warm steps split the global unordered-pair triangle
+    over the ranks (boids_symshard_*): two more collectives per step (the limits'
+    all-gather, the hits' all-to-all) instead of n/G x n ordered pairs per rank."""
 
     def __init__(self, n: int, params=None, seed: int = 1, group=None, kernel: int | None = None,
-                 record_steering: bool = False, profile: bool = False):
+                 record_steering: bool = False, profile: bool = False, sym: bool = False):
         import torch
         import torch.distributed as dist
 
@@ -98,6 +148,9 @@ class ShardedFlock:
         self.n = n
         info = abi.boids_info(self.h)
         self.lo, self.hi, self.m = info.lo, info.hi, info.slice
+        self.sym = sym and self.params.search_mode == abi.BOIDS_BRUTE and self.params.think_every == 1
+        self.sv = _SymViews(self.h, self.world, self.m, self.device) if self.sym else None
+        self.steps_done = 0
 
     def exchange(self):
         """a1: all-gather every rank's [pos4 | fwd4] slice into the full buffer (NCCL)."""
@@ -109,8 +162,26 @@ class ShardedFlock:
     def step(self, dt: float, steps: int = 1):
         for _ in range(steps):
             self.exchange()
-            abi.boids_step_shard(self.h, dt)
+            if self.sym and self.steps_done > 0:
+                self._sym_step(dt)
+            else:
+                abi.boids_step_shard(self.h, dt)
+            self.steps_done += 1
         return self
+
+    def _sym_step(self, dt: float):
+        d, v = self.dist, self.sv
+        try:
+            abi.boids_symshard_prep(self.h)
+            d.all_gather_into_tensor(v.lim_full, v.lim_send, group=self.group)
+            abi.boids_symshard_search(self.h)
+            d.all_to_all_single(v.recv, v.hits, group=self.group)
+            d.all_to_all_single(v.rcnt, v.hitcnt, group=self.group)
+        except abi.BoidsError:
+            raise
+        except Exception as e:  # surface as the ABI's NCCL error code
+            raise abi.BoidsError(abi.BOIDS_ENCCL, f"sym-shard collective failed: {e}") from e
+        abi.boids_symshard_finish(self.h, dt)
 
     def state(self):
         return abi.boids_get_state(self.h)

@@ -113,3 +113,41 @@ def test_sharded_flock_nccl_single_rank(boidslib, orc):
             assert np.array_equal(got[k], ref[k]), k
     finally:
         dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("n,world,steps", [(9000, 2, 5), (20000, 3, 4), (20000, 4, 4), (30001, 8, 3)])
+def test_symshard_emulation_oracle(boidslib, orc, n, world, steps):
+    """Sym-shards: the unordered-pair triangle split over `world` index shards
+    (boids_symshard_*), both exchanges emulated by device copies; the gathered
+    lists and states after `steps` steps equal the oracle's bit for bit."""
+    import torch
+
+    import paper_conf_ipps_breitbart09_b200 as pk
+    from paper_conf_ipps_breitbart09_b200 import abi
+    from paper_conf_ipps_breitbart09_b200.shard import _SymViews, device_view, emulated_symshard_step
+
+    p = pk.boids_default_params(init_mode=1, world_radius=25.0)
+    dev = torch.device("cuda", 0)
+    hs = [abi.boids_create_shard(n, p, 1, r, world) for r in range(world)]
+    try:
+        stream = torch.cuda.current_stream().cuda_stream
+        pos = []
+        for h in hs:
+            abi.boids_set_stream(h, stream)
+            send, full, nbytes = abi.boids_shard_buffers(h)
+            pos.append((device_view(send, nbytes, dev), device_view(full, nbytes * world, dev), nbytes // 4))
+        m = abi.boids_info(hs[0]).slice
+        views = {"pos": pos, "sym": [_SymViews(h, world, m, dev) for h in hs]}
+        for t in range(steps):
+            emulated_symshard_step(hs, views, DT, warm=t > 0)
+        torch.cuda.synchronize()
+        assert abi.boids_info(hs[0]).last_path == abi.BOIDS_PATH_SYM
+        got = {k: np.concatenate([abi.boids_get_state(h)[k] for h in hs]) for k in KEYS}
+        got_nbr = np.concatenate([abi.boids_get_neighbors(h)[0] for h in hs])
+    finally:
+        for h in hs:
+            abi.boids_destroy(h)
+    ref, ref_nbr = _oracle_run(orc, n, p, steps, seed=1)
+    assert np.array_equal(got_nbr, ref_nbr)
+    for k in KEYS:
+        assert np.array_equal(got[k], ref[k]), k
