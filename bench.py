@@ -264,7 +264,8 @@ def main():
                                      think_every=max(1, args.think))
     dt = float(W.DT)
     if dist is not None:
-        fl = ShardedFlock(cfg.n, params, seed=1, kernel=args.kernel)
+        # brute force: sym-shards (the unordered-pair triangle split over the ranks) unless --no-sym
+        fl = ShardedFlock(cfg.n, params, seed=1, kernel=args.kernel, sym=not args.no_sym)
         h = fl.h
         step = lambda: fl.step(dt, 1)  # noqa: E731
         nloc = fl.hi - fl.lo
@@ -341,8 +342,10 @@ def main():
         pairs_per_launch = float(grid_pairs) / max(k_n, 1)
         pairs_note = " (27-cell stencil candidates, device counter)"
     elif sym:  # k_sym: every unordered pair once, tested against both agents' limits
-        pairs_per_launch = float(cfg.n) * float(cfg.n - 1) / 2
+        pairs_per_launch = float(cfg.n) * float(cfg.n - 1) / 2 / world
         pairs_note = " (n(n-1)/2 unordered pairs: d2 is symmetric, each evaluated once for both agents)"
+        if world > 1:
+            pairs_note += f"; this rank's 1/{world} share of the triangle (sym-shards)"
     else:  # every thinking agent against all n (think mode: 1/k of the agents per step)
         pairs_per_launch = float(nloc) * float(cfg.n) / think
         pairs_note = " (n_local x n ordered pairs)"
@@ -365,6 +368,8 @@ def main():
                     abi.BOIDS_PATH_FUSED: "k_fused (cold-step cluster kernel)",
                     abi.BOIDS_PATH_SIMPLE: "k_search_simple (tiled search, thesis structure)",
                     abi.BOIDS_PATH_SMALL: "k_small (whole warm step in one kernel: search + merge + steer + modify)"}
+    if sym and dist is not None:
+        kernel_names[path] = "k_ss_spbuild + k_sym (this rank's share of the warm-step unordered-pair search)"
     roofline = {"bound": "alu",
                 "kernel": kernel_names.get(path, f"path {path}"), "path": path,
                 "achieved": achieved, "peak": peak, "unit": "TFLOP/s", "frac": achieved / peak,

@@ -914,7 +914,8 @@ BOIDS_API int boids_symshard_prep(boids_ctx* c) {
   }
   c->since_sort++;
   CK(cudaMemsetAsync(c->sym_rcount, 0, sizeof(int32_t), c->stream));
-  return launch(c, 0, [&] { return launch_ss_lim(a, c->ss_lim_send, c->stream); });
+  // class 4 (with the routing): the search class (0) holds one record per step, the triangle share
+  return launch(c, 4, [&] { return launch_ss_lim(a, c->ss_lim_send, c->stream); });
 }
 
 BOIDS_API int boids_symshard_search(boids_ctx* c) {

@@ -148,7 +148,8 @@ class ShardedFlock:
         self.n = n
         info = abi.boids_info(self.h)
         self.lo, self.hi, self.m = info.lo, info.hi, info.slice
-        self.sym = sym and self.params.search_mode == abi.BOIDS_BRUTE and self.params.think_every == 1
+        self.sym = (sym and self.params.search_mode == abi.BOIDS_BRUTE and self.params.think_every == 1
+                    and kernel in (None, abi.BOIDS_KERNEL_FUSED))
         self.sv = _SymViews(self.h, self.world, self.m, self.device) if self.sym else None
         self.steps_done = 0
 
