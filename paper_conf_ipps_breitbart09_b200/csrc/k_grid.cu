@@ -200,9 +200,12 @@ __device__ __forceinline__ void grid_tile(const float4* tile, int cnt, const flo
       // Every lane collects its passing (query, candidate) pairs as bits, then
       // the warp inserts them lane-parallel: each round every lane with bits
       // left inserts its lowest one, so the warp runs max-per-lane rounds of the
-      // insertion instead of one per distinct (q, u) any lane holds.  The order
-      // of insertions never matters (exact (d2, index) key; a pair above the
-      // tightened limit cannot be among the final 7).
+      // insertion instead of one per distinct (q, u) any lane holds.  A round
+      // re-reads its candidate from the tile and recomputes the d2 with the same
+      // operations (the same float) -- cheaper than selecting one of the 16
+      // distances held in registers.  The order of insertions never matters
+      // (exact (d2, index) key; a pair above the tightened limit cannot be among
+      // the final 7).
       unsigned bits = 0;
 #pragma unroll
       for (int u = 0; u < U; ++u) {
@@ -215,20 +218,23 @@ __device__ __forceinline__ void grid_tile(const float4* tile, int cnt, const flo
         if (bits) {
           const int b = __ffs(bits) - 1;
           bits &= bits - 1;
-          float dd = 0.f, lq = 0.f;
-          int j = 0, qq = 0;
+          const int qq = b / U;
+          float2 qxy = pxy[0];
+          float qz = pz[0], lq = lim[0];
 #pragma unroll
-          for (int q = 0; q < QV; ++q)
-#pragma unroll
-            for (int u = 0; u < U; ++u)
-              if (b == q * U + u) {
-                dd = d[q][u];
-                j = __float_as_int(cc[u].w);
-                lq = lim[q];
-                qq = q;
-              }
+          for (int q = 1; q < QV; ++q)
+            if (qq == q) {
+              qxy = pxy[q];
+              qz = pz[q];
+              lq = lim[q];
+            }
+          const float4 cu = tile[c + (b % U)];
+          const float2 dxy = __fadd2_rn(qxy, make_float2(-cu.x, -cu.y));
+          const float2 sq = __fmul2_rn(dxy, dxy);
+          const float dz = __fsub_rn(qz, cu.z);
+          const float dd = __fadd_rn(__fadd_rn(sq.x, sq.y), __fmul_rn(dz, dz));
           if (dd <= lq) {  // the limit may have tightened since the bit was set
-            const float nl = insert_smem7(&lists[qslot(warp, qq, lane, rr)], QBG, make_key(dd, j));
+            const float nl = insert_smem7(&lists[qslot(warp, qq, lane, rr)], QBG, make_key(dd, __float_as_int(cu.w)));
 #pragma unroll
             for (int q = 0; q < QV; ++q)
               if (q == qq) lim[q] = fminf(lim[q], nl);

@@ -25,6 +25,7 @@ for name in sys.argv[1:] or ["c3"]:
     prof = f.profile(reset=True)
     print(f"{name} n={cfg.n} per-step kernel means (us): "
           + ", ".join(f"{k}={v[0] / max(v[1], 1) * 1e3:.1f}x{v[1] // 8}" for k, v in prof.items() if v[1]))
+    abi.boids_set_option(f.h, abi.BOIDS_OPT_PROFILE, int(os.environ.get("PROF", "1")))  # 0: timeline without events
     abi.boids_set_option(f.h, abi.BOIDS_OPT_PHASES, 1024)
     f.step(float(W.DT), 1)
     f.sync()
