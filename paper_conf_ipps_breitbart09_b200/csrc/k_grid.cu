@@ -425,12 +425,13 @@ __global__ void __launch_bounds__(NTG, 5) k_grid(StepArgs a, GridArgs g) {  // 5
       const float4* tile = sm.ring[s];
       const int cnt = walk(sm, r, off);
       // warps without queries in this item only keep the ring protocol; a warp
-      // computes only its query groups that hold queries (the item's last warp
-      // is usually partial: the padded groups cost work and loosen the vote)
-      if (qv == 4) grid_tile<4>(tile, cnt, pxy, pz, lim, limc, gq, sm.lists, warp, lane, rr, groups, slow_groups);
-      else if (qv == 3) grid_tile<3>(tile, cnt, pxy, pz, lim, limc, gq, sm.lists, warp, lane, rr, groups, slow_groups);
-      else if (qv == 2) grid_tile<2>(tile, cnt, pxy, pz, lim, limc, gq, sm.lists, warp, lane, rr, groups, slow_groups);
-      else if (qv == 1) grid_tile<1>(tile, cnt, pxy, pz, lim, limc, gq, sm.lists, warp, lane, rr, groups, slow_groups);
+      // with 1-2 query groups holding queries computes two (the item's last warp
+      // is usually partial: padded groups cost work and loosen the vote)
+      // Two specialisations only: four (3 or 4 groups hold queries) and two -- the
+      // kernel's stall_no_inst (instruction fetch) fell with every copy removed
+      // (C5 k_grid 1.82 ms with 4 copies -> 1.72 ms with 2; 1.75 ms with 1)
+      if (qv >= 3) grid_tile<4>(tile, cnt, pxy, pz, lim, limc, gq, sm.lists, warp, lane, rr, groups, slow_groups);
+      else if (qv >= 1) grid_tile<2>(tile, cnt, pxy, pz, lim, limc, gq, sm.lists, warp, lane, rr, groups, slow_groups);
       // every thread releases the stage after its own reads (per-thread release
       // orders them before the stage's refill by the bulk copy; compute-sanitizer
       // racecheck does not count a __syncwarp before one lane's arrive as ordering)
