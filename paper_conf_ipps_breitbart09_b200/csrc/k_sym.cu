@@ -682,6 +682,35 @@ __global__ void __launch_bounds__(256) k_sym_prep(StepArgs a, float* __restrict_
 // 8 smallest keys per thread; a shuffle butterfly and a shared-memory pass merge
 // them.  The CTA then finishes the agent -- list, 8th nearest (the next step's
 // warm-bound seed), steering, modification -- and k_select skips it.
+// The 8 smallest keys over the warp's 32 ascending 8-lists (keys unique across
+// lanes), ascending, in every lane: extract the warp minimum of the list heads
+// (two 32-bit min reductions: d2 bits, then the index among the lanes holding
+// that d2) and pop it from its lane, up to 8 times, stopping at the first empty
+// minimum.  k_route's lists are nearly empty (a routed agent has few agents
+// within r, and they are spread over 512 threads x P parts), so this takes a
+// round or two where a shuffle butterfly of merge8 networks took five full
+// levels (C4 sym-shards, 8 ranks: k_route 66 us, most of it merging).
+__device__ __forceinline__ void warp_top8(key_t (&A)[8], key_t (&out)[8]) {
+#pragma unroll
+  for (int t = 0; t < 8; ++t) out[t] = KEY_EMPTY;
+#pragma unroll 1
+  for (int t = 0; t < 8; ++t) {
+    const unsigned hi = (unsigned)(A[0] >> 32), lo = (unsigned)A[0];
+    const unsigned mhi = __reduce_min_sync(0xffffffffu, hi);
+    const unsigned mlo = __reduce_min_sync(0xffffffffu, hi == mhi ? lo : 0xffffffffu);
+    const key_t m = ((key_t)mhi << 32) | mlo;
+    if (m == KEY_EMPTY) break;  // warp-uniform
+#pragma unroll
+    for (int s = 0; s < 8; ++s)
+      if (s == t) out[s] = m;
+    if (A[0] == m) {  // the one lane holding it pops its head
+#pragma unroll
+      for (int s = 0; s < 7; ++s) A[s] = A[s + 1];
+      A[7] = KEY_EMPTY;
+    }
+  }
+}
+
 constexpr int RT = 512, RU = 16;
 constexpr int RP_MAX = 16;  // candidate parts per routed agent (few routed agents -> more CTAs each)
 __device__ __forceinline__ void route_body(const StepArgs& a) {
@@ -730,24 +759,23 @@ __device__ __forceinline__ void route_body(const StepArgs& a) {
         }
       }
     }
+    {
+      key_t W[8];
+      warp_top8(A, W);
+      if (lane == 0)
 #pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      key_t B[8];
-#pragma unroll
-      for (int s = 0; s < 8; ++s) B[s] = __shfl_xor_sync(0xffffffffu, A[s], o);
-      merge8(A, B);
+        for (int s = 0; s < 8; ++s) wl[warp][s] = W[s];
     }
-    if (lane == 0)
-#pragma unroll
-      for (int s = 0; s < 8; ++s) wl[warp][s] = A[s];
     __syncthreads();
-    if (tid == 0) {
-      for (int v = 1; v < RT / 32; ++v) {
-        key_t B[8];
+    if (warp == 0) {  // the 16 warps' lists, one per lane
 #pragma unroll
-        for (int s = 0; s < 8; ++s) B[s] = wl[v][s];
-        merge8(A, B);
-      }
+      for (int s = 0; s < 8; ++s) A[s] = lane < RT / 32 ? wl[lane][s] : KEY_EMPTY;
+      key_t W[8];
+      warp_top8(A, W);
+#pragma unroll
+      for (int s = 0; s < 8; ++s) A[s] = W[s];
+    }
+    if (tid == 0) {
       s_last = 1;
       if (P > 1) {  // publish this part; the last part's CTA merges all of them
 #pragma unroll
@@ -756,17 +784,20 @@ __device__ __forceinline__ void route_body(const StepArgs& a) {
         s_last = atomicAdd(a.rbcount + r, 1) == P - 1;
         if (s_last) {
           __threadfence();
-#pragma unroll
-          for (int s = 0; s < 8; ++s) A[s] = KEY_EMPTY;
-          for (int q = 0; q < P; ++q) {
-            key_t B[8];
-#pragma unroll
-            for (int s = 0; s < 8; ++s) B[s] = __ldcg(a.rpart + ((int64_t)r * RP_MAX + q) * 8 + s);
-            merge8(A, B);
-          }
           a.rbcount[r] = 0;  // ready for the next step
         }
       }
+    }
+    __syncthreads();
+    if (P > 1 && s_last && warp == 0) {  // the P parts' lists, one per lane
+#pragma unroll
+      for (int s = 0; s < 8; ++s) A[s] = lane < P ? __ldcg(a.rpart + ((int64_t)r * RP_MAX + lane) * 8 + s) : KEY_EMPTY;
+      key_t W[8];
+      warp_top8(A, W);
+#pragma unroll
+      for (int s = 0; s < 8; ++s) A[s] = W[s];
+    }
+    if (tid == 0) {
       if (s_last) {
         a.nbr8[qi] = A[7] == KEY_EMPTY ? -1 : key_idx(A[7]);
         int nb[7], cnt = 0;
