@@ -902,30 +902,9 @@ BOIDS_API int boids_symshard_prep(boids_ctx* c) {
   if ((rc = ss_alloc(c))) return rc;
   StepArgs a = make_args(c, 0.f);
   a.routed = c->routed;
-  // this rank's Morton query order (the window bound looks agents up in it)
-  if (c->since_sort < 0 || c->since_sort >= c->resort_every) {
-    if ((rc = launch(c, 2, [&] {
-           return launch_bin(a.full, c->m, a.sdiv, c->lo, c->nloc, c->loc_grid, c->cellrank, c->bcnt, c->bstart,
-                             nullptr, c->qperm, (int)c->lo, c->stream, nullptr);
-         }, 3)))
-      return rc;
-    c->since_sort = 0;
-    c->steps_sorted++;
-  }
-  c->since_sort++;
-  CK(cudaMemsetAsync(c->sym_rcount, 0, sizeof(int32_t), c->stream));
-  // class 4 (with the routing): the search class (0) holds one record per step, the triangle share
-  return launch(c, 4, [&] { return launch_ss_lim(a, c->ss_lim_send, c->stream); });
-}
-
-BOIDS_API int boids_symshard_search(boids_ctx* c) {
-  int rc = ss_check(c);
-  if (rc) return rc;
-  if (!c->ss_lim_send) return fail(BOIDS_EINVAL, "boids_symshard_prep first");
-  DeviceGuard g(c->dev);
-  StepArgs a = make_args(c, 0.f);
   const int64_t slots = (int64_t)c->world * c->m;
-  // the global Morton order, identical on every rank (cells sorted by index)
+  // the global Morton order, identical on every rank (cells sorted by index): the
+  // limits' window bound looks agents up in it, and the search walks it
   if (c->ss_since_sort < 0 || c->ss_since_sort >= c->resort_every) {
     if ((rc = launch(c, 2, [&] {
            cudaError_t e = launch_bin(a.full, c->m, a.sdiv, 0, slots, c->loc_grid, c->cellrank, c->ss_gbcnt,
@@ -935,8 +914,21 @@ BOIDS_API int boids_symshard_search(boids_ctx* c) {
          }, 4)))
       return rc;
     c->ss_since_sort = 0;
+    c->steps_sorted++;
   }
   c->ss_since_sort++;
+  CK(cudaMemsetAsync(c->sym_rcount, 0, sizeof(int32_t), c->stream));
+  // class 4 (with the routing): the search class (0) holds one record per step, the triangle share
+  return launch(c, 4, [&] { return launch_ss_lim(a, c->ss_lim_send, c->ss_gperm, c->ss_gbstart, c->n, c->stream); });
+}
+
+BOIDS_API int boids_symshard_search(boids_ctx* c) {
+  int rc = ss_check(c);
+  if (rc) return rc;
+  if (!c->ss_lim_send) return fail(BOIDS_EINVAL, "boids_symshard_prep first");
+  DeviceGuard g(c->dev);
+  StepArgs a = make_args(c, 0.f);
+  const int64_t slots = (int64_t)c->world * c->m;
   CK(cudaMemsetAsync(c->ss_hitcnt, 0, slots * sizeof(int32_t), c->stream));
   StepArgs as = a;
   as.hits = c->ss_hits;

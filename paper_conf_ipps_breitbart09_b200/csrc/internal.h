@@ -239,7 +239,8 @@ cudaError_t launch_sym_scan(const StepArgs& a, float4* sp, int* sidx, const long
                             long long* splits, cudaStream_t s);
 cudaError_t launch_route(const StepArgs& a, cudaStream_t s);
 // sym-shards (k_sym.cu): the unordered-pair triangle split over index-sharded ranks
-cudaError_t launch_ss_lim(const StepArgs& a, float* lim_send, cudaStream_t s);
+cudaError_t launch_ss_lim(const StepArgs& a, float* lim_send, const int* gperm, const int* gstart, int64_t nsorted,
+                          cudaStream_t s);
 cudaError_t launch_ss_cellsort(int* perm, const int* start, int cells, cudaStream_t s);
 cudaError_t launch_ss_search(const StepArgs& a, const int* gperm, int64_t nsorted, const float* lim_full, float4* sp,
                              int* sidx, const long long* fb_prev, long long* fb_cur, long long* splits, int rank,

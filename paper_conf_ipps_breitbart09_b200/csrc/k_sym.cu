@@ -590,11 +590,14 @@ __device__ __forceinline__ float sym_t0(const StepArgs& a, int64_t qi, float4 me
 // sort is up to BOIDS_OPT_RESORT steps old: only the bound's tightness depends
 // on that, never the result.
 constexpr int WIN = 256;  // C4: 64 -> 11 routed agents per step, 256 -> 3 (route 32 -> 22 us, prep +17 us; net -0.5..1 %)
-__device__ float window_bound(const StepArgs& a, int qi, float4 me) {
-  const int n = (int)a.nloc;
-  if (!a.lstart || !a.qperm || n < 8 || !(me.x == me.x && me.y == me.y && me.z == me.z))
+// The window over an explicit order: perm[0..n) agent indices (offset by base
+// into the position buffer) in Morton order of grid g, start[c] = the first
+// position of cell c; self = the querying agent's own index in perm's terms.
+__device__ float window_bound_in(const StepArgs& a, const int* __restrict__ perm, const int* __restrict__ start,
+                                 const BinGrid& g, int n, int64_t base, int64_t self, float4 me) {
+  if (!start || !perm || n < 8 || !(me.x == me.x && me.y == me.y && me.z == me.z))
     return __int_as_float(0x7f800000);
-  const int p0 = __ldg(a.lstart + cell_of(me, a.loc));
+  const int p0 = __ldg(start + cell_of(me, g));
   int lo = p0 - WIN / 2;
   lo = lo > n - WIN ? n - WIN : lo;
   lo = lo < 0 ? 0 : lo;
@@ -606,13 +609,13 @@ __device__ float window_bound(const StepArgs& a, int qi, float4 me) {
   for (int p0 = lo; p0 < hi; p0 += G) {
     int j[G];
 #pragma unroll
-    for (int k = 0; k < G; ++k) j[k] = p0 + k < hi ? __ldg(a.qperm + p0 + k) : -1;
+    for (int k = 0; k < G; ++k) j[k] = p0 + k < hi ? __ldg(perm + p0 + k) : -1;
     float4 q[G];
 #pragma unroll
-    for (int k = 0; k < G; ++k) q[k] = __ldg(pos_of(a.full, a.m, a.sdiv, a.lo + (j[k] < 0 ? 0 : j[k])));
+    for (int k = 0; k < G; ++k) q[k] = __ldg(pos_of(a.full, a.m, a.sdiv, base + (j[k] < 0 ? 0 : j[k])));
 #pragma unroll
     for (int k = 0; k < G; ++k) {
-      if (j[k] < 0 || j[k] == qi) continue;
+      if (j[k] < 0 || j[k] == self) continue;
       float d = dist2(me.x, me.y, me.z, q[k]);
 #pragma unroll
       for (int t = 0; t < 7; ++t) {  // keep the 7 smallest, ascending
@@ -623,6 +626,10 @@ __device__ float window_bound(const StepArgs& a, int qi, float4 me) {
     }
   }
   return b[6];
+}
+
+__device__ float window_bound(const StepArgs& a, int qi, float4 me) {
+  return window_bound_in(a, a.qperm, a.lstart, a.loc, (int)a.nloc, a.lo, qi, me);
 }
 
 // Structure of arrays over the sorted positions p: spf[p], spf[cap + p], spf[2 cap + p] = x, y, z and
@@ -877,7 +884,8 @@ cudaError_t sym_with(const StepArgs& a, float4* sp, int* sidx, const long long* 
 // Every unordered pair is evaluated exactly once over all ranks (the ranks'
 // shares tile the triangle of ONE order), so the hit set of every agent is the
 // single-GPU one: identical lists.
-__global__ void __launch_bounds__(256) k_ss_lim(StepArgs a, float* __restrict__ lim_send) {
+__global__ void __launch_bounds__(256) k_ss_lim(StepArgs a, float* __restrict__ lim_send, const int* __restrict__ gperm,
+                                                const int* __restrict__ gstart, int nsorted) {
   const int64_t i = (int64_t)blockIdx.x * 256 + threadIdx.x;
   if (i >= a.m) return;
   if (i >= a.nloc) {
@@ -890,7 +898,10 @@ __global__ void __launch_bounds__(256) k_ss_lim(StepArgs a, float* __restrict__ 
   int c = 0;
   const float t0 = sym_t0(a, i, me, c);
   float lim = fminf(r2_in, t0);
-  if (t0 > r2_in) lim = fminf(lim, window_bound(a, (int)i, me));
+  // the window over the GLOBAL Morton order (every rank's agents): over this
+  // rank's own 1/G of them the 7th nearest lies ~G^(1/3) times farther and many
+  // more agents stayed unbounded (C4, 8 ranks: ~45 routed per rank vs ~36 in all)
+  if (t0 > r2_in) lim = fminf(lim, window_bound_in(a, gperm, gstart, a.loc, nsorted, 0, a.lo + i, me));
   if (c == 7 && lim > r2_in && a.rlist) {  // unbounded (a wrap): k_route searches it whole
     a.rlist[atomicAdd(a.rcount, 1)] = (int)i;
     a.routed[i] = 1;
@@ -984,9 +995,10 @@ __global__ void __launch_bounds__(128) k_ss_select(StepArgs a, const key_t* __re
 
 }  // namespace
 
-cudaError_t launch_ss_lim(const StepArgs& a, float* lim_send, cudaStream_t s) {
+cudaError_t launch_ss_lim(const StepArgs& a, float* lim_send, const int* gperm, const int* gstart, int64_t nsorted,
+                          cudaStream_t s) {
   if (a.m <= 0) return cudaSuccess;
-  k_ss_lim<<<(unsigned)((a.m + 255) / 256), 256, 0, s>>>(a, lim_send);
+  k_ss_lim<<<(unsigned)((a.m + 255) / 256), 256, 0, s>>>(a, lim_send, gperm, gstart, (int)nsorted);
   return cudaGetLastError();
 }
 

@@ -115,7 +115,7 @@ def test_sharded_flock_nccl_single_rank(boidslib, orc):
         dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("n,world,steps", [(9000, 2, 5), (20000, 3, 4), (20000, 4, 4), (30001, 8, 3)])
+@pytest.mark.parametrize("n,world,steps", [(9000, 2, 5), (20000, 3, 4), (20000, 4, 4), (30001, 8, 3), (6000, 3, 12)])
 def test_symshard_emulation_oracle(boidslib, orc, n, world, steps):
     """Sym-shards: the unordered-pair triangle split over `world` index shards
     (boids_symshard_*), both exchanges emulated by device copies; the gathered
