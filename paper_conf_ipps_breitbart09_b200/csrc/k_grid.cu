@@ -30,6 +30,7 @@
 // agents (steering + modification) itself: search, steering and modification
 // in one kernel, no merge.
 #include <algorithm>
+#include <cstdlib>
 
 #include "step_common.cuh"
 #include "tma.cuh"
@@ -427,11 +428,14 @@ __global__ void __launch_bounds__(NTG, 5) k_grid(StepArgs a, GridArgs g) {  // 5
       // warps without queries in this item only keep the ring protocol; a warp
       // with 1-2 query groups holding queries computes two (the item's last warp
       // is usually partial: padded groups cost work and loosen the vote)
-      // Two specialisations only: four (3 or 4 groups hold queries) and two -- the
-      // kernel's stall_no_inst (instruction fetch) fell with every copy removed
-      // (C5 k_grid 1.82 ms with 4 copies -> 1.72 ms with 2; 1.75 ms with 1)
+      // Three specialisations: four (3 or 4 groups hold queries), two and one (the
+      // small round-robin items of spatial shards hold 1-2 groups per warp).  The
+      // kernel's stall_no_inst (instruction fetch) grows with every copy: C5 k_grid
+      // 1.82 ms with 4 copies, 1.72 with {4, 2}, 1.74 with {4, 2, 1}; a spatial
+      // rank at 8 ranks 0.69 ms with {4, 2} (one-group warps padded to two), 0.57 here
       if (qv >= 3) grid_tile<4>(tile, cnt, pxy, pz, lim, limc, gq, sm.lists, warp, lane, rr, groups, slow_groups);
-      else if (qv >= 1) grid_tile<2>(tile, cnt, pxy, pz, lim, limc, gq, sm.lists, warp, lane, rr, groups, slow_groups);
+      else if (qv == 2) grid_tile<2>(tile, cnt, pxy, pz, lim, limc, gq, sm.lists, warp, lane, rr, groups, slow_groups);
+      else if (qv == 1) grid_tile<1>(tile, cnt, pxy, pz, lim, limc, gq, sm.lists, warp, lane, rr, groups, slow_groups);
       // every thread releases the stage after its own reads (per-thread release
       // orders them before the stage's refill by the bulk copy; compute-sanitizer
       // racecheck does not count a __syncwarp before one lane's arrive as ordering)
@@ -574,6 +578,11 @@ int grid_chunk(int64_t nq) {
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   const int64_t ctas = (int64_t)sms * r;
+  static const int force = [] {
+    const char* e = getenv("BOIDS_GRID_CHUNK");  // diagnostics: queries per item
+    return e ? atoi(e) : 0;
+  }();
+  if (force >= 32 && force <= QBG) return force;
   int64_t c = (nq / (3 * ctas) + 31) / 32 * 32;
   return (int)std::max<int64_t>(128, std::min<int64_t>(QBG, c));
 }
