@@ -14,7 +14,8 @@ a6 modification; a2 binning in grid mode), through the C ABI of libboids.so.
 * e2e        the same metric through the public C ABI with HOST buffers: every
              step boids_set_state (H2D) + step + boids_get_state (D2H), wall clock.
 * roofline   the search kernel of the path the library reports it ran
-             (boids_info.last_path: k_sym_prep + k_sym, k_bound + k_scan, k_grid):
+             (boids_info.last_path: k_sym -- its prologue k_sym_prep reported apart
+             and combined --, k_bound + k_scan, k_grid, k_small):
              algorithmic FP32 lane-ops per launch (8 per evaluated pair,
              DESIGN.md sec 5) / its mean launch duration (library-side CUDA
              events on the handle's stream; inside the timed region, or with
@@ -362,7 +363,7 @@ def main():
         except Exception:
             traffic = None
     kernel_names = {abi.BOIDS_PATH_GRID: "k_grid (binned search + steer + modify)",
-                    abi.BOIDS_PATH_SYM: "k_sym_prep + k_sym (warm-step unordered-pair search)",
+                    abi.BOIDS_PATH_SYM: "k_sym (warm-step unordered-pair search)",
                     abi.BOIDS_PATH_SCAN: "k_bound + k_scan (warm-step ordered-pair search)",
                     abi.BOIDS_PATH_THINK: "k_bound + k_scan over this step's thinkers (k_fused for never-searched ones)",
                     abi.BOIDS_PATH_FUSED: "k_fused (cold-step cluster kernel)",
@@ -420,6 +421,18 @@ def main():
                            "frac": ub / hbm, "bytes_per_agent": per_agent, "launches": u_n,
                            "kernel_ms_per_launch": u_ms / u_n, "peak_note": hbm_note,
                            "measured": "profiled pass of K steps after the timed region, L2 flushed per step"}
+    if sym and dist is None:  # k_sym's prologue (k_sym_prep: warm limits + the ordered SoA copy), timed apart
+        p_ms, p_n = prof1["search_prep"]
+        s_ms, s_n = prof1["fused_or_search"]
+        if p_n and s_n:
+            both = p_ms / p_n + s_ms / s_n
+            a_both = OPS_PER_PAIR * pairs_per_launch / (both / 1e3) / 1e12
+            roofline["prologue"] = {
+                "kernel": "k_sym_prep (warm limits, routing, agents in Morton order as SoA)",
+                "ms_per_launch": p_ms / p_n,
+                "search_incl_prologue": {"kernels": "k_sym_prep + k_sym", "ms_per_launch": both,
+                                         "achieved": a_both, "frac": a_both / peak},
+                "measured": "profiled pass of K steps after the timed region (events around each launch)"}
     b_ms, b_n = prof1["binning"]
     binning_roofline = None
     if b_n and grid:

@@ -335,8 +335,9 @@ BOIDS_API int boids_info(boids_ctx* ctx, boids_info_t* out);
 /* Accumulated kernel time (ms) and launch count per kernel class since the last
  * reset, measured with CUDA events on the handle's stream (BOIDS_OPT_PROFILE).
  * Classes: 0 fused/search, 1 update, 2 binning, 3 grid search, 4 k_route (agents searched
- * whole after a hit-buffer overflow or a wrap).  Synchronises. */
-#define BOIDS_PROF_CLASSES 5
+ * whole after a hit-buffer overflow or a wrap), 5 search prologue (k_sym_prep: the warm limits
+ * and the agents' spatially ordered copy k_sym reads).  Synchronises. */
+#define BOIDS_PROF_CLASSES 6
 BOIDS_API int boids_get_profile(boids_ctx* ctx, double* ms, int64_t* launches, int32_t reset);
 
 /* Diagnostics: copy `count` u64 phase stamps (8 per CTA) of the last fused step to host. */

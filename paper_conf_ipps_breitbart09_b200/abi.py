@@ -24,8 +24,8 @@ BOIDS_KERNEL_FUSED, BOIDS_KERNEL_SIMPLE, BOIDS_KERNEL_CLUSTER = 0, 1, 2
 BOIDS_OPT_RECORD_STEERING, BOIDS_OPT_KERNEL, BOIDS_OPT_PROFILE, BOIDS_OPT_CLUSTER, BOIDS_OPT_PHASES = 1, 2, 3, 4, 5
 BOIDS_OPT_RESORT, BOIDS_OPT_VOTE_U, BOIDS_OPT_SYMMETRIC, BOIDS_OPT_BALANCE, BOIDS_OPT_GRAPH = 6, 7, 8, 9, 10
 BOIDS_OPT_SMALL = 11
-BOIDS_PROF_CLASSES = 5
-PROF_NAMES = ("fused_or_search", "update", "binning", "grid_search", "route")
+BOIDS_PROF_CLASSES = 6
+PROF_NAMES = ("fused_or_search", "update", "binning", "grid_search", "route", "search_prep")
 
 # Every symbol include/boids.h declares (tests/test_abi.py checks the header against this).
 EXPORTS = (

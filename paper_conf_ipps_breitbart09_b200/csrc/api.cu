@@ -167,8 +167,8 @@ struct boids_ctx {
   };
   std::vector<Rec> recs;
   std::vector<cudaEvent_t> pool;
-  double prof_ms[BOIDS_PROF_CLASSES] = {0, 0, 0, 0, 0};
-  int64_t prof_n[BOIDS_PROF_CLASSES] = {0, 0, 0, 0, 0};
+  double prof_ms[BOIDS_PROF_CLASSES] = {};
+  int64_t prof_n[BOIDS_PROF_CLASSES] = {};
 
   float4* local() const { return shard ? buf[1] : buf[cur]; }
 };
@@ -640,11 +640,13 @@ int one_step(boids_ctx* c, float dt) {
         long long* fb_prev = c->sym_fb + (c->sym_fb_par ^ 1) * SYM_FB_LEN;
         long long* fb_cur = c->sym_fb + c->sym_fb_par * SYM_FB_LEN;
         c->sym_fb_par ^= 1;
-        if ((rc = launch(c, 0, [&] {
-               return launch_sym_scan(as, c->sym_sp, c->sym_idx, c->balance ? fb_prev : nullptr, fb_cur,
-                                      c->sym_fb + 2 * SYM_FB_LEN, c->stream);
-             }, 2)))
-          return rc;
+        // two launch records: the prologue (class 5) and k_sym itself (class 0, the search roofline)
+        for (int part = 1; part <= 2; ++part)
+          if ((rc = launch(c, part == 1 ? 5 : 0, [&] {
+                 return launch_sym_scan(as, c->sym_sp, c->sym_idx, c->balance ? fb_prev : nullptr, fb_cur,
+                                        c->sym_fb + 2 * SYM_FB_LEN, c->stream, part);
+               })))
+            return rc;
         if ((rc = launch(c, 1, [&] { return launch_warm_select(as, c->stream, false); }))) return rc;
         if ((rc = launch(c, 4, [&] { return launch_route(as, c->stream); }))) return rc;
       } else {

@@ -236,7 +236,8 @@ constexpr int SYM_FB_MAX_CTAS = 1024;
 constexpr int SYM_FB_LEN = 2 + 3 * SYM_FB_MAX_CTAS;
 // splits: [SYM_FB_MAX_CTAS + 1] int64 scratch: k_sym_prep writes every k_sym CTA's item range there
 cudaError_t launch_sym_scan(const StepArgs& a, float4* sp, int* sidx, const long long* fb_prev, long long* fb_cur,
-                            long long* splits, cudaStream_t s);
+                            long long* splits, cudaStream_t s,
+                            int part = 0);  // part 0: k_sym_prep + k_sym, 1: k_sym_prep, 2: k_sym
 cudaError_t launch_route(const StepArgs& a, cudaStream_t s);
 // sym-shards (k_sym.cu): the unordered-pair triangle split over index-sharded ranks
 cudaError_t launch_ss_lim(const StepArgs& a, float* lim_send, const int* gperm, const int* gstart, int64_t nsorted,

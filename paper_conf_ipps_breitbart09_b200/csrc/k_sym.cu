@@ -848,7 +848,7 @@ int sym_grid(int sms) {
 
 template <int NT>
 cudaError_t sym_with(const StepArgs& a, float4* sp, int* sidx, const long long* fb_prev, long long* fb_cur,
-                     long long* splits, int sms, cudaStream_t s) {
+                     long long* splits, int sms, cudaStream_t s, int part) {
   constexpr int64_t QBS = NT * Q;
   const int64_t npad = (a.nloc + QBS - 1) / QBS * QBS;
   const int64_t nb = npad / QBS;
@@ -861,8 +861,11 @@ cudaError_t sym_with(const StepArgs& a, float4* sp, int* sidx, const long long* 
   BOIDS_PREFER_SMEM(k_sym_prep);
   const int64_t cap = sym_capacity(a.nloc);  // sp holds 4 * cap floats: x[cap] | y[cap] | z[cap] | lim[cap]
   float* spf = reinterpret_cast<float*>(sp);
-  k_sym_prep<<<(unsigned)((npad + 255) / 256), 256, 0, s>>>(a, spf, cap, sidx, npad, QBS, g, wd4, fb_prev, splits);
-  if (cudaError_t e = cudaGetLastError()) return e;
+  if (part != 2) {
+    k_sym_prep<<<(unsigned)((npad + 255) / 256), 256, 0, s>>>(a, spf, cap, sidx, npad, QBS, g, wd4, fb_prev, splits);
+    if (cudaError_t e = cudaGetLastError()) return e;
+  }
+  if (part == 1) return cudaSuccess;
   return launch_pdl(k_sym<NT>, dim3(g), dim3(NT), sizeof(SymSmem<NT>), s, a, (const float*)spf, cap,
                     (const int*)sidx, npad, (const long long*)splits, fb_cur);
 }
@@ -1057,7 +1060,7 @@ cudaError_t launch_route(const StepArgs& a, cudaStream_t s) {
 }
 
 cudaError_t launch_sym_scan(const StepArgs& a, float4* sp, int* sidx, const long long* fb_prev, long long* fb_cur,
-                            long long* splits, cudaStream_t s) {
+                            long long* splits, cudaStream_t s, int part) {
   if (a.nloc <= 0) return cudaSuccess;
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
@@ -1069,9 +1072,9 @@ cudaError_t launch_sym_scan(const StepArgs& a, float4* sp, int* sidx, const long
     const char* e = getenv("BOIDS_SYM_NT");  // diagnostics: force a CTA shape (128 or 512)
     return e ? atoi(e) : 0;
   }();
-  if (force == 256) return sym_with<256>(a, sp, sidx, fb_prev, fb_cur, splits, sms, s);
-  if (force == 512 || (force != 128 && tiles512 >= 2LL * sms)) return sym_with<512>(a, sp, sidx, fb_prev, fb_cur, splits, sms, s);
-  return sym_with<128>(a, sp, sidx, fb_prev, fb_cur, splits, sms, s);
+  if (force == 256) return sym_with<256>(a, sp, sidx, fb_prev, fb_cur, splits, sms, s, part);
+  if (force == 512 || (force != 128 && tiles512 >= 2LL * sms)) return sym_with<512>(a, sp, sidx, fb_prev, fb_cur, splits, sms, s, part);
+  return sym_with<128>(a, sp, sidx, fb_prev, fb_cur, splits, sms, s, part);
 }
 
 }  // namespace boids
