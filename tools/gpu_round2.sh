@@ -22,8 +22,8 @@ for w in c4 c5; do
   timeout 900 python tools/rank_emulation.py --workload $w --ranks 1 2 4 8 > $OUT/ranks_$w.json 2> $OUT/ranks_$w.err
 done
 if [ -z "$NO_NCU" ]; then
-for w in ${NCU_WORKLOADS:-c3 c4 c5}; do
-  K=k_sym; [ $w = c5 ] && K=k_grid; [ $w = c1 ] && K=k_scan
+for w in ${NCU_WORKLOADS:-c2 c3 c4 c5}; do
+  K=k_sym; [ $w = c5 ] && K=k_grid; case $w in c1|c2) K=k_small;; esac
   timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches_$w.csv \
      python bench.py --workload $w --steps 3 --warmup 3 --no-cpu-baseline --no-e2e > $OUT/ncu_launch_$w.log 2>&1
   timeout 1200 ncu --set full --clock-control none --import-source on -k $K -s 3 -c 1 -o $OUT/${w}_$K \

@@ -29,7 +29,7 @@ UNIT_SCALE = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}
 for f in sorted(os.listdir(src)):
     if not f.endswith(".ncu-rep"):
         continue
-    w = f.split("_")[-1].split(".")[0]
+    w = f.split("_")[0]  # the workload (c3, c5think10, ...)
     rep = os.path.join(src, f)
     raw = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
     rows = list(csv.reader(io.StringIO(raw)))
