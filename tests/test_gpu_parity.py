@@ -358,6 +358,27 @@ def test_errors(pk):
             abi.boids_step_shard(f.h, 0.1)  # not a shard handle
 
 
+def test_profile_classes_sym_step(pk):
+    """A warm k_sym step records its prologue (k_sym_prep, class 5) and k_sym
+    (class 0) as two launches: bench.py's search roofline is k_sym alone, with
+    the prologue reported beside it."""
+    from paper_conf_ipps_breitbart09_b200 import abi
+
+    with pk.Flock(16384, seed=1) as f:
+        f.step(DT, 2)
+        abi.boids_set_option(f.h, abi.BOIDS_OPT_PROFILE, 1)
+        abi.boids_get_profile(f.h, reset=True)
+        f.step(DT, 3)
+        prof = abi.boids_get_profile(f.h, reset=True)
+        assert f.info().last_path == abi.BOIDS_PATH_SYM
+        assert prof["search_prep"][1] == 3 and prof["fused_or_search"][1] == 3
+        assert prof["fused_or_search"][0] > prof["search_prep"][0] > 0
+        abi.boids_set_option(f.h, abi.BOIDS_OPT_PROFILE, 2)  # level 2: the search class only
+        f.step(DT, 2)
+        prof = abi.boids_get_profile(f.h, reset=True)
+        assert prof["fused_or_search"][1] == 2 and prof["search_prep"][1] == 0
+
+
 def test_launch_count_and_info(pk):
     with pk.Flock(16384, seed=1) as f:
         i0 = f.info().launches
