@@ -51,6 +51,8 @@ def build(verbose: bool = False, force: bool = False) -> str:
     os.makedirs(objdir, exist_ok=True)
     objs = []
     extra = ["-Xptxas", "-v"] if verbose else []
+    if os.environ.get("BOIDS_CHECKS") == "1":  # device bounds checks (internal.h BOIDS_CHECK); test builds only
+        extra += ["-DBOIDS_CHECKS"]
     procs = []
     for src in sources():
         obj = os.path.join(objdir, os.path.basename(src) + ".o")

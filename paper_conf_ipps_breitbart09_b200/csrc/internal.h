@@ -1,5 +1,6 @@
 // internal.h -- private declarations shared by the CUDA translation units of libboids.
 #pragma once
+#include <cstdio>
 #include <utility>
 #include <cuda_runtime.h>
 #include <stdint.h>
@@ -33,9 +34,26 @@ struct SliceDiv {
   uint32_t mult;
   int32_t shift;  // l = ceil(log2 m) >= 8 (m is a multiple of 256)
   int32_t one;    // world == 1: every agent is in slice 0
+  int32_t world;  // slices (BOIDS_CHECKS builds bound agent indices by world x m)
 };
+
+// Device-side bounds checks of the checks build (build.py: BOIDS_CHECKS=1, used
+// in place of compute-sanitizer where the pool does not run it): a failed
+// check prints its place and traps, so the launch -- and the test -- fails.
+#if defined(BOIDS_CHECKS) && defined(__CUDA_ARCH__)
+#define BOIDS_CHECK(c)                                                         \
+  do {                                                                         \
+    if (!(c)) {                                                                \
+      printf("BOIDS_CHECK failed %s:%d: %s\n", __FILE__, __LINE__, #c);       \
+      __trap();                                                                \
+    }                                                                          \
+  } while (0)
+#else
+#define BOIDS_CHECK(c) ((void)0)
+#endif
 inline SliceDiv make_slice_div(int64_t m, int32_t world) {
   SliceDiv s{};
+  s.world = world;
   int l = 0;
   while ((1ull << l) < (unsigned long long)m) ++l;
   s.mult = (uint32_t)((((unsigned long long)1 << 32) * ((1ull << l) - (unsigned long long)m)) / (unsigned long long)m + 1);
@@ -54,9 +72,11 @@ __host__ __device__ inline int64_t slice_of(const SliceDiv& s, int64_t j) {
 #endif
 }
 __host__ __device__ inline const float4* pos_of(const float4* full, int64_t m, const SliceDiv& s, int64_t j) {
+  BOIDS_CHECK(j >= 0 && j < (int64_t)s.world * m);
   return full + j + slice_of(s, j) * m;
 }
 __host__ __device__ inline const float4* fwd_of(const float4* full, int64_t m, const SliceDiv& s, int64_t j) {
+  BOIDS_CHECK(j >= 0 && j < (int64_t)s.world * m);
   return full + j + (slice_of(s, j) + 1) * m;
 }
 
