@@ -625,9 +625,9 @@ int one_step(boids_ctx* c, float dt) {
       if ((rc = launch(c, 4, [&] { return launch_route(a, c->stream); }))) return rc;
     } else if (warm_path) {
       // warm step: all-pairs scan appending passing keys, then select + update;
-      // a single-GPU handle evaluates each unordered pair once (k_sym)
-      // (below 8192 agents the step is latency-bound and the ordered-pair path,
-      // with one launch less, is faster: measured C1/C2 55 vs 68 us)
+      // a single-GPU handle evaluates each unordered pair once (k_sym) from 8192
+      // agents on (below, k_small runs the whole step unless BOIDS_OPT_SMALL is
+      // off; then the ordered-pair path, one launch shorter, is the faster one)
       static const int64_t sym_min = [] {
         const char* e = getenv("BOIDS_SYM_MIN");  // diagnostics: smallest n on k_sym
         return e ? atoll(e) : 8192LL;
