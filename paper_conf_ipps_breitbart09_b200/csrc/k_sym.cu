@@ -593,43 +593,76 @@ constexpr int WIN = 256;  // C4: 64 -> 11 routed agents per step, 256 -> 3 (rout
 // The window over an explicit order: perm[0..n) agent indices (offset by base
 // into the position buffer) in Morton order of grid g, start[c] = the first
 // position of cell c; self = the querying agent's own index in perm's terms.
-__device__ float window_bound_in(const StepArgs& a, const int* __restrict__ perm, const int* __restrict__ start,
-                                 const BinGrid& g, int n, int64_t base, int64_t self, float4 me) {
-  if (!start || !perm || n < 8 || !(me.x == me.x && me.y == me.y && me.z == me.z))
-    return __int_as_float(0x7f800000);
-  const int p0 = __ldg(start + cell_of(me, g));
-  int lo = p0 - WIN / 2;
-  lo = lo > n - WIN ? n - WIN : lo;
-  lo = lo < 0 ? 0 : lo;
-  const int hi = lo + WIN < n ? lo + WIN : n;
-  float b[7];
+// The bound is computed by the whole warp for each lane that needs it
+// (`need`; every lane of the warp calls this): the WIN window agents are split
+// over the 32 lanes (WIN / 32 gathers each, all in flight at once), each lane
+// keeps its 7 smallest d2, and the 7th smallest of the warp comes from seven
+// warp-minimum extractions -- one gather round trip per needing agent instead
+// of WIN / 16 dependent rounds in one thread (round 2's serial version set
+// k_sym_prep's time: C4 46 us for a handful of agents).  Agents this handle
+// does not hold (NaN) are skipped, never counted.
+__device__ float window_bound_warp(const StepArgs& a, const int* __restrict__ perm, const int* __restrict__ start,
+                                   const BinGrid& g, int n, int64_t base, int64_t self, float4 me, bool need) {
+  const int lane = threadIdx.x & 31;
+  const float INF = __int_as_float(0x7f800000);
+  float out = INF;
+  unsigned todo = __ballot_sync(0xffffffffu, need);
+  while (todo) {
+    const int src = __ffs(todo) - 1;
+    todo &= todo - 1;
+    const float mx = __shfl_sync(0xffffffffu, me.x, src), my = __shfl_sync(0xffffffffu, me.y, src),
+                mz = __shfl_sync(0xffffffffu, me.z, src);
+    const long long sf = __shfl_sync(0xffffffffu, (long long)self, src);
+    if (!start || !perm || n < 8 || !(mx == mx && my == my && mz == mz)) continue;  // warp-uniform: +inf
+    const float4 m4 = make_float4(mx, my, mz, 0.f);
+    const int p0 = __ldg(start + cell_of(m4, g));
+    int lo = p0 - WIN / 2;
+    lo = lo > n - WIN ? n - WIN : lo;
+    lo = lo < 0 ? 0 : lo;
+    const int hi = lo + WIN < n ? lo + WIN : n;
+    constexpr int PER = WIN / 32;
+    int j[PER];
 #pragma unroll
-  for (int k = 0; k < 7; ++k) b[k] = __int_as_float(0x7f800000);
-  constexpr int G = 16;  // loads in flight: the agents that take this path are scattered
-  for (int p0 = lo; p0 < hi; p0 += G) {
-    int j[G];
+    for (int k = 0; k < PER; ++k) {
+      const int pos = lo + k * 32 + lane;
+      j[k] = pos < hi ? __ldg(perm + pos) : -1;
+    }
+    float4 q[PER];
 #pragma unroll
-    for (int k = 0; k < G; ++k) j[k] = p0 + k < hi ? __ldg(perm + p0 + k) : -1;
-    float4 q[G];
+    for (int k = 0; k < PER; ++k) q[k] = __ldg(pos_of(a.full, a.m, a.sdiv, base + (j[k] < 0 ? 0 : j[k])));
+    float b[7];
 #pragma unroll
-    for (int k = 0; k < G; ++k) q[k] = __ldg(pos_of(a.full, a.m, a.sdiv, base + (j[k] < 0 ? 0 : j[k])));
+    for (int t = 0; t < 7; ++t) b[t] = INF;
 #pragma unroll
-    for (int k = 0; k < G; ++k) {
-      if (j[k] < 0 || j[k] == self) continue;
-      float d = dist2(me.x, me.y, me.z, q[k]);
+    for (int k = 0; k < PER; ++k) {
+      if (j[k] < 0 || j[k] == sf) continue;
+      float d = dist2(mx, my, mz, q[k]);
+      if (!(d == d)) continue;  // an agent this handle does not hold
 #pragma unroll
       for (int t = 0; t < 7; ++t) {  // keep the 7 smallest, ascending
-        const float lo_ = fminf(b[t], d);
+        const float l = fminf(b[t], d);
         d = fmaxf(b[t], d);
-        b[t] = lo_;
+        b[t] = l;
       }
     }
+    // 7 extractions of the warp minimum (d2 >= 0: its bits order like the value;
+    // ties broken by lane, so exactly one lane pops per round)
+    float kth = INF;
+#pragma unroll 1
+    for (int t = 0; t < 7; ++t) {
+      const unsigned hb = __float_as_uint(b[0]);
+      const unsigned mb = __reduce_min_sync(0xffffffffu, hb);
+      kth = __uint_as_float(mb);
+      const unsigned who = __reduce_min_sync(0xffffffffu, hb == mb ? (unsigned)lane : 32u);
+      if (lane == (int)who) {
+#pragma unroll
+        for (int s2 = 0; s2 < 6; ++s2) b[s2] = b[s2 + 1];
+        b[6] = INF;
+      }
+    }
+    if (lane == src) out = kth;
   }
-  return b[6];
-}
-
-__device__ float window_bound(const StepArgs& a, int qi, float4 me) {
-  return window_bound_in(a, a.qperm, a.lstart, a.loc, (int)a.nloc, a.lo, qi, me);
+  return out;
 }
 
 // Structure of arrays over the sorted positions p: spf[p], spf[cap + p], spf[2 cap + p] = x, y, z and
@@ -641,25 +674,20 @@ __device__ float window_bound(const StepArgs& a, int qi, float4 me) {
 __device__ __forceinline__ void sym_prep_body(const StepArgs& a, float* __restrict__ spf, int64_t cap,
                                               int* __restrict__ sidx, int64_t npad) {
   const int64_t p = (int64_t)blockIdx.x * 256 + threadIdx.x;
-  if (p >= npad) return;
-  if (p >= a.nloc) {
-    const float nan = __int_as_float(0x7fc00000);
-    spf[p] = nan;
-    spf[cap + p] = nan;
-    spf[2 * cap + p] = nan;
-    spf[3 * cap + p] = -1.f;
-    sidx[p] = -1;
-    return;
-  }
-  const int qi = a.qperm ? __ldg(a.qperm + p) : (int)p;
+  if (p >= npad) return;  // (npad is a multiple of 256: whole warps)
+  const bool real = p < a.nloc;  // else a phantom slot: NaN position, limit -1
+  const int qi = real ? (a.qperm ? __ldg(a.qperm + p) : (int)p) : 0;
   const float r2 = __fmul_rn(a.p.search_radius, a.p.search_radius);
   const float r2_in = __uint_as_float(__float_as_uint(r2) - 1u);  // d2 < r2  <=>  d2 <= r2_in
-  const float4 me = __ldg(pos_of(a.full, a.m, a.sdiv, a.lo + qi));
+  const float nan = __int_as_float(0x7fc00000);
+  const float4 me = real ? __ldg(pos_of(a.full, a.m, a.sdiv, a.lo + qi)) : make_float4(nan, nan, nan, 0.f);
   int c = 0;
-  const float t0 = sym_t0(a, qi, me, c);
+  const float t0 = real ? sym_t0(a, qi, me, c) : 0.f;
   float lim = fminf(r2_in, t0);
-  if (t0 > r2_in) lim = fminf(lim, window_bound(a, qi, me));
-  if (c == 7 && lim > r2_in && a.rlist) {
+  // every lane of the warp takes part in the warp's window bounds
+  const float wb = window_bound_warp(a, a.qperm, a.lstart, a.loc, (int)a.nloc, a.lo, qi, me, real && t0 > r2_in);
+  if (real && t0 > r2_in) lim = fminf(lim, wb);
+  if (real && c == 7 && lim > r2_in && a.rlist) {
     a.rlist[atomicAdd(a.rcount, 1)] = qi;
     a.routed[qi] = 1;
     if (a.stats) atomicAdd(a.stats + 2, 1ull);
@@ -668,8 +696,8 @@ __device__ __forceinline__ void sym_prep_body(const StepArgs& a, float* __restri
   spf[p] = me.x;
   spf[cap + p] = me.y;
   spf[2 * cap + p] = me.z;
-  spf[3 * cap + p] = lim;
-  sidx[p] = qi;
+  spf[3 * cap + p] = real ? lim : -1.f;
+  sidx[p] = real ? qi : -1;
 }
 
 __global__ void __launch_bounds__(256) k_sym_prep(StepArgs a, float* __restrict__ spf, int64_t cap,
@@ -890,28 +918,26 @@ cudaError_t sym_with(const StepArgs& a, float4* sp, int* sidx, const long long* 
 __global__ void __launch_bounds__(256) k_ss_lim(StepArgs a, float* __restrict__ lim_send, const int* __restrict__ gperm,
                                                 const int* __restrict__ gstart, int nsorted) {
   const int64_t i = (int64_t)blockIdx.x * 256 + threadIdx.x;
-  if (i >= a.m) return;
-  if (i >= a.nloc) {
-    lim_send[i] = -1.f;
-    return;
-  }
+  const bool real = i < a.nloc;  // (threads up to the block's end take part in the warp's window bounds)
   const float r2 = __fmul_rn(a.p.search_radius, a.p.search_radius);
   const float r2_in = __uint_as_float(__float_as_uint(r2) - 1u);
-  const float4 me = __ldg(pos_of(a.full, a.m, a.sdiv, a.lo + i));
+  const float nan = __int_as_float(0x7fc00000);
+  const float4 me = real ? __ldg(pos_of(a.full, a.m, a.sdiv, a.lo + i)) : make_float4(nan, nan, nan, 0.f);
   int c = 0;
-  const float t0 = sym_t0(a, i, me, c);
+  const float t0 = real ? sym_t0(a, i, me, c) : 0.f;
   float lim = fminf(r2_in, t0);
   // the window over the GLOBAL Morton order (every rank's agents): over this
   // rank's own 1/G of them the 7th nearest lies ~G^(1/3) times farther and many
   // more agents stayed unbounded (C4, 8 ranks: ~45 routed per rank vs ~36 in all)
-  if (t0 > r2_in) lim = fminf(lim, window_bound_in(a, gperm, gstart, a.loc, nsorted, 0, a.lo + i, me));
-  if (c == 7 && lim > r2_in && a.rlist) {  // unbounded (a wrap): k_route searches it whole
+  const float wb = window_bound_warp(a, gperm, gstart, a.loc, nsorted, 0, a.lo + i, me, real && t0 > r2_in);
+  if (real && t0 > r2_in) lim = fminf(lim, wb);
+  if (real && c == 7 && lim > r2_in && a.rlist) {  // unbounded (a wrap): k_route searches it whole
     a.rlist[atomicAdd(a.rcount, 1)] = (int)i;
     a.routed[i] = 1;
     if (a.stats) atomicAdd(a.stats + 2, 1ull);
     lim = -1.f;
   }
-  lim_send[i] = lim;
+  if (i < a.m) lim_send[i] = real ? lim : -1.f;
 }
 
 // The binning's order inside a cell follows its atomics: sort every cell's
